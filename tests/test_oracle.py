@@ -1,0 +1,291 @@
+"""Pins for the CPU oracle (oracle/oracle.c) against things other than itself.
+
+Each test names what fixes the oracle: a library routine (LAPACK dgesv, triangular
+solves), the matrix form of the splitting, exact rational arithmetic,
+closed forms / published constants, and the paper's printed tables (soft pins).
+A plausible mistake (dropped term, wrong sign/index, transposed operand, wrong
+subdomain boundary, in-place instead of double-buffered sweep) fails at least one.
+"""
+from fractions import Fraction
+
+import numpy as np
+import pytest
+import scipy.linalg as sla
+
+import oracle as O
+import workloads as W
+
+
+def _dense(A):
+    return A.to_dense()
+
+
+# ----------------------------------------------------------------- O4 residual
+def test_residual_matches_numpy(rng):
+    A = W.random_dd(80, 6, seed=3)
+    x = rng.standard_normal(80)
+    b = rng.standard_normal(80)
+    ref = np.linalg.norm(b - _dense(A) @ x)
+    assert abs(O.residual_norm(A, b, x) - ref) <= 1e-13 * ref
+
+
+# ----------------------------------------------------- matrix-form brute force
+def _jacobi_matrix_form(Ad, b, x):
+    """x^{k+1} = D^-1 (b - (L+U) x^k)  (matrix form; the oracle uses eq. 2)."""
+    D = np.diag(np.diag(Ad))
+    LU = Ad - D
+    return np.linalg.solve(D, b - LU @ x)
+
+
+def _block_jacobi_matrix_form(Ad, b, x, R, k):
+    """sb-(k): M = block-diagonal part (row//R == col//R), N = A - M; s = b - N x,
+    y^{t+1} = D^-1 (s - (M - D) y^t), y^0 = x (Alg. 1 in splitting form)."""
+    n = Ad.shape[0]
+    blk = np.arange(n) // R
+    Mask = blk[:, None] == blk[None, :]
+    M = np.where(Mask, Ad, 0.0)
+    N = Ad - M
+    D = np.diag(np.diag(Ad))
+    s = b - N @ x
+    y = x.copy()
+    for _ in range(k):
+        y = np.linalg.solve(D, s - (M - D) @ y)
+    return y
+
+
+def _gauss_seidel_matrix_form(Ad, b, x):
+    """(D + L) x^{new} = b - U x^{old} (forward G-S), via a triangular solve."""
+    U = np.triu(Ad, 1)
+    return sla.solve_triangular(np.tril(Ad), b - U @ x, lower=True)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_steps_match_matrix_forms(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(5, 70))
+    A = W.random_dd(n, 5, seed=seed, symmetric_pattern=bool(seed % 2))
+    Ad = _dense(A)
+    b = rng.standard_normal(n)
+    x = rng.standard_normal(n)
+    tol = 1e-12 * (1 + np.abs(x).max())
+    np.testing.assert_allclose(O.jacobi_step(A, b, x), _jacobi_matrix_form(Ad, b, x), rtol=0, atol=tol)
+    np.testing.assert_allclose(O.gauss_seidel_step(A, b, x), _gauss_seidel_matrix_form(Ad, b, x), rtol=0, atol=tol)
+    for R in (1, 3, 7, 16, n, n + 5):
+        for k in (1, 2, 5):
+            np.testing.assert_allclose(O.block_jacobi_step(A, b, x, R, k), _block_jacobi_matrix_form(Ad, b, x, R, k),
+                                       rtol=0, atol=tol)
+
+
+# -------------------------------------------------------------- dense LU (P6)
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("method,R,k", [(O.JACOBI, 1, 1), (O.BLOCK_JACOBI, 8, 5), (O.BLOCK_JACOBI, 3, 2),
+                                        (O.GAUSS_SEIDEL, 1, 1)])
+def test_solve_converges_to_dgesv(seed, method, R, k):
+    """Every mode converges to the dense LU solution when rho(|B|) < 1."""
+    A = W.random_dd(90, 5, seed=seed, dominance=1.3)
+    b = np.random.default_rng(seed + 100).standard_normal(A.n)
+    xs = np.linalg.solve(_dense(A), b)
+    r = O.solve(A, b, method=method, R=R, k=k, tol=1e-13, max_iters=5000)
+    assert r.converged and r.rel_res <= 1e-13
+    assert np.abs(r.x - xs).max() <= 1e-11 * np.abs(xs).max()
+
+
+# --------------------------------------------------------- fixed point (P7)
+@pytest.mark.parametrize("method,R,k", [(O.JACOBI, 1, 1), (O.BLOCK_JACOBI, 128, 5), (O.GAUSS_SEIDEL, 1, 1)])
+def test_fixed_point_invariant(method, R, k):
+    """x* = D^-1 (b - (L+U) x*): starting at x* the iterates stay there."""
+    A = W.trefethen(500)
+    b = np.ones(A.n)
+    xs = np.linalg.solve(_dense(A), b)
+    r = O.solve(A, b, xs, method=method, R=R, k=k, tol=0.0, max_iters=10)
+    assert r.iters == 10 and not r.converged
+    assert np.abs(r.x - xs).max() <= 1e-14 * np.abs(xs).max() * 10
+
+
+# ------------------------------------------------- special cases (P8)
+def test_R1_is_jacobi_bitwise():
+    A = W.trefethen(300)
+    x = np.random.default_rng(1).standard_normal(300)
+    b = np.ones(300)
+    for k in (1, 3, 7):
+        assert np.array_equal(O.block_jacobi_step(A, b, x, 1, k), O.jacobi_step(A, b, x))
+
+
+def test_R_ge_n_is_k_jacobi_bitwise():
+    A = W.random_dd(50, 5, seed=9)
+    x = np.random.default_rng(2).standard_normal(50)
+    b = np.random.default_rng(3).standard_normal(50)
+    y = x
+    for _ in range(4):
+        y = O.jacobi_step(A, b, y)
+    assert np.array_equal(O.block_jacobi_step(A, b, x, 50, 4), y)
+    assert np.array_equal(O.block_jacobi_step(A, b, x, 1000, 4), y)
+
+
+def test_k1_equals_jacobi():
+    A = W.stencil9_2d(20)
+    x = np.random.default_rng(4).standard_normal(A.n)
+    b = np.ones(A.n)
+    np.testing.assert_allclose(O.block_jacobi_step(A, b, x, 32, 1), O.jacobi_step(A, b, x), rtol=1e-15, atol=1e-15)
+
+
+def test_k_infinity_is_exact_local_solve():
+    """k -> inf: each subdomain solves A_JJ y = b_J - A_{J,notJ} x exactly."""
+    A = W.trefethen(256)
+    Ad = _dense(A)
+    x = np.random.default_rng(5).standard_normal(256)
+    b = np.ones(256)
+    R = 64
+    y = O.block_jacobi_step(A, b, x, R, 400)
+    for l in range(4):
+        J = slice(l * R, (l + 1) * R)
+        s = b[J] - Ad[J, :] @ x + Ad[J, J] @ x[J]
+        np.testing.assert_allclose(y[J], np.linalg.solve(Ad[J, J], s), rtol=1e-12, atol=1e-14)
+
+
+def test_diagonal_matrix_exact_in_one_step():
+    n = 40
+    d = np.arange(1, n + 1, dtype=float) * 1.5
+    A = W.CSR(n, np.arange(n + 1, dtype=np.int32), np.arange(n, dtype=np.int32), d)
+    b = np.random.default_rng(6).standard_normal(n)
+    for method in (O.JACOBI, O.BLOCK_JACOBI, O.GAUSS_SEIDEL):
+        r = O.solve(A, b, method=method, R=7, k=3, tol=1e-15)
+        assert r.iters == 1 and np.array_equal(r.x, b / d)
+
+
+def test_subdomain_matches_full_step():
+    A = W.stencil7_3d(8)
+    b = np.ones(A.n)
+    x = np.random.default_rng(7).standard_normal(A.n)
+    full = O.block_jacobi_step(A, b, x, 64, 5)
+    for l in (0, 3, 7):
+        rows = W.stencil7_3d(8, row_lo=l * 64, row_hi=(l + 1) * 64)
+        assert np.array_equal(O.block_jacobi_subdomain(rows, b[l * 64:(l + 1) * 64], x, 5), full[l * 64:(l + 1) * 64])
+    rows = W.stencil7_3d(8, row_lo=100, row_hi=180)
+    assert np.array_equal(O.jacobi_rows(rows, b[100:180], x), O.jacobi_step(A, b, x)[100:180])
+
+
+# --------------------------------------------------------- exact dyadic (P9)
+def _exact_block_jacobi(Ad, b, x, R, k):
+    n = len(b)
+    out = [None] * n
+    for TS in range(0, n, R):
+        TE = min(n, TS + R)
+        s = [Fraction(b[i]) - sum(Fraction(Ad[i, j]) * x[j] for j in range(n) if not TS <= j < TE and Ad[i, j] != 0)
+             for i in range(TS, TE)]
+        y = [x[i] for i in range(TS, TE)]
+        for _ in range(k):
+            y = [(s[i - TS] - sum(Fraction(Ad[i, j]) * y[j - TS] for j in range(TS, TE) if j != i and Ad[i, j] != 0))
+                 / Fraction(Ad[i, i]) for i in range(TS, TE)]
+        out[TS:TE] = y
+    return out
+
+
+def test_dyadic_bitwise_exact():
+    """Diagonal 2^p, off-diagonals -1, integer b: iterates are exact dyadic rationals
+    (SURVEY.md §8(c) P9), so the fp64 oracle must equal exact rational arithmetic."""
+    A = W.dyadic_stencil9_2d(6, p=4)
+    Ad = _dense(A)
+    b = np.arange(A.n, dtype=float) % 5 - 2
+    xf = np.zeros(A.n)
+    xq = [Fraction(0)] * A.n
+    for _ in range(4):
+        xf = O.block_jacobi_step(A, b, xf, 8, 3)
+        xq = _exact_block_jacobi(Ad, b, xq, 8, 3)
+        assert [Fraction(v) for v in xf] == xq
+
+
+# ----------------------------------------------- external constant (P2)
+def test_siam_trefethen20000_a11(golden):
+    """(A^-1)_11 of Trefethen_20000 = 0.725078346268401167... (SIAM 100-digit, problem 7)."""
+    ref = float(golden("siam_trefethen20000_a11.txt")[0][0])
+    A = W.trefethen(20000)
+    b = np.zeros(A.n)
+    b[0] = 1.0
+    r = O.solve(A, b, method=O.BLOCK_JACOBI, R=128, k=5, tol=1e-13, max_iters=200)
+    assert r.converged
+    assert abs(r.x[0] - ref) < 1e-12
+
+
+# ------------------------------------------------ paper tables (soft pins)
+def test_table2_fv1_history_softpin(golden):
+    """fv1-shaped, R=128, b=1, x0=0: sync-block-(5) vs Table 2's async-(5) averages,
+    ratio within [0.7, 1.3] up to 130 global iterations."""
+    A = W.stencil9_2d(98)
+    r = O.solve(A, np.ones(A.n), method=O.BLOCK_JACOBI, R=128, k=5, tol=0.0, max_iters=130)
+    for it, avg, *_ in golden("table2_fv1.txt"):
+        it = int(it)
+        if it <= 130:
+            ratio = r.history[it] / float(avg)
+            assert 0.7 <= ratio <= 1.3, (it, ratio)
+
+
+def test_table3_trefethen_iterations_softpin(golden):
+    """Trefethen_2000, R=128, b=1: the paper's async-(5) reaches ~1e-10 at ~22 iterations
+    (Table 3); sync-block-(5) must land in the envelope [15, 35] (P5)."""
+    tab = {int(r[0]): float(r[1]) for r in golden("table3_trefethen2000.txt")}
+    assert tab[20] > 1e-10 > tab[25]
+    A = W.trefethen(2000)
+    r = O.solve(A, np.ones(A.n), method=O.BLOCK_JACOBI, R=128, k=5, tol=1e-10)
+    assert 15 <= r.iters <= 35
+
+
+def test_asymptotic_rate_is_rho(golden):
+    """P10: ||r_{m+1}||/||r_m|| -> rho(B) = 0.8601 (Table 1) under Jacobi."""
+    rho = {r[0]: float(r[5]) for r in golden("table1.txt")}["Trefethen_2000"]
+    A = W.trefethen(2000)
+    r = O.solve(A, np.ones(A.n), method=O.JACOBI, tol=0.0, max_iters=130)
+    rate = r.history[121:131] / r.history[120:130]
+    assert np.all(np.abs(rate - rho) < 0.01 * rho)
+
+
+def test_local_sweep_rate_is_rho_pow_k():
+    """[S7]: on Trefethen the sb-(k) per-iteration rate is ~rho(B)^k."""
+    A = W.trefethen(2000)
+    for k in (2, 5):
+        r = O.solve(A, np.ones(A.n), method=O.BLOCK_JACOBI, R=128, k=k, tol=0.0, max_iters=14)
+        rate = (r.history[14] / r.history[10]) ** 0.25
+        assert abs(rate - 0.8601 ** k) < 0.03
+
+
+# ------------------------------------------------ expected counts (P12)
+@pytest.mark.parametrize("gen,method,R,k,expect", [
+    ("tref2000", O.JACOBI, 128, 1, 137), ("tref2000", O.BLOCK_JACOBI, 128, 2, 68),
+    ("tref2000", O.BLOCK_JACOBI, 128, 5, 28), ("tref2000", O.BLOCK_JACOBI, 128, 9, 16),
+    ("tref2000", O.GAUSS_SEIDEL, 1, 1, 14),
+    ("fv1", O.JACOBI, 128, 1, 146), ("fv1", O.BLOCK_JACOBI, 128, 5, 92), ("fv1", O.BLOCK_JACOBI, 448, 5, 48),
+    ("fv1", O.GAUSS_SEIDEL, 1, 1, 78),
+])
+def test_iteration_counts(gen, method, R, k, expect):
+    """Iterations to rel_res <= 1e-10 (b=1, x0=0), from the survey's independent numpy
+    implementation [S2]."""
+    A = W.trefethen(2000) if gen == "tref2000" else W.stencil9_2d(98)
+    r = O.solve(A, np.ones(A.n), method=method, R=R, k=k, tol=1e-10)
+    assert r.converged and r.iters == expect
+
+
+# ------------------------------------------------ divergence (P11)
+def test_divergence_rho_gt_1():
+    """SPD with rho(B) = 1.8 > 1: Jacobi diverges (P:697 s1rmt3m1 analogue)."""
+    Ad = np.full((3, 3), 0.9) + 0.1 * np.eye(3)
+    rp = np.array([0, 3, 6, 9], dtype=np.int32)
+    A = W.CSR(3, rp, np.tile(np.arange(3, dtype=np.int32), 3), Ad.ravel())
+    assert abs(np.abs(np.linalg.eigvals(np.eye(3) - Ad)).max() - 1.8) < 1e-12
+    r = O.solve(A, np.ones(3), method=O.JACOBI, tol=1e-10, max_iters=10000)
+    assert r.status == O.DIVERGED and not r.converged
+
+
+def test_zero_rhs_and_initial_convergence():
+    A = W.trefethen(100)
+    r = O.solve(A, np.zeros(100), np.ones(100))
+    assert r.iters == 0 and r.converged and np.all(r.x == 0)
+    xs = np.linalg.solve(_dense(A), np.ones(100))
+    r = O.solve(A, np.ones(100), xs, tol=1e-10)
+    assert r.iters == 0 and r.converged
+
+
+def test_max_iters_not_converged():
+    A = W.trefethen(2000)
+    r = O.solve(A, np.ones(2000), method=O.JACOBI, tol=1e-10, max_iters=20)
+    assert r.iters == 20 and not r.converged and r.rel_res > 1e-10
+    assert abs(r.rel_res - O.rel_res(A, np.ones(2000), r.x)) == 0
