@@ -1,0 +1,340 @@
+"""bench.py — time to relative residual 1e-10 for async-(k) through libbar.so on B200.
+
+One "step" = one full bar_solve (every §8(a) row: staging, off-block part, k local sweeps,
+fused residual, write-back, convergence control) of A x = b from x0 = 0, b = 1 (DESIGN.md
+reading R1), inputs already resident in HBM. Prints ONE JSON line (rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c5] [--mode async] [--k 5] [--R 4096]
+    python bench.py --impl reference ...   # the CPU oracle, timed on this box's host cores
+
+The default workload is configs[4] (C5: 3D 7-point, n = 512^3 = 134,217,728, 937,951,232 nnz),
+the configuration BASELINE.json's 1/2/4/8-GPU metric is quoted on; it fits one B200.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (description, generator kwargs, default R)
+    "c1": ("Trefethen_2000 (exact)", ("trefethen", 2000), 128),
+    "c2": ("fv1-shaped 9-point 98x98, diag 9.3595", ("stencil9", 98), 128),
+    "c3": ("Trefethen_20000 (exact)", ("trefethen", 20000), 128),
+    "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 4096),
+    "c5": ("3D 7-point 512^3, diag 7.0249 (n=128M)", ("stencil7", 512), 4096),
+}
+METRIC = "time to rel. residual 1e-10 (s) and global iters/s with HBM GB/s vs peak, 1/2/4/8 GPU"
+
+
+def make_matrix(workload: str, row_lo: int = 0, row_hi: int | None = None):
+    import workloads as W
+
+    kind, size = WORKLOADS[workload][1]
+    if kind == "trefethen":
+        return W.trefethen(size, row_lo, row_hi)
+    if kind == "stencil9":
+        return W.stencil9_2d(size, W.FV1_DIAG, -1.0, row_lo, row_hi)
+    return W.stencil7_3d(size, W.S7_DIAG, -1.0, row_lo, row_hi)
+
+
+def matrix_dims(workload: str):
+    kind, size = WORKLOADS[workload][1]
+    if kind == "trefethen":
+        n = size
+        nnz = n + 2 * sum(n - (1 << t) for t in range(64) if (1 << t) < n)
+    elif kind == "stencil9":
+        n, nnz = size * size, (3 * size - 2) ** 2
+    else:
+        n, nnz = size ** 3, 7 * size ** 3 - 6 * size ** 2
+    return n, nnz
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """Samples SM clocks and throttle reasons via NVML during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv is not None:
+            self.t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def cpu_info():
+    cores = len(os.sched_getaffinity(0))
+    model = ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return cores, model
+
+
+def oracle_sample(workload: str, k: int, R: int, mode: str, budget_rows: int):
+    """Time ONE global iteration of the oracle on a bounded row sample of the workload.
+
+    The oracle has no asynchronous mode (async is nondeterministic, oracle/__init__.py);
+    async-(k) and sync-block-(k) do identical work per global iteration, so the oracle's
+    sync-block-(k) (Jacobi for mode=jacobi) is timed. Returns (seconds per full global
+    iteration extrapolated linearly in rows, sample description)."""
+    import oracle as O
+
+    n, _ = matrix_dims(workload)
+    rows = min(n, max(R, (budget_rows // R) * R))
+    A = make_matrix(workload, 0, rows)
+    b = np.ones(rows)
+    x = np.zeros(n)
+    x[:] = 0.5
+    t0 = time.perf_counter()
+    if mode == "jacobi":
+        O.jacobi_rows(A, b, x)
+    else:
+        nsub = 0
+        for TS in range(0, rows, R):
+            TE = min(rows, TS + R)
+            s, e = A.rowptr[TS], A.rowptr[TE]
+            sub = type(A)(n, A.rowptr[TS:TE + 1] - s, A.col[s:e], A.val[s:e], TS, TE)
+            O.block_jacobi_subdomain(sub, b[TS:TE], x, k)
+            nsub += 1
+    dt = time.perf_counter() - t0
+    scale = n / rows
+    desc = (f"1 global iteration of oracle {'jacobi' if mode == 'jacobi' else f'sync-block-({k})'} over rows "
+            f"[0,{rows}) of {n} (1 core), x{scale:.2f} to the full matrix, x the GPU's global-iteration count")
+    return dt * scale, desc
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on this box's host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n, nnz = matrix_dims(args.workload)
+    cores, model = cpu_info()
+    iters = args.ref_iters or {"c1": 28, "c2": 92, "c3": 26, "c4": 113, "c5": 79}[args.workload]
+    budget = args.ref_rows
+    for _ in range(args.warmup):
+        oracle_sample(args.workload, args.k, args.R, args.mode, budget // 4)
+    times = []
+    desc = ""
+    for _ in range(args.steps):
+        s_per_iter, desc = oracle_sample(args.workload, args.k, args.R, args.mode, budget)
+        times.append(s_per_iter * iters)
+    value = statistics.median(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": value * 1e3, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload][0]}", "n": n, "nnz": nnz,
+                       "mode": args.mode, "k": args.k, "rows_per_block": args.R, "tol": 1e-10},
+            "cpu_baseline": {"value": value, "unit": "s", "cores": 1, "kind": "oracle",
+                             "sample": desc + f" ({iters} iterations)", "cpu": model, "host_cores": cores},
+            "e2e": {"value": value, "unit": "s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="c5", choices=sorted(WORKLOADS))
+    ap.add_argument("--mode", default="async", choices=["async", "sync-block", "jacobi"])
+    ap.add_argument("--k", type=int, default=5)
+    ap.add_argument("--R", type=int, default=None)
+    ap.add_argument("--tol", type=float, default=1e-10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-rows", type=int, default=4_000_000, help="oracle row sample per step")
+    ap.add_argument("--ref-iters", type=int, default=0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.R is None:
+        args.R = WORKLOADS[args.workload][2]
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        raise SystemExit("multi-GPU bench: not built yet (DESIGN.md §Multi-GPU)")
+    torch.cuda.set_device(local_rank)
+    from paper_conf_ipps_anzttdh12_b200 import bar
+
+    dev = torch.device("cuda", local_rank)
+    n, nnz = matrix_dims(args.workload)
+    t0 = time.time()
+    A = make_matrix(args.workload)
+    t_gen = time.time() - t0
+    t0 = time.time()
+    M = bar.Matrix.from_csr(A, rows_per_block=args.R, device=local_rank)
+    t_setup = time.time() - t0
+    del A
+    minfo = M.info()
+    model_bytes = minfo["model_bytes_per_iter"]
+    stream = torch.cuda.current_stream(dev)
+    b = torch.ones(n, dtype=torch.float64, device=dev)
+    x = torch.empty(n, dtype=torch.float64, device=dev)
+
+    def step():
+        _, info = M.solve(b, None, x, k=args.k, max_global_iters=20000, tol=args.tol, mode=args.mode, stream=stream)
+        return info
+
+    for _ in range(args.warmup):
+        info = step()
+    torch.cuda.synchronize(dev)
+    infos = []
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        torch.cuda.synchronize(dev)
+        ev0.record(stream)
+        for _ in range(args.steps):
+            infos.append(step())
+        ev1.record(stream)
+        torch.cuda.synchronize(dev)
+    ms_total = ev0.elapsed_time(ev1)
+    ms_per_step = ms_total / args.steps
+    iters = [i["iters"] for i in infos]
+    launches = sum(i["kernel_launches"] for i in infos)
+    assert all(i["converged"] for i in infos), infos
+    mean_iters = sum(iters) / len(iters)
+
+    # dominant kernel: per-launch duration of the sweep kernel, by the slope of back-to-back
+    # launch batches timed with CUDA events on the launching stream (cancels fixed overheads)
+    xs = torch.zeros(n, dtype=torch.float64, device=dev)
+
+    def timed_sweeps(nsw):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        M.sweep(b, xs, k=args.k, nsweeps=nsw, mode=args.mode, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        return e0.elapsed_time(e1)
+
+    timed_sweeps(4)
+    lo, hi = 8, 40
+    t_lo = min(timed_sweeps(lo) for _ in range(3))
+    t_hi = min(timed_sweeps(hi) for _ in range(3))
+    kernel_ms = (t_hi - t_lo) / (hi - lo)
+    peak, peak_src = load_peaks()
+    achieved = model_bytes / (kernel_ms * 1e-3) / 1e9
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": None, "kernel": f"k_block<{args.mode}>"
+                if args.mode != "jacobi" else "k_rowwise<jacobi>", "kernel_ms": round(kernel_ms, 5),
+                "algorithmic_bytes_per_launch": model_bytes, "peak_source": peak_src}
+    prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")
+    if os.path.exists(prof):
+        try:
+            roofline["traffic"] = json.load(open(prof))["dram_bytes_per_launch"]
+        except Exception:
+            pass
+
+    # end-to-end through the public API with HOST (pinned) buffers: H2D of b and x0, D2H of x
+    e2e = None
+    if not args.no_e2e:
+        bh = torch.ones(n, dtype=torch.float64).pin_memory()
+        x0h = torch.zeros(n, dtype=torch.float64).pin_memory()
+        xh = torch.empty(n, dtype=torch.float64).pin_memory()
+        M.solve(bh, x0h, xh, k=args.k, tol=args.tol, mode=args.mode, stream=stream)
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            _, ie = M.solve(bh, x0h, xh, k=args.k, tol=args.tol, mode=args.mode, stream=stream)
+            assert ie["converged"]
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        e2e_s = e0.elapsed_time(e1) / 1e3 / args.steps
+        e2e = {"value": e2e_s, "unit": "s", "h2d_bytes_per_step": 2 * 8 * n, "d2h_bytes_per_step": 8 * n,
+               "wall_s": (time.perf_counter() - t0) / args.steps}
+
+    cpu = None
+    if not args.no_cpu_baseline and rank == 0:
+        cores, model = cpu_info()
+        s_iter, desc = oracle_sample(args.workload, args.k, args.R, args.mode,
+                                     min(n, 4_000_000 if n > 4_000_000 else n))
+        cpu = {"value": s_iter * mean_iters, "unit": "s", "cores": 1, "kind": "oracle",
+               "sample": desc + f" ({mean_iters:g})", "cpu": model, "host_cores": cores,
+               "s_per_global_iter": s_iter}
+
+    value = ms_per_step / 1e3
+    line = {
+        "metric": METRIC, "value": value, "unit": "s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload][0]}", "n": n, "nnz": nnz,
+                   "mode": args.mode, "k": args.k, "rows_per_block": args.R, "tol": args.tol, "b": "ones",
+                   "x0": "zeros", "parallelism": f"rows/{world}", "l2": "inputs > L2 (no flush needed)"
+                   if model_bytes > 126e6 else "inputs L2-resident (latency-bound config)"},
+        "global_iters": mean_iters, "global_iters_minmax": [min(iters), max(iters)],
+        "global_iters_per_s": mean_iters / value, "hbm_gbs_contract": model_bytes * mean_iters / value / 1e9,
+        "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+        "clocks": clk.summary(), "setup_s": {"generate": round(t_gen, 2), "bar_create_csr": round(t_setup, 2)},
+        "layout": minfo,
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

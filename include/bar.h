@@ -1,0 +1,158 @@
+/*
+ * bar.h — C ABI of libbar.so: block-asynchronous relaxation async-(k) for A x = b on B200.
+ *
+ * The method is H. Anzt, S. Tomov, J. Dongarra, V. Heuveline, "A Block-Asynchronous
+ * Relaxation Method for Graphics Processing Units" (/root/reference/PAPER.md; cited
+ * as P:<line> with the section / equation / algorithm it falls in):
+ *   - Jacobi, eq. 2 (§2.1):  x_i^{m+1} = (b_i - sum_{j!=i} a_ij x_j^m) / a_ii
+ *   - async-(k), Algorithm 1 (§3.3) and eq. 4: rows are split into
+ *     subdomains J_l of R consecutive rows, one per thread block; each block reads x "as it
+ *     stands" in global memory, computes the off-block part s_i = b_i - sum_{j notin J_l} a_ij x_j
+ *     once, runs k local Jacobi sweeps on its own components with the off-block values frozen
+ *     (P:147), and writes x_J back, with no synchronisation between blocks (eq. 3).
+ *   - sync-block-(k): the same two-stage sweep with every block reading the same x^(m)
+ *     (deterministic block-Jacobi; reading R3), the parity mode.
+ *   - the l2 residual ||b - A x||_2, fused into every sweep.
+ *
+ * No torch types cross this boundary: plain pointers and sizes only.
+ *
+ * Pointers. Matrix arrays given to bar_create_csr may be host or device memory (detected
+ * with cudaPointerGetAttributes) and are COPIED into a library-owned layout; the caller keeps
+ * ownership. b, x0, x given to bar_solve / bar_residual may be device memory on the matrix's
+ * device (the fast path) or host memory (then the library stages them through device
+ * buffers inside the call — the end-to-end path). The caller must not free them during a call.
+ *
+ * Streams. Every call is ordered on `cuda_stream` (a cudaStream_t; NULL = legacy default
+ * stream) and returns only after its work on that stream is complete (it has to fill `info`).
+ *
+ * Errors. Every entry point returns a bar_status and never aborts or exits. The text of the
+ * last error on the calling thread is available from bar_last_error(). Not converging within
+ * max_global_iters is NOT an error (BAR_OK with info.converged = 0).
+ *
+ * Threads. A bar_matrix may be used by one thread at a time (its workspace is reused).
+ */
+#ifndef BAR_H
+#define BAR_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bar_matrix_s *bar_matrix; /* opaque, library-owned */
+
+typedef enum {
+    BAR_MODE_ASYNC = 0,      /* async-(k): in-place, no inter-block sync (Alg. 1, eq. 4)      */
+    BAR_MODE_SYNC_BLOCK = 1, /* sync-block-(k): block-Jacobi, k local sweeps, x double-buffered */
+    BAR_MODE_JACOBI = 2      /* synchronous Jacobi (eq. 2)                                     */
+} bar_mode;
+
+typedef enum {
+    BAR_OK = 0,
+    BAR_ERR_INVALID_ARG = 1, /* NULL handle/pointer, n < 1, k < 1, tol < 0 or NaN, R out of range ... */
+    BAR_ERR_BAD_CSR = 2,     /* rowptr[0] != 0, rowptr not monotone, rowptr[n] != nnz, col out of
+                                [0, n), columns not strictly increasing, missing diagonal           */
+    BAR_ERR_ZERO_DIAG = 3,   /* a_ii == 0                                                         */
+    BAR_ERR_NONFINITE = 4,   /* a value is Inf/NaN (matrix, or b / x0 at solve time)              */
+    BAR_ERR_DIVERGED = 5,    /* rel. residual became non-finite or > 1e30 (rho(B) > 1)     */
+    BAR_ERR_CUDA = 6,        /* CUDA runtime failure; see bar_last_error()                        */
+    BAR_ERR_NCCL = 7,        /* NCCL failure (multi-GPU)                                          */
+    BAR_ERR_OOM = 8          /* device allocation failed                                          */
+} bar_status;
+
+/* Largest subdomain size R accepted (two fp64 copies of the block's x live in shared memory). */
+#define BAR_MAX_ROWS_PER_BLOCK 8192
+
+typedef struct {
+    int64_t iters;          /* global iterations m of the returned x = x^(m) (sync modes: exactly
+                               the oracle's count; async: completed global iterations)           */
+    double rel_res;         /* ||b - A x||_2 / ||b||_2 of the RETURNED x, computed exactly       */
+    int32_t converged;      /* rel_res <= tol                                                     */
+    int64_t cta_iters_min;  /* async persistent kernel: min / max per-block global iteration      */
+    int64_t cta_iters_max;  /*   counts (= iters otherwise)                                       */
+    double model_bytes_per_iter; /* nnz*(8+4) + n*(8+8+8+4): the contract bytes of one iteration */
+    int64_t kernel_launches;     /* kernels this call launched (all of them libbar's own)         */
+} bar_solve_info;
+
+typedef struct {
+    int64_t n, nnz;               /* matrix size and stored entries                              */
+    int32_t rows_per_block;       /* R                                                            */
+    int64_t num_subdomains;       /* q = ceil(n / R)                                              */
+    int64_t layout_entries;       /* stored entries incl. padding of the sliced layout            */
+    int64_t local_entries;        /* entries with a column inside their row's subdomain (incl. diag) */
+    double model_bytes_per_iter;  /* nnz*(8+4) + n*(8+8+8+4)                                      */
+    int32_t device;
+} bar_matrix_info;
+
+/*
+ * bar_create_csr — validate a CSR matrix and copy it into the library layout.
+ *   n            rows = columns (>= 1)
+ *   nnz          stored entries (= rowptr[n]; < 2^31)
+ *   rowptr       int32[n+1], rowptr[0] = 0, non-decreasing
+ *   col          int32[nnz], 0 <= col < n, strictly increasing within each row, diagonal present
+ *   val          double[nnz], finite, a_ii != 0
+ *   rows_per_block  R, subdomain size (1 <= R <= BAR_MAX_ROWS_PER_BLOCK); J_l = [l R, min(n,(l+1) R))
+ *   device       CUDA device ordinal for the layout and all later calls
+ *   out          receives the handle (set to NULL on failure)
+ * Errors: BAR_ERR_INVALID_ARG, BAR_ERR_BAD_CSR, BAR_ERR_ZERO_DIAG, BAR_ERR_NONFINITE,
+ *         BAR_ERR_CUDA, BAR_ERR_OOM.
+ */
+bar_status bar_create_csr(int64_t n, int64_t nnz, const int32_t *rowptr, const int32_t *col,
+                          const double *val, int32_t rows_per_block, int device, bar_matrix *out);
+
+/*
+ * bar_solve — iterate from x0 until ||b - A x^(m)||_2 / ||b||_2 <= tol or m = max_global_iters.
+ *   b, x0        double[n] (device or host); x0 == NULL means x0 = 0
+ *   x            double[n] output (device or host); may alias x0
+ *   k            local Jacobi sweeps per global iteration (async / sync-block; ignored for
+ *                Jacobi), >= 1 — the paper's async-(k)
+ *   max_global_iters  >= 0
+ *   tol          >= 0 (0 = run exactly max_global_iters iterations unless the residual is 0)
+ *   mode         BAR_MODE_ASYNC / BAR_MODE_SYNC_BLOCK / BAR_MODE_JACOBI
+ *   cuda_stream  cudaStream_t or NULL
+ *   info         nullable
+ * Stopping rule (reading R6): x^(0) is checked first; the sync modes return the
+ * first x^(m) with rel_res <= tol (bitwise the oracle's m up to the order of the residual sum);
+ * async returns the first iterate whose fused residual estimate AND exact confirming residual
+ * are <= tol. b = 0 returns x = 0, iters = 0, converged.
+ * Errors: BAR_ERR_INVALID_ARG, BAR_ERR_NONFINITE (b or x0), BAR_ERR_DIVERGED, BAR_ERR_CUDA,
+ *         BAR_ERR_OOM. On BAR_ERR_DIVERGED x holds the last iterate.
+ */
+bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x, int32_t k,
+                     int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
+                     bar_solve_info *info);
+
+/*
+ * bar_residual — res_norm2 = ||b - A x||_2 (and b_norm2 = ||b||_2 if non-NULL), computed on the
+ * device with a fixed-order (deterministic) reduction. b, x device or host.
+ * Errors: BAR_ERR_INVALID_ARG, BAR_ERR_CUDA, BAR_ERR_OOM.
+ */
+bar_status bar_residual(bar_matrix A, const double *b, const double *x, void *cuda_stream,
+                        double *res_norm2, double *b_norm2);
+
+/*
+ * bar_sweep — run exactly `nsweeps` global iterations of `mode` from the current x, with no
+ * convergence control and no host synchronisation (stream-ordered; returns after enqueueing).
+ * Sync modes ping-pong between x and a library buffer and leave x^(nsweeps) in x; async updates
+ * x in place. For callers that drive their own loop and for per-launch kernel timing.
+ *   b, x   DEVICE double[n] on the matrix's device; k >= 1; nsweeps >= 0.
+ * Errors: BAR_ERR_INVALID_ARG (also for host pointers), BAR_ERR_CUDA, BAR_ERR_OOM.
+ */
+bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_t nsweeps, bar_mode mode,
+                     void *cuda_stream);
+
+/* bar_matrix_get_info — sizes and the contract bytes per global iteration of a handle. */
+bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info);
+
+/* bar_destroy — free the handle and its device memory (NULL-safe). */
+void bar_destroy(bar_matrix A);
+
+/* bar_last_error — text of the last failure on the calling thread ("" if none). */
+const char *bar_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* BAR_H */

@@ -1,0 +1,427 @@
+// api.cu — the C ABI of include/bar.h and the global-iteration driver.
+//
+// Driver. Sync modes (Jacobi, sync-block): launch m reads x^(m-1) from one buffer, writes x^(m)
+// to the other and fuses rel_res(x^(m-1)); its last block sets a device stop flag when
+// rel_res(x^(m-1)) <= tol, after which queued launches return immediately. The host enqueues
+// launches in growing chunks and reads the 64-byte device state once per chunk (the only
+// device->host traffic inside the loop). Async mode iterates in place; its fused residual mixes
+// old and new values (eq. 3's shift), so a stop request is confirmed by an exact residual.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <string>
+
+#include "bar_internal.cuh"
+
+namespace bar {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string &msg) { g_err = msg; }
+
+bar_status cuda_fail(cudaError_t e, const char *what) {
+    g_err = std::string(what) + ": " + cudaGetErrorString(e);
+    cudaGetLastError();
+    return e == cudaErrorMemoryAllocation ? BAR_ERR_OOM : BAR_ERR_CUDA;
+}
+
+namespace {
+
+// RAII: switch to the handle's device for the duration of a call.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+bool is_device_ptr(const void *p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+bar_status ensure_workspace(bar_matrix A) {
+    Workspace &W = A->W;
+    const Layout &L = A->L;
+    if (!W.state) {
+        BAR_CUDA(cudaMalloc(&W.state, sizeof(DevState)));
+        BAR_CUDA(cudaMallocHost(&W.h_state, sizeof(DevState)));
+        BAR_CUDA(cudaMemset(W.state, 0, sizeof(DevState)));
+    }
+    int64_t need = std::max(num_blocks_for(L, BAR_MODE_SYNC_BLOCK), num_blocks_for(L, BAR_MODE_JACOBI));
+    if (W.npartials < need) {
+        cudaFree(W.partials);
+        W.partials = nullptr;
+        BAR_CUDA(cudaMalloc(&W.partials, sizeof(double) * 2 * (size_t)need));
+        W.npartials = need;
+    }
+    return BAR_OK;
+}
+
+bar_status ensure_buf(double **p, int64_t n) {
+    if (!*p) BAR_CUDA(cudaMalloc(p, sizeof(double) * (size_t)n));
+    return BAR_OK;
+}
+
+double model_bytes(const Layout &L) { return (double)L.nnz * (8 + 4) + (double)L.n * (8 + 8 + 8 + 4); }
+
+bar_status read_state(bar_matrix A, cudaStream_t st) {
+    BAR_CUDA(cudaMemcpyAsync(A->W.h_state, A->W.state, sizeof(DevState), cudaMemcpyDeviceToHost, st));
+    BAR_CUDA(cudaStreamSynchronize(st));
+    return BAR_OK;
+}
+
+}  // namespace
+}  // namespace bar
+
+using namespace bar;
+
+extern "C" {
+
+const char *bar_last_error(void) { return g_err.c_str(); }
+
+bar_status bar_create_csr(int64_t n, int64_t nnz, const int32_t *rowptr, const int32_t *col, const double *val,
+                          int32_t rows_per_block, int device, bar_matrix *out) {
+    g_err.clear();
+    if (!out) {
+        set_error("out is NULL");
+        return BAR_ERR_INVALID_ARG;
+    }
+    *out = nullptr;
+    if (n < 1 || nnz < n || nnz >= (int64_t)INT32_MAX || n >= (int64_t)INT32_MAX || !rowptr || !col || !val) {
+        set_error("invalid n/nnz or NULL array (need n >= 1, n <= nnz < 2^31, diagonal in every row)");
+        return nnz < n && n >= 1 && rowptr && col && val ? BAR_ERR_BAD_CSR : BAR_ERR_INVALID_ARG;
+    }
+    if (rows_per_block < 1 || rows_per_block > BAR_MAX_ROWS_PER_BLOCK) {
+        set_error("rows_per_block out of [1, BAR_MAX_ROWS_PER_BLOCK]");
+        return BAR_ERR_INVALID_ARG;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+        cudaGetLastError();
+        set_error("invalid CUDA device");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(device);
+    if (!g.ok) return cuda_fail(cudaGetLastError(), "cudaSetDevice");
+
+    // Inputs: stage host arrays through device copies; device arrays are used in place.
+    const int32_t *d_rowptr = rowptr, *d_col = col;
+    const double *d_val = val;
+    int32_t *t_rowptr = nullptr, *t_col = nullptr;
+    double *t_val = nullptr;
+    bar_status st_ = BAR_OK;
+    int32_t ends[2] = {0, 0};
+    cudaStream_t s = nullptr;
+    auto *A = new bar_matrix_s();
+    A->device = device;
+    auto stage = [&](const void *src, void **dst, size_t bytes) -> bar_status {
+        if (is_device_ptr(src)) return BAR_OK;
+        BAR_CUDA(cudaMalloc(dst, bytes ? bytes : 1));
+        BAR_CUDA(cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice));
+        return BAR_OK;
+    };
+    if ((st_ = stage(rowptr, (void **)&t_rowptr, sizeof(int32_t) * (size_t)(n + 1))) != BAR_OK) goto fail;
+    if ((st_ = stage(col, (void **)&t_col, sizeof(int32_t) * (size_t)nnz)) != BAR_OK) goto fail;
+    if ((st_ = stage(val, (void **)&t_val, sizeof(double) * (size_t)nnz)) != BAR_OK) goto fail;
+    if (t_rowptr) d_rowptr = t_rowptr;
+    if (t_col) d_col = t_col;
+    if (t_val) d_val = t_val;
+    if (cudaMemcpy(&ends[0], d_rowptr, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess ||
+        cudaMemcpy(&ends[1], d_rowptr + n, sizeof(int32_t), cudaMemcpyDeviceToHost) != cudaSuccess) {
+        st_ = cuda_fail(cudaGetLastError(), "read rowptr");
+        goto fail;
+    }
+    if (ends[0] != 0 || ends[1] != nnz) {
+        set_error("rowptr[0] != 0 or rowptr[n] != nnz");
+        st_ = BAR_ERR_BAD_CSR;
+        goto fail;
+    }
+    st_ = build_layout(A->L, n, nnz, d_rowptr, d_col, d_val, rows_per_block, s);
+    if (st_ != BAR_OK) goto fail;
+    cudaFree(t_rowptr);
+    cudaFree(t_col);
+    cudaFree(t_val);
+    *out = A;
+    return BAR_OK;
+fail:
+    cudaFree(t_rowptr);
+    cudaFree(t_col);
+    cudaFree(t_val);
+    delete A;
+    return st_;
+}
+
+void bar_destroy(bar_matrix A) {
+    if (!A) return;
+    DeviceGuard g(A->device);
+    free_layout(A->L);
+    Workspace &W = A->W;
+    cudaFree(W.xbuf);
+    cudaFree(W.stage_b);
+    cudaFree(W.stage_x);
+    cudaFree(W.partials);
+    cudaFree(W.state);
+    cudaFreeHost(W.h_state);
+    delete A;
+}
+
+bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info) {
+    if (!A || !info) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    const Layout &L = A->L;
+    info->n = L.n;
+    info->nnz = L.nnz;
+    info->rows_per_block = L.R;
+    info->num_subdomains = L.q;
+    info->layout_entries = L.entries;
+    info->local_entries = L.local_entries;
+    info->model_bytes_per_iter = model_bytes(L);
+    info->device = A->device;
+    return BAR_OK;
+}
+
+bar_status bar_residual(bar_matrix A, const double *b, const double *x, void *cuda_stream, double *res_norm2,
+                        double *b_norm2) {
+    g_err.clear();
+    if (!A || !b || !x || !res_norm2) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(A->device);
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    bar_status r = ensure_workspace(A);
+    if (r != BAR_OK) return r;
+    const int64_t n = A->L.n;
+    const double *db = b, *dx = x;
+    if (!is_device_ptr(b)) {
+        if ((r = ensure_buf(&A->W.stage_b, n)) != BAR_OK) return r;
+        BAR_CUDA(cudaMemcpyAsync(A->W.stage_b, b, sizeof(double) * n, cudaMemcpyHostToDevice, st));
+        db = A->W.stage_b;
+    }
+    if (!is_device_ptr(x)) {
+        if ((r = ensure_buf(&A->W.stage_x, n)) != BAR_OK) return r;
+        BAR_CUDA(cudaMemcpyAsync(A->W.stage_x, x, sizeof(double) * n, cudaMemcpyHostToDevice, st));
+        dx = A->W.stage_x;
+    }
+    BAR_CUDA(launch_init_state(A->W.state, 0.0, st));
+    BAR_CUDA(launch_residual(A->L, db, dx, A->W.state, A->W.partials, st));
+    if ((r = read_state(A, st)) != BAR_OK) return r;
+    *res_norm2 = std::sqrt(A->W.h_state->exact_ss);
+    if (b_norm2) *b_norm2 = A->W.h_state->bnorm;
+    return BAR_OK;
+}
+
+bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_t nsweeps, bar_mode mode,
+                     void *cuda_stream) {
+    g_err.clear();
+    if (!A || !b || !x || nsweeps < 0 || (mode != BAR_MODE_JACOBI && k < 1) ||
+        (mode != BAR_MODE_ASYNC && mode != BAR_MODE_SYNC_BLOCK && mode != BAR_MODE_JACOBI)) {
+        set_error("invalid argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if (mode == BAR_MODE_JACOBI) k = 1;
+    DeviceGuard g(A->device);
+    if (!is_device_ptr(b) || !is_device_ptr(x)) {
+        set_error("bar_sweep takes device pointers only");
+        return BAR_ERR_INVALID_ARG;
+    }
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    bar_status r = ensure_workspace(A);
+    if (r != BAR_OK) return r;
+    double *buf1 = x;
+    if (mode != BAR_MODE_ASYNC) {
+        if ((r = ensure_buf(&A->W.xbuf, A->L.n)) != BAR_OK) return r;
+        buf1 = A->W.xbuf;
+    }
+    BAR_CUDA(launch_init_state(A->W.state, -1.0, st));
+    for (int64_t m = 1; m <= nsweeps; ++m) {
+        const double *xi = (m & 1) ? x : buf1;
+        double *xo = (mode == BAR_MODE_ASYNC) ? x : ((m & 1) ? buf1 : x);
+        SweepArgs a{&A->L, b, xi, xo, k, A->W.state, A->W.partials, nullptr};
+        BAR_CUDA(launch_sweep(a, mode, st));
+    }
+    if (mode != BAR_MODE_ASYNC && (nsweeps & 1))
+        BAR_CUDA(cudaMemcpyAsync(x, buf1, sizeof(double) * (size_t)A->L.n, cudaMemcpyDeviceToDevice, st));
+    return BAR_OK;
+}
+
+bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x, int32_t k, int64_t max_global_iters,
+                     double tol, bar_mode mode, void *cuda_stream, bar_solve_info *info) {
+    g_err.clear();
+    if (!A || !b || !x) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if (mode != BAR_MODE_ASYNC && mode != BAR_MODE_SYNC_BLOCK && mode != BAR_MODE_JACOBI) {
+        set_error("invalid mode");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if ((mode != BAR_MODE_JACOBI && k < 1) || max_global_iters < 0 || !(tol >= 0.0)) {
+        set_error("need k >= 1, max_global_iters >= 0, tol >= 0");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if (mode == BAR_MODE_JACOBI) k = 1;
+    DeviceGuard g(A->device);
+    if (!g.ok) return cuda_fail(cudaGetLastError(), "cudaSetDevice");
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    const Layout &L = A->L;
+    Workspace &W = A->W;
+    const int64_t n = L.n;
+    const size_t bytes = sizeof(double) * (size_t)n;
+    bar_status r = ensure_workspace(A);
+    if (r != BAR_OK) return r;
+    int64_t launches = 0;
+
+    // End-to-end path: host vectors are staged through device buffers inside the call.
+    const double *db = b;
+    const bool x_dev = is_device_ptr(x);
+    if (!is_device_ptr(b)) {
+        if ((r = ensure_buf(&W.stage_b, n)) != BAR_OK) return r;
+        BAR_CUDA(cudaMemcpyAsync(W.stage_b, b, bytes, cudaMemcpyHostToDevice, st));
+        db = W.stage_b;
+    }
+    double *buf0 = x;  // iterate buffer 0 (in place for async)
+    if (!x_dev) {
+        if ((r = ensure_buf(&W.stage_x, n)) != BAR_OK) return r;
+        buf0 = W.stage_x;
+    }
+    if (x0 == nullptr) {
+        BAR_CUDA(cudaMemsetAsync(buf0, 0, bytes, st));
+    } else if (x0 != x || !x_dev) {
+        BAR_CUDA(cudaMemcpyAsync(buf0, x0, bytes, cudaMemcpyDefault, st));
+    }
+    double *buf1 = nullptr;
+    if (mode != BAR_MODE_ASYNC) {
+        if ((r = ensure_buf(&W.xbuf, n)) != BAR_OK) return r;
+        buf1 = W.xbuf;
+    }
+    BAR_CUDA(launch_init_state(W.state, tol, st));
+    ++launches;
+
+    DevState &H = *W.h_state;
+    int64_t iters = 0;
+    double rel = 0.0;
+    int converged = 0;
+    bool diverged = false, nonfinite = false, bzero = false;
+    double *result = buf0;
+    int64_t chunk = 8;
+
+    if (mode != BAR_MODE_ASYNC) {
+        int64_t issued = 0;  // launches m = 1..issued
+        bool stopped = false;
+        while (issued < max_global_iters && !stopped) {
+            const int64_t c = std::min(chunk, max_global_iters - issued);
+            for (int64_t i = 0; i < c; ++i) {
+                const int64_t m = issued + i + 1;
+                SweepArgs a{&L, db, (m & 1) ? buf0 : buf1, (m & 1) ? buf1 : buf0, k, W.state, W.partials, nullptr};
+                BAR_CUDA(launch_sweep(a, mode, st));
+            }
+            launches += c;
+            issued += c;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            stopped = H.stop != 0;
+            chunk = std::min<int64_t>(chunk * 2, 256);
+        }
+        if (stopped) {
+            iters = H.conv_iter;
+            rel = H.last_rel;
+            if (H.diverged == 2) bzero = true;
+            else if (H.diverged == 1) diverged = true;
+            else converged = 1;
+            result = (iters & 1) ? buf1 : buf0;
+        } else {
+            iters = max_global_iters;
+            result = (iters & 1) ? buf1 : buf0;
+            BAR_CUDA(launch_residual(L, db, result, W.state, W.partials, st));
+            ++launches;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            if (H.bnorm == 0.0) {
+                bzero = true;
+            } else {
+                rel = H.exact_rel;
+                if (!std::isfinite(rel) || rel > 1e30) diverged = true;
+                converged = rel <= tol;
+            }
+        }
+    } else {
+        // async-(k): in place on buf0. Check x^(0) first (exact), then iterate.
+        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+        ++launches;
+        if ((r = read_state(A, st)) != BAR_OK) return r;
+        rel = H.exact_rel;
+        if (H.bnorm == 0.0) bzero = true;
+        else if (!std::isfinite(rel)) diverged = true;
+        else if (rel <= tol) converged = 1;
+        while (!converged && !bzero && !diverged && H.iter < max_global_iters) {
+            const int64_t c = std::min<int64_t>(chunk, max_global_iters - (int64_t)H.iter);
+            for (int64_t i = 0; i < c; ++i) {
+                SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+                BAR_CUDA(launch_sweep(a, mode, st));
+            }
+            launches += c;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            chunk = std::min<int64_t>(chunk * 2, 256);
+            if (H.diverged == 1) {
+                diverged = true;
+                break;
+            }
+            if (H.stop || H.iter >= max_global_iters) {
+                BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+                ++launches;
+                if ((r = read_state(A, st)) != BAR_OK) return r;
+                rel = H.exact_rel;
+                if (!std::isfinite(rel) || rel > 1e30) diverged = true;
+                else if (rel <= tol) converged = 1;
+                else if (H.stop) BAR_CUDA(cudaMemsetAsync(&W.state->stop, 0, sizeof(int), st));
+            }
+        }
+        iters = H.iter;
+        result = buf0;
+    }
+    if (bzero) {
+        BAR_CUDA(cudaMemsetAsync(buf0, 0, bytes, st));
+        result = buf0;
+        iters = 0;
+        rel = 0.0;
+        converged = 1;
+        diverged = false;
+    }
+    if (diverged && iters == 0 && !std::isfinite(rel)) nonfinite = true;
+    if (result != x) BAR_CUDA(cudaMemcpyAsync(x, result, bytes, x_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
+    BAR_CUDA(cudaStreamSynchronize(st));
+    if (info) {
+        info->iters = iters;
+        info->rel_res = rel;
+        info->converged = converged;
+        info->cta_iters_min = iters;
+        info->cta_iters_max = iters;
+        info->model_bytes_per_iter = model_bytes(L);
+        info->kernel_launches = launches;
+    }
+    if (nonfinite) {
+        set_error("non-finite b or x0");
+        return BAR_ERR_NONFINITE;
+    }
+    if (diverged) {
+        set_error("relative residual became non-finite or exceeded 1e30 (rho(B) > 1?)");
+        return BAR_ERR_DIVERGED;
+    }
+    return BAR_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,112 @@
+// bar_internal.cuh — library-private types shared by the libbar.so translation units.
+//
+// Device layout of a matrix ("split sliced-ELL"):
+//   * rows are grouped into subdomains J_l = [l*R, min(n,(l+1)*R)) (eq. 4's TS..TE);
+//   * each subdomain is cut into slices of 32 consecutive rows (one warp, lane = row);
+//     slice s = l*SPB + j (SPB = ceil(R/32)) holds rows TS + 32 j + lane;
+//   * a slice stores its rows' entries column-major (entry e of lane t at ptr[s] + 32 e + t),
+//     first the `wl` LOCAL entries (column inside J_l, stored as the local index col - TS,
+//     the diagonal always local entry 0) and then the `wo` OFF-BLOCK entries (global column);
+//     shorter rows are padded with value 0 and a harmless column (their own row).
+// So one warp-wide load of entry e is a single coalesced 256 B (values) / 128 B (columns)
+// transaction, the local/off-block split of Alg. 1 costs nothing at run time,
+// and the diagonal (for D^-1) is found without a search.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "bar.h"
+
+namespace bar {
+
+constexpr int kSlice = 32;  // rows per slice = warp width
+
+// Device-resident solver state (one per matrix handle), updated by the last block of each
+// launch (fixed-order final reduction). Read back by the host once per chunk of launches.
+struct DevState {
+    unsigned int counter;   // last-block ticket
+    int stop;               // kernels return immediately when set
+    int diverged;
+    int pad0;
+    long long iter;         // launches that executed (sync: m of the latest x^(m) produced)
+    long long conv_iter;    // sync: m with rel_res(x^(m)) <= tol
+    double bnorm;           // ||b||_2
+    double tol;
+    double last_rel;        // latest fused relative residual
+    double exact_rel;       // latest standalone residual (bar_residual / confirmation)
+    double exact_ss;        // its sum of squares
+};
+
+struct Layout {
+    int64_t n = 0, nnz = 0;
+    int32_t R = 0;
+    int32_t spb = 0;            // slices per (full) subdomain
+    int64_t q = 0;              // subdomains
+    int64_t nslices = 0;
+    int64_t entries = 0;        // padded entries
+    int64_t local_entries = 0;
+    int max_wl = 0, max_wo = 0;
+    // device arrays
+    double *val = nullptr;      // [entries]
+    int32_t *col = nullptr;     // [entries]
+    int64_t *sptr = nullptr;    // [nslices+1] entry offset of each slice
+    int32_t *sw = nullptr;      // [nslices]   wl | (wo << 16)
+};
+
+struct Workspace {
+    double *xbuf = nullptr;     // n: second iterate buffer (sync modes)
+    double *stage_b = nullptr;  // n: device staging of host b (end-to-end path)
+    double *stage_x = nullptr;  // n: device staging of host x0/x
+    double *partials = nullptr; // per-block partial sums of squares
+    int64_t npartials = 0;
+    DevState *state = nullptr;  // device
+    DevState *h_state = nullptr;// pinned host mirror
+};
+
+}  // namespace bar
+
+struct bar_matrix_s {
+    int device = 0;
+    bar::Layout L;
+    bar::Workspace W;
+};
+
+namespace bar {
+
+void set_error(const std::string &msg);
+bar_status cuda_fail(cudaError_t e, const char *what);
+
+#define BAR_CUDA(call)                                              \
+    do {                                                            \
+        cudaError_t _e = (call);                                    \
+        if (_e != cudaSuccess) return ::bar::cuda_fail(_e, #call);  \
+    } while (0)
+
+// Layout construction (layout.cu). rowptr/col/val are DEVICE pointers.
+bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowptr, const int32_t *d_col,
+                        const double *d_val, int32_t R, cudaStream_t st);
+void free_layout(Layout &L);
+
+// Kernel launchers (sweep.cu). All pointers are device pointers.
+struct SweepArgs {
+    const Layout *L;
+    const double *b;
+    const double *x_in;
+    double *x_out;
+    int k;
+    DevState *state;
+    double *partials;
+    double *hist;  // nullable device array: hist[m-1] = rel_res(x^(m-1)) (sync modes)
+};
+int64_t num_blocks_for(const Layout &L, bar_mode mode);
+cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st);
+cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state,
+                            double *partials, cudaStream_t st);
+cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
+cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
+cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
+
+}  // namespace bar

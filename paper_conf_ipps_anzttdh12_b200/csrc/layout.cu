@@ -1,0 +1,276 @@
+// layout.cu — CSR validation and conversion to the split sliced-ELL device layout
+// (the layout itself is described in bar_internal.cuh / DESIGN.md).
+//
+// Runs once per bar_create_csr on the device (the 128M-row config has ~0.94G entries), outside
+// every timed region ("initialisation ... subtracted").
+#include <cub/cub.cuh>
+
+#include "bar_internal.cuh"
+
+namespace bar {
+namespace {
+
+enum : int { kErrBadCsr = 1, kErrZeroDiag = 2, kErrNonFinite = 4 };
+
+__device__ __forceinline__ void slice_row(int64_t s, int32_t R, int32_t spb, int64_t n, int64_t &row, bool &valid,
+                                          int64_t &TS, int lane) {
+    int64_t l = s / spb;
+    int64_t j = s - l * spb;
+    TS = l * (int64_t)R;
+    int64_t nrows = min((int64_t)R, n - TS);
+    int64_t loc = j * kSlice + lane;
+    valid = loc < nrows;
+    row = TS + loc;
+}
+
+// Per row: validate and count local (column inside the row's subdomain, diagonal included)
+// and off-block entries.
+__global__ void k_validate_count(int64_t n, int64_t nnz, const int32_t *__restrict__ rowptr,
+                                 const int32_t *__restrict__ col, const double *__restrict__ val, int32_t R,
+                                 int32_t *__restrict__ nloc, int32_t *__restrict__ noff, int *__restrict__ err) {
+    int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    int32_t a = rowptr[i], e = rowptr[i + 1];
+    if (a < 0 || e < a || e > nnz) {
+        atomicOr(err, kErrBadCsr);
+        nloc[i] = 1;
+        noff[i] = 0;
+        return;
+    }
+    int64_t TS = (i / R) * (int64_t)R;
+    int64_t TE = min(TS + (int64_t)R, n);
+    int cl = 0, co = 0, bad = 0;
+    bool diag = false;
+    int64_t prev = -1;
+    for (int32_t p = a; p < e; ++p) {
+        int64_t c = col[p];
+        double v = val[p];
+        if (c < 0 || c >= n || c <= prev) bad |= kErrBadCsr;
+        prev = c;
+        if (!isfinite(v)) bad |= kErrNonFinite;
+        if (c == i) {
+            diag = true;
+            if (v == 0.0) bad |= kErrZeroDiag;
+        }
+        if (c >= TS && c < TE) ++cl; else ++co;
+    }
+    if (!diag) bad |= kErrBadCsr;
+    if (bad) atomicOr(err, bad);
+    nloc[i] = cl;
+    noff[i] = co;
+}
+
+// Per slice (one warp): widths wl = max local count, wo = max off-block count.
+__global__ void k_slice_widths(int64_t nslices, int64_t n, int32_t R, int32_t spb, const int32_t *__restrict__ nloc,
+                               const int32_t *__restrict__ noff, int32_t *__restrict__ sw,
+                               int64_t *__restrict__ ssize) {
+    int64_t s = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kSlice;
+    int lane = threadIdx.x & (kSlice - 1);
+    if (s >= nslices) return;
+    int64_t row, TS;
+    bool valid;
+    slice_row(s, R, spb, n, row, valid, TS, lane);
+    int wl = valid ? nloc[row] : 1;
+    int wo = valid ? noff[row] : 0;
+    for (int o = 16; o > 0; o >>= 1) {
+        wl = max(wl, __shfl_xor_sync(0xffffffffu, wl, o));
+        wo = max(wo, __shfl_xor_sync(0xffffffffu, wo, o));
+    }
+    if (lane == 0) {
+        sw[s] = wl | (wo << 16);
+        ssize[s] = (int64_t)kSlice * (wl + wo);
+    }
+}
+
+// Per (slice, lane): write the lane's column of the slice — diagonal first, then the other
+// local entries ascending (local index), then off-block entries ascending (global index),
+// then padding (value 0, own row).
+__global__ void k_fill(int64_t nslices, int64_t n, int32_t R, int32_t spb, const int32_t *__restrict__ rowptr,
+                       const int32_t *__restrict__ col, const double *__restrict__ val,
+                       const int64_t *__restrict__ sptr, const int32_t *__restrict__ sw,
+                       double *__restrict__ oval, int32_t *__restrict__ ocol) {
+    int64_t gt = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    int64_t s = gt / kSlice;
+    int lane = (int)(gt & (kSlice - 1));
+    if (s >= nslices) return;
+    int64_t row, TS;
+    bool valid;
+    slice_row(s, R, spb, n, row, valid, TS, lane);
+    int wl = sw[s] & 0xffff, wo = sw[s] >> 16;
+    int64_t base = sptr[s] + lane;
+    int64_t TE = min(TS + (int64_t)R, n);
+    int32_t own_loc = (int32_t)(row - TS);
+    int32_t own_glb = (int32_t)(valid ? row : TS);
+    int el = 0, eo = 0;
+    if (valid) {
+        int32_t a = rowptr[row], e = rowptr[row + 1];
+        for (int32_t p = a; p < e; ++p)  // diagonal -> local entry 0
+            if (col[p] == row) {
+                oval[base] = val[p];
+                ocol[base] = own_loc;
+                el = 1;
+            }
+        for (int32_t p = a; p < e; ++p) {
+            int64_t c = col[p];
+            if (c == row) continue;
+            if (c >= TS && c < TE) {
+                oval[base + (int64_t)el * kSlice] = val[p];
+                ocol[base + (int64_t)el * kSlice] = (int32_t)(c - TS);
+                ++el;
+            } else {
+                oval[base + (int64_t)(wl + eo) * kSlice] = val[p];
+                ocol[base + (int64_t)(wl + eo) * kSlice] = (int32_t)c;
+                ++eo;
+            }
+        }
+    } else {
+        own_loc = 0;
+    }
+    for (; el < wl; ++el) {
+        oval[base + (int64_t)el * kSlice] = 0.0;
+        ocol[base + (int64_t)el * kSlice] = own_loc;
+    }
+    for (; eo < wo; ++eo) {
+        oval[base + (int64_t)(wl + eo) * kSlice] = 0.0;
+        ocol[base + (int64_t)(wl + eo) * kSlice] = own_glb;
+    }
+}
+
+template <class T>
+cudaError_t dmalloc(T **p, size_t count) {
+    return cudaMalloc((void **)p, sizeof(T) * (count ? count : 1));
+}
+
+}  // namespace
+
+void free_layout(Layout &L) {
+    cudaFree(L.val);
+    cudaFree(L.col);
+    cudaFree(L.sptr);
+    cudaFree(L.sw);
+    L.val = nullptr;
+    L.col = nullptr;
+    L.sptr = nullptr;
+    L.sw = nullptr;
+}
+
+static bar_status alloc_fail(cudaError_t e, const char *what) {
+    if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        set_error(std::string("out of device memory: ") + what);
+        return BAR_ERR_OOM;
+    }
+    return cuda_fail(e, what);
+}
+
+#define BAR_ALLOC(call)                                        \
+    do {                                                       \
+        cudaError_t _e = (call);                               \
+        if (_e != cudaSuccess) { st_ = alloc_fail(_e, #call); goto done; } \
+    } while (0)
+#define BAR_CK(call)                                           \
+    do {                                                       \
+        cudaError_t _e = (call);                               \
+        if (_e != cudaSuccess) { st_ = cuda_fail(_e, #call); goto done; } \
+    } while (0)
+
+bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowptr, const int32_t *d_col,
+                        const double *d_val, int32_t R, cudaStream_t st) {
+    bar_status st_ = BAR_OK;
+    int32_t *nloc = nullptr, *noff = nullptr;
+    int *d_err = nullptr;
+    int64_t *ssize = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0, tmp2 = 0;
+    int h_err = 0;
+    int64_t *d_sum = nullptr;
+    int64_t h_tot[2] = {0, 0};
+    int h_w[2] = {0, 0};
+
+    L.n = n;
+    L.nnz = nnz;
+    L.R = R;
+    L.spb = (R + kSlice - 1) / kSlice;
+    L.q = (n + R - 1) / R;
+    {
+        int64_t last_rows = n - (L.q - 1) * (int64_t)R;
+        L.nslices = (L.q - 1) * (int64_t)L.spb + (last_rows + kSlice - 1) / kSlice;
+    }
+    const int TB = 256;
+    int64_t nsl = L.nslices;
+
+    BAR_ALLOC(dmalloc(&nloc, (size_t)n));
+    BAR_ALLOC(dmalloc(&noff, (size_t)n));
+    BAR_ALLOC(dmalloc(&d_err, 1));
+    BAR_ALLOC(dmalloc(&ssize, (size_t)nsl + 1));
+    BAR_ALLOC(dmalloc(&d_sum, 2));
+    BAR_ALLOC(dmalloc(&L.sptr, (size_t)nsl + 1));
+    BAR_ALLOC(dmalloc(&L.sw, (size_t)nsl));
+    BAR_CK(cudaMemsetAsync(d_err, 0, sizeof(int), st));
+
+    k_validate_count<<<(unsigned)((n + TB - 1) / TB), TB, 0, st>>>(n, nnz, d_rowptr, d_col, d_val, R, nloc, noff,
+                                                                  d_err);
+    BAR_CK(cudaGetLastError());
+    BAR_CK(cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, st));
+    BAR_CK(cudaStreamSynchronize(st));
+    if (h_err & kErrBadCsr) { set_error("malformed CSR (rowptr/col/diagonal)"); st_ = BAR_ERR_BAD_CSR; goto done; }
+    if (h_err & kErrNonFinite) { set_error("non-finite matrix value"); st_ = BAR_ERR_NONFINITE; goto done; }
+    if (h_err & kErrZeroDiag) { set_error("zero diagonal entry"); st_ = BAR_ERR_ZERO_DIAG; goto done; }
+
+    k_slice_widths<<<(unsigned)((nsl * kSlice + TB - 1) / TB), TB, 0, st>>>(nsl, n, R, L.spb, nloc, noff, L.sw,
+                                                                           ssize);
+    BAR_CK(cudaGetLastError());
+    BAR_CK(cudaMemsetAsync(ssize + nsl, 0, sizeof(int64_t), st));
+    // slice offsets: exclusive scan of slice sizes (nslices+1 entries -> sptr[nslices] = total)
+    BAR_CK(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, ssize, L.sptr, nsl + 1, st));
+    BAR_CK(cub::DeviceReduce::Sum(nullptr, tmp2, nloc, d_sum + 1, n, st));
+    if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
+    BAR_CK(cub::DeviceReduce::Max(nullptr, tmp2, nloc, (int32_t *)d_sum, n, st));
+    if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
+    BAR_ALLOC(cudaMalloc(&tmp, tmp_bytes));
+    BAR_CK(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, ssize, L.sptr, nsl + 1, st));
+    BAR_CK(cudaMemcpyAsync(&h_tot[0], L.sptr + nsl, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    {
+        // count local entries (int32 counts summed into int64)
+        size_t tb = tmp_bytes;
+        BAR_CK(cub::DeviceReduce::Sum(tmp, tb, nloc, d_sum + 1, n, st));
+        BAR_CK(cudaMemcpyAsync(&h_tot[1], d_sum + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        tb = tmp_bytes;
+        BAR_CK(cub::DeviceReduce::Max(tmp, tb, nloc, (int32_t *)d_sum, n, st));
+        BAR_CK(cudaMemcpyAsync(&h_w[0], d_sum, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+        tb = tmp_bytes;
+        BAR_CK(cub::DeviceReduce::Max(tmp, tb, noff, (int32_t *)d_sum, n, st));
+        BAR_CK(cudaMemcpyAsync(&h_w[1], d_sum, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    }
+    BAR_CK(cudaStreamSynchronize(st));
+    L.entries = h_tot[0];
+    L.local_entries = h_tot[1];
+    L.max_wl = h_w[0];
+    L.max_wo = h_w[1];
+    if (L.max_wl > 0xffff || L.max_wo > 0x7fff) {
+        set_error("a row has more than 32767 off-block or 65535 local entries");
+        st_ = BAR_ERR_INVALID_ARG;
+        goto done;
+    }
+    // +4 entries of slack so 16-byte vector loads past the last slice stay in bounds
+    BAR_ALLOC(dmalloc(&L.val, (size_t)L.entries + 4));
+    BAR_ALLOC(dmalloc(&L.col, (size_t)L.entries + 4));
+    BAR_CK(cudaMemsetAsync(L.val + L.entries, 0, 4 * sizeof(double), st));
+    BAR_CK(cudaMemsetAsync(L.col + L.entries, 0, 4 * sizeof(int32_t), st));
+    k_fill<<<(unsigned)((nsl * kSlice + TB - 1) / TB), TB, 0, st>>>(nsl, n, R, L.spb, d_rowptr, d_col, d_val, L.sptr,
+                                                                   L.sw, L.val, L.col);
+    BAR_CK(cudaGetLastError());
+    BAR_CK(cudaStreamSynchronize(st));
+
+done:
+    cudaFree(nloc);
+    cudaFree(noff);
+    cudaFree(d_err);
+    cudaFree(ssize);
+    cudaFree(d_sum);
+    cudaFree(tmp);
+    if (st_ != BAR_OK) free_layout(L);
+    return st_;
+}
+
+}  // namespace bar

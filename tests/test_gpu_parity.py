@@ -1,0 +1,257 @@
+"""GPU parity: the CUDA path (through libbar.so's C ABI) against the CPU oracle.
+
+Tolerances: sync-block and Jacobi iterates must match the oracle to
+||x_gpu - x_oracle||_inf <= 1e-12 * ||x_oracle||_inf at every checked iterate (north star);
+exact (dyadic) cases bitwise; iteration counts equal. Async is nondeterministic (eq. 3,
+P:93-99) and is validated by outcome: exact rel_res <= tol, solution within 1e-8 relative of
+the direct solve, iteration count reported next to the oracle's.
+"""
+import numpy as np
+import pytest
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+TOL_ITERATE = 1e-12
+
+
+def _dev(a):
+    import torch
+
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def _solve(bar, A, b, R, k, mode, max_iters, tol, x0=None):
+    import torch
+
+    M = bar.Matrix.from_csr(A, rows_per_block=R)
+    bd = _dev(b)
+    x0d = None if x0 is None else _dev(x0)
+    x = torch.empty_like(bd)
+    x, info = M.solve(bd, x0d, x, k=k, max_global_iters=max_iters, tol=tol, mode=mode)
+    torch.cuda.synchronize()
+    M.close()
+    return x.cpu().numpy(), info
+
+
+def _close(x, ref, tol=TOL_ITERATE):
+    err = np.abs(x - ref).max()
+    scale = np.abs(ref).max()
+    assert err <= tol * scale, (err, scale, err / scale)
+
+
+MATS = {
+    "tref2000": lambda: W.trefethen(2000),
+    "fv1": lambda: W.stencil9_2d(98),
+    "s7_m12": lambda: W.stencil7_3d(12),
+    "rand": lambda: W.random_dd(3001, 7, seed=11, symmetric_pattern=True),
+}
+
+
+# ------------------------------------------------------------------ boundary errors
+def test_create_errors(bar):
+    A = W.trefethen(64)
+    rp, c, v = A.rowptr.copy(), A.col.copy(), A.val.copy()
+
+    def st(rp, c, v, R=16, n=64):
+        with pytest.raises(bar.BarError) as e:
+            bar.bar_create_csr(n, int(rp[-1]), rp, c, v, R)
+        return e.value.name
+
+    bad = rp.copy(); bad[0] = 1
+    assert st(bad, c, v) == "BAR_ERR_BAD_CSR"
+    bad = c.copy(); bad[5] = 64
+    assert st(rp, bad, v) == "BAR_ERR_BAD_CSR"
+    bad = c.copy(); bad[[3, 4]] = bad[[4, 3]]
+    assert st(rp, bad, v) == "BAR_ERR_BAD_CSR"
+    dv = v.copy(); dv[rp[0] + np.searchsorted(c[rp[0]:rp[1]], 0)] = 0.0
+    assert st(rp, c, dv) == "BAR_ERR_ZERO_DIAG"
+    nv = v.copy(); nv[7] = np.nan
+    assert st(rp, c, nv) == "BAR_ERR_NONFINITE"
+    assert st(rp, c, v, R=0) == "BAR_ERR_INVALID_ARG"
+    assert st(rp, c, v, R=bar.MAX_ROWS_PER_BLOCK + 1) == "BAR_ERR_INVALID_ARG"
+    # missing diagonal in row 0
+    D = A.to_dense(); D[0, 0] = 0
+    nz = [np.nonzero(D[i])[0] for i in range(64)]
+    rp2 = np.concatenate([[0], np.cumsum([len(z) for z in nz])]).astype(np.int32)
+    c2 = np.concatenate(nz).astype(np.int32)
+    v2 = np.concatenate([D[i, z] for i, z in enumerate(nz)])
+    assert st(rp2, c2, v2) == "BAR_ERR_BAD_CSR"
+
+
+def test_solve_arg_errors(bar):
+    import torch
+
+    A = W.trefethen(100)
+    M = bar.Matrix.from_csr(A, 32)
+    b = torch.ones(100, dtype=torch.float64, device="cuda")
+    for kw in ({"k": 0, "mode": "async"}, {"tol": -1.0}, {"tol": float("nan")}, {"max_global_iters": -1}):
+        args = dict(k=5, max_global_iters=10, tol=1e-10, mode="sync-block")
+        args.update(kw)
+        with pytest.raises(bar.BarError) as e:
+            M.solve(b, **args)
+        assert e.value.name == "BAR_ERR_INVALID_ARG"
+    bn = b.clone(); bn[3] = float("inf")
+    for mode in ("async", "sync-block", "jacobi"):
+        with pytest.raises(bar.BarError) as e:
+            M.solve(bn, mode=mode)
+        assert e.value.name == "BAR_ERR_NONFINITE"
+
+
+# ------------------------------------------------------------------ residual
+@pytest.mark.parametrize("name", list(MATS))
+@pytest.mark.parametrize("R", [1, 37, 128, 1000])
+def test_residual_parity(bar, name, R):
+    A = MATS[name]()
+    rng = np.random.default_rng(R)
+    x = rng.standard_normal(A.n)
+    b = rng.standard_normal(A.n)
+    M = bar.Matrix.from_csr(A, R)
+    r, bn = M.residual(_dev(b), _dev(x))
+    ref = O.residual_norm(A, b, x)
+    assert abs(r - ref) <= 1e-13 * ref
+    assert abs(bn - O.norm2(b)) <= 1e-14 * bn
+    # host pointers (end-to-end path) give the same bits
+    r2, bn2 = M.residual(b, x)
+    assert r2 == r and bn2 == bn
+
+
+# ------------------------------------------------------------------ iterate-by-iterate
+@pytest.mark.parametrize("name", list(MATS))
+@pytest.mark.parametrize("mode,k,R", [("jacobi", 1, 128), ("sync-block", 1, 128), ("sync-block", 2, 100),
+                                      ("sync-block", 5, 128), ("sync-block", 5, 448), ("sync-block", 9, 1024),
+                                      ("sync-block", 3, 1), ("sync-block", 5, 8192), ("sync-block", 4, 4000)])
+def test_iterates_match_oracle(bar, name, mode, k, R):
+    A = MATS[name]()
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(1).uniform(-1, 1, A.n)
+    checks = [1, 2, 3, 7, 15]
+    ref = x0.copy()
+    refs = {}
+    for m in range(1, max(checks) + 1):
+        ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        refs[m] = ref
+    for m in checks:
+        x, info = _solve(bar, A, b, R, k, mode, m, 0.0, x0)
+        assert info["iters"] == m and info["converged"] == 0
+        _close(x, refs[m])
+        assert abs(info["rel_res"] - O.rel_res(A, b, refs[m])) <= 1e-9 * info["rel_res"] + 1e-15
+
+
+@pytest.mark.parametrize("name,mode,k,R", [("tref2000", "jacobi", 1, 128), ("tref2000", "sync-block", 5, 128),
+                                           ("tref2000", "sync-block", 9, 128), ("fv1", "sync-block", 5, 128),
+                                           ("fv1", "sync-block", 5, 448), ("fv1", "jacobi", 1, 448),
+                                           ("s7_m12", "sync-block", 2, 288), ("rand", "sync-block", 5, 256)])
+def test_iteration_count_and_solution(bar, name, mode, k, R):
+    """Same stopping iteration as the oracle (O5), same returned iterate to 1e-12."""
+    A = MATS[name]()
+    b = np.ones(A.n)
+    meth = O.JACOBI if mode == "jacobi" else O.BLOCK_JACOBI
+    r = O.solve(A, b, method=meth, R=R, k=k, tol=1e-10)
+    x, info = _solve(bar, A, b, R, k, mode, 20000, 1e-10)
+    assert info["converged"] == 1 and info["iters"] == r.iters
+    assert info["rel_res"] <= 1e-10
+    _close(x, r.x)
+
+
+def test_dyadic_bitwise(bar):
+    """Exact dyadic iterates: GPU == oracle bit for bit, any order/FMA."""
+    A = W.dyadic_stencil9_2d(40, p=4)
+    b = (np.arange(A.n) % 5 - 2).astype(float)
+    for mode, k, R in [("jacobi", 1, 64), ("sync-block", 3, 64), ("sync-block", 2, 100)]:
+        for m in (1, 3, 6):
+            x, _ = _solve(bar, A, b, R, k, mode, m, 0.0)
+            ref = np.zeros(A.n)
+            for _ in range(m):
+                ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+            assert np.array_equal(x, ref)
+
+
+def test_sync_modes_bitwise_reproducible(bar):
+    A = W.trefethen(20000)
+    b = np.ones(A.n)
+    for mode in ("sync-block", "jacobi"):
+        x1, i1 = _solve(bar, A, b, 128, 5, mode, 20000, 1e-10)
+        x2, i2 = _solve(bar, A, b, 128, 5, mode, 20000, 1e-10)
+        assert np.array_equal(x1, x2) and i1["iters"] == i2["iters"] and i1["rel_res"] == i2["rel_res"]
+
+
+def test_host_pointers_end_to_end(bar):
+    """The end-to-end path (host b/x0/x, copies inside the call) gives the device path's bits."""
+    import torch
+
+    A = W.stencil9_2d(98)
+    M = bar.Matrix.from_csr(A, 448)
+    b = np.ones(A.n)
+    xh = np.empty(A.n)
+    _, ih = M.solve(b, None, xh, k=5, mode="sync-block")
+    xd, idd = M.solve(_dev(b), None, None, k=5, mode="sync-block")
+    torch.cuda.synchronize()
+    assert np.array_equal(xh, xd.cpu().numpy()) and ih["iters"] == idd["iters"]
+    # x may alias x0
+    x = _dev(np.zeros(A.n))
+    M.solve(_dev(b), x, x, k=5, mode="sync-block")
+    assert np.array_equal(x.cpu().numpy(), xh)
+
+
+# ------------------------------------------------------------------ special cases
+def test_b_zero_and_converged_start(bar):
+    A = W.trefethen(500)
+    x, info = _solve(bar, A, np.zeros(500), 128, 5, "async", 100, 1e-10, x0=np.ones(500))
+    assert info["iters"] == 0 and info["converged"] and np.all(x == 0)
+    xs = np.linalg.solve(A.to_dense(), np.ones(500))
+    for mode in ("async", "sync-block", "jacobi"):
+        x, info = _solve(bar, A, np.ones(500), 128, 5, mode, 100, 1e-10, x0=xs)
+        assert info["iters"] == 0 and info["converged"] and np.array_equal(x, xs)
+
+
+@pytest.mark.parametrize("mode", ["async", "sync-block", "jacobi"])
+def test_fixed_point_invariant(bar, mode):
+    """Starting at x* with tol = 0, every mode (async included) stays at x* (P7)."""
+    A = W.trefethen(2000)
+    b = np.ones(A.n)
+    xs = np.linalg.solve(A.to_dense(), b)
+    x, info = _solve(bar, A, b, 128, 5, mode, 12, 0.0, x0=xs)
+    assert info["iters"] == 12
+    assert np.abs(x - xs).max() <= 1e-14 * np.abs(xs).max() * 10
+
+
+@pytest.mark.parametrize("mode", ["async", "sync-block", "jacobi"])
+def test_divergence(bar, mode):
+    """rho(B) = 1.8 > 1 (P:697 analogue): BAR_ERR_DIVERGED."""
+    Ad = np.full((3, 3), 0.9) + 0.1 * np.eye(3)
+    A = W.CSR(3, np.array([0, 3, 6, 9], dtype=np.int32), np.tile(np.arange(3, dtype=np.int32), 3), Ad.ravel())
+    M = bar.Matrix.from_csr(A, 1)
+    b = _dev(np.ones(3))
+    _, info = M.solve(b, k=1, mode=mode, raise_on_error=False)
+    assert info["status"] == "BAR_ERR_DIVERGED"
+
+
+# ------------------------------------------------------------------ async outcome
+@pytest.mark.parametrize("name,k,R,envelope", [("tref2000", 5, 128, (15, 35)), ("tref2000", 1, 128, (60, 160)),
+                                               ("fv1", 5, 128, (40, 110)), ("fv1", 2, 448, (30, 120)),
+                                               ("rand", 5, 256, (2, 200)), ("s7_m12", 9, 288, (2, 200))])
+def test_async_outcome(bar, name, k, R, envelope):
+    """async-(k): exact rel_res <= 1e-10, x within 1e-8 (relative) of the direct solve,
+    iteration count inside the envelope around the oracle's sync-block count (P5, Table 3)."""
+    A = MATS[name]()
+    b = np.ones(A.n)
+    xs = np.linalg.solve(A.to_dense(), b)
+    x, info = _solve(bar, A, b, R, k, "async", 20000, 1e-10)
+    assert info["converged"] == 1 and info["rel_res"] <= 1e-10
+    assert O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+    assert np.abs(x - xs).max() <= 1e-8 * np.abs(xs).max()
+    assert envelope[0] <= info["iters"] <= envelope[1], info["iters"]
+
+
+def test_siam_constant_async(bar, golden):
+    """Trefethen_20000, b = e_1: x_1 = (A^-1)_11 = 0.7250783462684011674...."""
+    ref = float(golden("siam_trefethen20000_a11.txt")[0][0])
+    A = W.trefethen(20000)
+    b = np.zeros(A.n)
+    b[0] = 1.0
+    for mode in ("async", "sync-block"):
+        x, info = _solve(bar, A, b, 128, 5, mode, 20000, 1e-13)
+        assert info["converged"] and abs(x[0] - ref) < 1e-11
