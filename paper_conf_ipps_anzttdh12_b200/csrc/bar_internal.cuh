@@ -5,9 +5,9 @@
 //   * each subdomain is cut into slices of 32 consecutive rows (one warp, lane = row);
 //     slice s = l*SPB + j (SPB = ceil(R/32)) holds rows TS + 32 j + lane;
 //   * a slice stores its rows' entries column-major (entry e of lane t at ptr[s] + 32 e + t),
-//     first the `wl` LOCAL entries (column inside J_l, stored as the local index col - TS,
-//     the diagonal always local entry 0) and then the `wo` OFF-BLOCK entries (global column);
-//     shorter rows are padded with value 0 and a harmless column (their own row).
+//     first the `wo` OFF-BLOCK entries (global column) and then the `wl` LOCAL entries (column
+//     inside J_l, stored as the local index col - TS, the diagonal always the first local entry
+//     e = wo); shorter rows are padded with value 0 and a harmless column (their own row).
 // So one warp-wide load of entry e is a single coalesced 256 B (values) / 128 B (columns)
 // transaction, the local/off-block split of Alg. 1 costs nothing at run time,
 // and the diagonal (for D^-1) is found without a search.
@@ -38,6 +38,7 @@ struct DevState {
     double last_rel;        // latest fused relative residual
     double exact_rel;       // latest standalone residual (bar_residual / confirmation)
     double exact_ss;        // its sum of squares
+    unsigned long long work;// async work queue: next subdomain to claim in this launch
 };
 
 struct Layout {
@@ -49,6 +50,8 @@ struct Layout {
     int64_t entries = 0;        // padded entries
     int64_t local_entries = 0;
     int max_wl = 0, max_wo = 0;
+    int max_w = 0;              // widest slice: max over slices of wl + wo
+    int sms = 148;              // SMs of the device (persistent grids)
     // device arrays
     double *val = nullptr;      // [entries]
     int32_t *col = nullptr;     // [entries]
@@ -102,6 +105,7 @@ struct SweepArgs {
     double *hist;  // nullable device array: hist[m-1] = rel_res(x^(m-1)) (sync modes)
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
+int64_t rowwise_grid(const Layout &L);
 cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st);
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state,
                             double *partials, cudaStream_t st);

@@ -82,9 +82,10 @@ __global__ void k_slice_widths(int64_t nslices, int64_t n, int32_t R, int32_t sp
     }
 }
 
-// Per (slice, lane): write the lane's column of the slice — diagonal first, then the other
-// local entries ascending (local index), then off-block entries ascending (global index),
-// then padding (value 0, own row).
+// Per (slice, lane): write the lane's column of the slice — first the off-block entries
+// ascending (global index), then the diagonal, then the other local entries ascending (local
+// index), then padding (value 0, own row). Off-block first means one ascending pass over a row
+// produces s_i = b_i - sum_off a_ij x_j before the local part starts (Alg. 1 line 3).
 __global__ void k_fill(int64_t nslices, int64_t n, int32_t R, int32_t spb, const int32_t *__restrict__ rowptr,
                        const int32_t *__restrict__ col, const double *__restrict__ val,
                        const int64_t *__restrict__ sptr, const int32_t *__restrict__ sw,
@@ -99,40 +100,38 @@ __global__ void k_fill(int64_t nslices, int64_t n, int32_t R, int32_t spb, const
     int wl = sw[s] & 0xffff, wo = sw[s] >> 16;
     int64_t base = sptr[s] + lane;
     int64_t TE = min(TS + (int64_t)R, n);
-    int32_t own_loc = (int32_t)(row - TS);
+    int32_t own_loc = valid ? (int32_t)(row - TS) : 0;
     int32_t own_glb = (int32_t)(valid ? row : TS);
     int el = 0, eo = 0;
     if (valid) {
         int32_t a = rowptr[row], e = rowptr[row + 1];
-        for (int32_t p = a; p < e; ++p)  // diagonal -> local entry 0
+        for (int32_t p = a; p < e; ++p)  // diagonal -> first local entry
             if (col[p] == row) {
-                oval[base] = val[p];
-                ocol[base] = own_loc;
+                oval[base + (int64_t)wo * kSlice] = val[p];
+                ocol[base + (int64_t)wo * kSlice] = own_loc;
                 el = 1;
             }
         for (int32_t p = a; p < e; ++p) {
             int64_t c = col[p];
             if (c == row) continue;
             if (c >= TS && c < TE) {
-                oval[base + (int64_t)el * kSlice] = val[p];
-                ocol[base + (int64_t)el * kSlice] = (int32_t)(c - TS);
+                oval[base + (int64_t)(wo + el) * kSlice] = val[p];
+                ocol[base + (int64_t)(wo + el) * kSlice] = (int32_t)(c - TS);
                 ++el;
             } else {
-                oval[base + (int64_t)(wl + eo) * kSlice] = val[p];
-                ocol[base + (int64_t)(wl + eo) * kSlice] = (int32_t)c;
+                oval[base + (int64_t)eo * kSlice] = val[p];
+                ocol[base + (int64_t)eo * kSlice] = (int32_t)c;
                 ++eo;
             }
         }
-    } else {
-        own_loc = 0;
-    }
-    for (; el < wl; ++el) {
-        oval[base + (int64_t)el * kSlice] = 0.0;
-        ocol[base + (int64_t)el * kSlice] = own_loc;
     }
     for (; eo < wo; ++eo) {
-        oval[base + (int64_t)(wl + eo) * kSlice] = 0.0;
-        ocol[base + (int64_t)(wl + eo) * kSlice] = own_glb;
+        oval[base + (int64_t)eo * kSlice] = 0.0;
+        ocol[base + (int64_t)eo * kSlice] = own_glb;
+    }
+    for (; el < wl; ++el) {
+        oval[base + (int64_t)(wo + el) * kSlice] = 0.0;
+        ocol[base + (int64_t)(wo + el) * kSlice] = own_loc;
     }
 }
 
@@ -186,6 +185,7 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     int64_t *d_sum = nullptr;
     int64_t h_tot[2] = {0, 0};
     int h_w[2] = {0, 0};
+    int64_t h_maxsz = 0;
 
     L.n = n;
     L.nnz = nnz;
@@ -227,6 +227,8 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
     BAR_CK(cub::DeviceReduce::Max(nullptr, tmp2, nloc, (int32_t *)d_sum, n, st));
     if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
+    BAR_CK(cub::DeviceReduce::Max(nullptr, tmp2, ssize, d_sum, nsl, st));
+    if (tmp2 > tmp_bytes) tmp_bytes = tmp2;
     BAR_ALLOC(cudaMalloc(&tmp, tmp_bytes));
     BAR_CK(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, ssize, L.sptr, nsl + 1, st));
     BAR_CK(cudaMemcpyAsync(&h_tot[0], L.sptr + nsl, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
@@ -241,8 +243,19 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
         tb = tmp_bytes;
         BAR_CK(cub::DeviceReduce::Max(tmp, tb, noff, (int32_t *)d_sum, n, st));
         BAR_CK(cudaMemcpyAsync(&h_w[1], d_sum, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+        BAR_CK(cudaStreamSynchronize(st));
+        tb = tmp_bytes;
+        BAR_CK(cub::DeviceReduce::Max(tmp, tb, ssize, d_sum, nsl, st));
+        BAR_CK(cudaMemcpyAsync(&h_maxsz, d_sum, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
     }
     BAR_CK(cudaStreamSynchronize(st));
+    L.max_w = (int)(h_maxsz / kSlice);
+    {
+        int dev = 0, sms = 0;
+        if (cudaGetDevice(&dev) == cudaSuccess &&
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && sms > 0)
+            L.sms = sms;
+    }
     L.entries = h_tot[0];
     L.local_entries = h_tot[1];
     L.max_wl = h_w[0];

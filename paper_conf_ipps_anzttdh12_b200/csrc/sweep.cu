@@ -1,21 +1,26 @@
 // sweep.cu — the hot path: block-asynchronous relaxation sweeps on sm_100a.
 //
-//   k_block<MAXR, ASYNC>  one thread block per subdomain J_l (Alg. 1):
+//   k_block<ASYNC, STAGE>  one thread block per subdomain J_l (Alg. 1):
 //       a2/a3  read x "as it stands" (ASYNC: relaxed gpu-scope loads of the live in-place x,
 //              eq. 3's shift function; SYNC: x^(m) through the read-only path) and form the
 //              off-block part s_i = b_i - sum_{j notin J_l} a_ij x_j once (Alg. 1 line 3)
 //       a4     k local Jacobi sweeps on shared-memory copies y of x_J (Alg. 1 lines 4-8,
-//              double-buffered, CTA barrier between sweeps), in the residual-correction form
-//              of eq. 4: y_i <- y_i + (s_i - sum_{j in J_l} a_ij y_j) / a_ii
+//              double-buffered, CTA barrier between sweeps). The first sweep uses the
+//              residual-correction form of eq. 4, y_i <- y_i + (s_i - sum_{j in J_l}
+//              a_ij y_j) / a_ii; sweeps 2..k the direct form of Alg. 1 line 6 with the block's
+//              local entries staged in shared memory (1/a_ii in the diagonal's slot)
 //       a5     the first sweep's correction numerator IS r_i = (b - A x)_i, so the l2 residual
 //               is fused: per-block sum of squares -> fixed-order last-block reduction
 //       a6     write y^k back (x_next for sync-block; in place with relaxed stores for async)
-//   k_jacobi  eq. 2 in the same correction form, warp per 32-row slice, residual fused.
-//   k_residual  standalone ||b - A x||_2 and ||b||_2 (bar_residual, async confirmation).
+//   k_rowwise<false>  eq. 2 in the same correction form, warp per 32-row slice, residual fused.
+//   k_rowwise<true>  standalone ||b - A x||_2 and ||b||_2 (bar_residual, async confirmation).
 //
 // Every kernel is HBM-bound (about 0.17 flop/byte): no tensor cores. Matrix entries are read
 // with coalesced warp-wide loads from the sliced layout (bar_internal.cuh).
+#include <cstdlib>
+
 #include "bar_internal.cuh"
+#include "tma.cuh"
 
 namespace bar {
 namespace {
@@ -36,9 +41,13 @@ struct KP {
     DevState *state;
     double *partials;  // 2 doubles per block: sum r_i^2, sum b_i^2
     double *hist;
+    int wlmax;
+    int wmax;  // widest slice (local + off-block entries)
 };
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
+
+constexpr size_t kSmemBudget = 200 * 1024;  // dynamic smem per block; leaves room for static scratch
 
 template <bool ASYNC>
 __device__ __forceinline__ double ldx(const double *p) {
@@ -117,6 +126,7 @@ __device__ __forceinline__ void reduce_finalize(double rr, double bb, const KP &
     }
     DevState *S = p.state;
     S->counter = 0;
+    S->work = 0;
     double bn = sqrt(bsq);
     S->bnorm = bn;
     if (KIND == kResidual) {
@@ -142,71 +152,215 @@ __device__ __forceinline__ void reduce_finalize(double rr, double bb, const KP &
     }
 }
 
-template <int MAXR, bool ASYNC>
+constexpr int U = 4;  // stored entries of a row loaded together (loads in flight per thread)
+
+// One ascending pass over a row's stored entries — the off-block entries first, then the local
+// ones with the diagonal first (layout.cu) — with U loads in flight per chunk:
+//   s    = b_i - sum_{j notin J} a_ij x_j          (Alg. 1 line 3, x "as it stands")
+//   r    = s - sum_{j in J} a_ij y_j               (= (b - A x)_i when y = x_J: the residual, a5)
+//   dinv = 1 / a_ii
+// LOCAL_SMEM: local columns index y (shared memory); otherwise y points at x + TS (global).
+// STAGE: copy the local entries into shared memory for sweeps 2..k (a4).
+template <bool ASYNC, bool LOCAL_SMEM, bool STAGE>
+__device__ __forceinline__ void row_pass(const double *__restrict__ v, const int32_t *__restrict__ c, int wo, int w,
+                                         const double *x, const double *y, double bi, double &s, double &r,
+                                         double &dinv, double *sv, int32_t *sc, int sstride) {
+    double acc = bi;
+    s = bi;
+    dinv = 0.0;
+    for (int e0 = 0; e0 < w; e0 += U) {
+        double a[U], xv[U];
+        int ci[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            if (e0 + u < w) {
+                a[u] = __ldg(v + (e0 + u) * kSlice);
+                ci[u] = __ldg(c + (e0 + u) * kSlice);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int e = e0 + u;
+            if (e < w) {
+                if (e < wo) xv[u] = ldx<ASYNC>(x + ci[u]);
+                else if (LOCAL_SMEM) xv[u] = y[ci[u]];
+                else xv[u] = ldx<ASYNC>(y + ci[u]);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int e = e0 + u;
+            if (e < w) {
+                if (e == wo) {
+                    s = acc;
+                    dinv = 1.0 / a[u];
+                }
+                acc -= a[u] * xv[u];
+                if (STAGE && e >= wo) {  // slot 0 (the diagonal) keeps 1/a_ii for the direct form
+                    sv[(e - wo) * sstride] = e == wo ? dinv : a[u];
+                    sc[(e - wo) * sstride] = ci[u];
+                }
+            }
+        }
+    }
+    r = acc;
+}
+
+template <bool ASYNC, bool STAGE>
 __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
     if (*(volatile int *)&p.state->stop) return;
-    extern __shared__ double sm[];
+    extern __shared__ __align__(16) unsigned char smraw[];
     const int R = p.R;
-    double *y0 = sm;
-    double *y1 = sm + R;
+    const int sstride = p.spb * kSlice;
+    double *y0 = reinterpret_cast<double *>(smraw);  // y^t, double-buffered
+    double *y1 = y0 + R;
+    double *ss = y1 + R;                              // s_i (off-block part, frozen)
+    double *sv = ss + R;                              // [wlmax][spb*32] staged local values
+    int32_t *sc = reinterpret_cast<int32_t *>(sv + (STAGE ? (size_t)p.wlmax * sstride : 0));  // local cols
     const int64_t l = blockIdx.x;
     const int64_t TS = l * (int64_t)R;
     const int nrows = (int)min((int64_t)R, p.n - TS);
     const int nsl = (nrows + kSlice - 1) / kSlice;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, W = blockDim.x >> 5;
+    const int64_t sl0 = l * p.spb;
 
     // y^0 = x_J (Alg. 1: "read x from global memory")
     for (int i = threadIdx.x; i < nrows; i += blockDim.x) y0[i] = ldx<ASYNC>(p.x_in + TS + i);
     __syncthreads();
 
-    double s[MAXR], dinv[MAXR];
     double rr = 0.0, bb = 0.0;
-#pragma unroll
-    for (int r = 0; r < MAXR; ++r) {
-        const int j = warp + r * W;
+    for (int j = warp; j < nsl; j += W) {
         const int loc = j * kSlice + lane;
-        s[r] = 0.0;
-        dinv[r] = 0.0;
-        if (j < nsl && loc < nrows) {
-            const int64_t sl = l * p.spb + j;
-            const int64_t base = p.sptr[sl] + lane;
-            const int w = p.sw[sl];
+        if (loc < nrows) {
+            const int64_t base = p.sptr[sl0 + j] + lane;
+            const int w = p.sw[sl0 + j];
             const int wl = w & 0xffff, wo = w >> 16;
             const double bi = p.b[TS + loc];
             bb += bi * bi;
-            // off-block part, x as it stands (a3)
-            double acc = bi;
-            const double *vo = p.val + base + (int64_t)wl * kSlice;
-            const int32_t *co = p.col + base + (int64_t)wl * kSlice;
-            for (int e = 0; e < wo; ++e) acc -= __ldg(vo + e * kSlice) * ldx<ASYNC>(p.x_in + __ldg(co + e * kSlice));
-            s[r] = acc;
-            const double *vl = p.val + base;
-            const int32_t *cl = p.col + base;
-            dinv[r] = 1.0 / __ldg(vl);  // local entry 0 is a_ii
-            // first local sweep; its correction numerator is the residual r_i (a5)
-            for (int e = 0; e < wl; ++e) acc -= __ldg(vl + e * kSlice) * y0[__ldg(cl + e * kSlice)];
-            rr += acc * acc;
-            y1[loc] = y0[loc] + dinv[r] * acc;
+            double s, res, dinv;
+            // a3 + first local sweep (its correction numerator is the residual, a5)
+            row_pass<ASYNC, true, STAGE>(p.val + base, p.col + base, wo, wo + wl, p.x_in, y0, bi, s, res, dinv,
+                                         sv + loc, sc + loc, sstride);
+            rr += res * res;
+            ss[loc] = s;
+            y1[loc] = y0[loc] + dinv * res;
         }
     }
     __syncthreads();
-    // sweeps 2..k with the off-block part frozen
+    // a4: sweeps 2..k on the subdomain with the off-block part frozen, in the direct
+    // form of Alg. 1 line 6: y_i <- (s_i - sum_{j in J, j != i} a_ij y_j) / a_ii
+    for (int t = 1; t < p.k; ++t) {
+        const double *yi = (t & 1) ? y1 : y0;
+        double *yo = (t & 1) ? y0 : y1;
+        for (int j = warp; j < nsl; j += W) {
+            const int loc = j * kSlice + lane;
+            if (loc < nrows) {
+                const int w = p.sw[sl0 + j];
+                const int wl = w & 0xffff;
+                double acc = ss[loc];
+                if (STAGE) {
+                    const double *lv = sv + loc;
+                    const int32_t *lc = sc + loc;
+#pragma unroll 4
+                    for (int e = 1; e < wl; ++e) acc -= lv[e * sstride] * yi[lc[e * sstride]];
+                    yo[loc] = lv[0] * acc;
+                } else {
+                    const int64_t base = p.sptr[sl0 + j] + lane + (int64_t)(w >> 16) * kSlice;
+                    const double *vl = p.val + base;
+                    const int32_t *cl = p.col + base;
+#pragma unroll 4
+                    for (int e = 1; e < wl; ++e) acc -= __ldg(vl + e * kSlice) * yi[__ldg(cl + e * kSlice)];
+                    yo[loc] = acc / __ldg(vl);
+                }
+            }
+        }
+        __syncthreads();
+    }
+    // a6: write back
+    const double *yk = (p.k & 1) ? y1 : y0;
+    for (int i = threadIdx.x; i < nrows; i += blockDim.x) stx<ASYNC>(p.x_out + TS + i, yk[i]);
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
+// Register-resident variant of k_block for subdomains of at most 32*32*RPT rows whose rows have
+// at most WLR local entries: each thread keeps its RPT rows' local entries (values and local
+// columns) in registers, so sweeps 2..k read only y from shared memory, and the shared-memory
+// footprint (y^t double buffer, 16 B/row) lets two or more blocks share an SM — one block's HBM
+// phase overlaps another's local sweeps.
+template <bool ASYNC, int WLR, int RPT>
+__global__ void __launch_bounds__(1024, 1) k_reg(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(16) unsigned char smraw[];
+    const int R = p.R;
+    double *y0 = reinterpret_cast<double *>(smraw);
+    double *y1 = y0 + R;
+    const int64_t l = blockIdx.x;
+    const int64_t TS = l * (int64_t)R;
+    const int nrows = (int)min((int64_t)R, p.n - TS);
+    const int nsl = (nrows + kSlice - 1) / kSlice;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, W = blockDim.x >> 5;
+    const int64_t sl0 = l * p.spb;
+    constexpr int NP = WLR / 2;  // local columns packed two per register (R <= 65536)
+
+    for (int i = threadIdx.x; i < nrows; i += blockDim.x) y0[i] = ldx<ASYNC>(p.x_in + TS + i);
+    __syncthreads();
+
+    double lv[RPT][WLR];   // lv[r][0] = 1/a_ii, lv[r][e>0] = local off-diagonal a_ij
+    uint32_t lc[RPT][NP];  // local column e in 16-bit half (e & 1) of lc[r][e >> 1]
+    double s[RPT];
+    bool ok[RPT];
+    double rr = 0.0, bb = 0.0;
+#pragma unroll
+    for (int r = 0; r < RPT; ++r) {
+        const int j = warp + r * W;
+        const int loc = j * kSlice + lane;
+        ok[r] = j < nsl && loc < nrows;
+        s[r] = 0.0;
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) lv[r][e] = 0.0;
+#pragma unroll
+        for (int e = 0; e < NP; ++e) lc[r][e] = 0;
+        if (ok[r]) {
+            const int64_t base = p.sptr[sl0 + j] + lane;
+            const int w = p.sw[sl0 + j];
+            const int wl = w & 0xffff, wo = w >> 16;
+            const double *vl = p.val + base + (int64_t)wo * kSlice;
+            const int32_t *cl = p.col + base + (int64_t)wo * kSlice;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[r][e] = __ldg(vl + e * kSlice);
+                    lc[r][e >> 1] |= (uint32_t)__ldg(cl + e * kSlice) << (16 * (e & 1));
+                }
+            }
+            const double bi = p.b[TS + loc];
+            bb += bi * bi;
+            double acc, sdum, ddum;
+            // a3: off-block part, x as it stands
+            row_pass<ASYNC, false, false>(p.val + base, p.col + base, wo, wo, p.x_in, nullptr, bi, sdum, acc, ddum,
+                                          nullptr, nullptr, 0);
+            s[r] = acc;
+            // first local sweep = residual (a5)
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[r][e] * y0[(lc[r][e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[r][0] = 1.0 / lv[r][0];
+            rr += acc * acc;
+            y1[loc] = y0[loc] + lv[r][0] * acc;
+        }
+    }
+    __syncthreads();
+    // a4: sweeps 2..k, direct form, off-block part frozen
     for (int t = 1; t < p.k; ++t) {
         const double *yi = (t & 1) ? y1 : y0;
         double *yo = (t & 1) ? y0 : y1;
 #pragma unroll
-        for (int r = 0; r < MAXR; ++r) {
-            const int j = warp + r * W;
-            const int loc = j * kSlice + lane;
-            if (j < nsl && loc < nrows) {
-                const int64_t sl = l * p.spb + j;
-                const int64_t base = p.sptr[sl] + lane;
-                const int wl = p.sw[sl] & 0xffff;
-                const double *vl = p.val + base;
-                const int32_t *cl = p.col + base;
+        for (int r = 0; r < RPT; ++r) {
+            if (ok[r]) {
+                const int loc = (warp + r * W) * kSlice + lane;
                 double acc = s[r];
-                for (int e = 0; e < wl; ++e) acc -= __ldg(vl + e * kSlice) * yi[__ldg(cl + e * kSlice)];
-                yo[loc] = yi[loc] + dinv[r] * acc;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[r][e] * yi[(lc[r][e >> 1] >> (16 * (e & 1))) & 0xffff];
+                yo[loc] = lv[r][0] * acc;
             }
         }
         __syncthreads();
@@ -214,6 +368,315 @@ __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
     const double *yk = (p.k & 1) ? y1 : y0;
     for (int i = threadIdx.x; i < nrows; i += blockDim.x) stx<ASYNC>(p.x_out + TS + i, yk[i]);
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
+// Bytes of one warp's slice buffer (values + columns) for slices of width <= wmax entries.
+__host__ __device__ __forceinline__ uint32_t slice_buf_bytes(int wmax) {
+    return (uint32_t)wmax * kSlice * (sizeof(double) + sizeof(int32_t));
+}
+
+// Lane 0 of a warp: stream slice `sl` (width w) into buf with two bulk copies completing on bar.
+__device__ __forceinline__ void issue_slice(const KP &p, int64_t sl, int w, unsigned char *buf, uint64_t *bar,
+                                            int wmax) {
+    const int64_t e0 = p.sptr[sl];
+    const uint32_t vb = (uint32_t)w * kSlice * sizeof(double), cb = (uint32_t)w * kSlice * sizeof(int32_t);
+    mbar_arrive_expect_tx(bar, vb + cb);
+    bulk_g2s(buf, p.val + e0, vb, bar);
+    bulk_g2s(buf + (size_t)wmax * kSlice * sizeof(double), p.col + e0, cb, bar);
+}
+
+// k_reg with the slice stream moved off the register file: each warp bulk-copies (TMA) its
+// slice's values and columns into shared memory before anything else, the block then loads
+// y^0 = x_J while the copies are in flight, and every lane reads its row's entries from
+// shared memory (conflict-free: lane-contiguous). Local entries then live in registers for
+// the k sweeps; only the dependent x gathers of the off-block part touch L2/HBM.
+template <bool ASYNC, int WLR>
+__global__ void __launch_bounds__(1024, 1) k_reg_tma(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[32];
+    const int R = p.R;
+    const int wmax = p.wmax;
+    const int64_t l = blockIdx.x;
+    const int64_t TS = l * (int64_t)R;
+    const int nrows = (int)min((int64_t)R, p.n - TS);
+    const int nsl = (nrows + kSlice - 1) / kSlice;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t sl = l * p.spb + warp;
+    unsigned char *buf = smraw + (size_t)warp * slice_buf_bytes(wmax);
+    double *y0 = reinterpret_cast<double *>(smraw + (size_t)(blockDim.x >> 5) * slice_buf_bytes(wmax));
+    double *y1 = y0 + R;
+    const bool has_slice = warp < nsl;
+    int w = 0, wo = 0, wl = 0;
+    if (has_slice) {
+        const int sw = p.sw[sl];
+        wl = sw & 0xffff;
+        wo = sw >> 16;
+        w = wl + wo;
+        if (lane == 0) {
+            mbar_init(&bars[warp], 1);
+            fence_mbar_init();
+            issue_slice(p, sl, w, buf, &bars[warp], wmax);
+        }
+    }
+    // y^0 = x_J while the slice streams in (Alg. 1: "read x from global memory")
+    for (int i = threadIdx.x; i < nrows; i += blockDim.x) y0[i] = ldx<ASYNC>(p.x_in + TS + i);
+    __syncthreads();
+
+    constexpr int NP = WLR / 2;
+    double lv[WLR];
+    uint32_t lc[NP];
+    double s = 0.0, rr = 0.0, bb = 0.0;
+    const int loc = warp * kSlice + lane;
+    const bool ok = has_slice && loc < nrows;
+#pragma unroll
+    for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+    for (int e = 0; e < NP; ++e) lc[e] = 0;
+    if (has_slice) {
+        mbar_wait(&bars[warp], 0);
+        const double *sv = reinterpret_cast<const double *>(buf) + lane;
+        const int32_t *sc = reinterpret_cast<const int32_t *>(buf + (size_t)wmax * kSlice * sizeof(double)) + lane;
+        if (ok) {
+            const double bi = p.b[TS + loc];
+            bb = bi * bi;
+            // a3: off-block part with the x gathers batched U at a time
+            double acc = bi;
+            for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+            }
+            s = acc;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[e] = sv[(wo + e) * kSlice];
+                    lc[e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                }
+            }
+            // first local sweep = residual (a5)
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[0] = 1.0 / lv[0];
+            rr = acc * acc;
+            y1[loc] = y0[loc] + lv[0] * acc;
+        }
+    }
+    __syncthreads();
+    // a4: sweeps 2..k, direct form, off-block part frozen
+    for (int t = 1; t < p.k; ++t) {
+        const double *yi = (t & 1) ? y1 : y0;
+        double *yo = (t & 1) ? y0 : y1;
+        if (ok) {
+            double acc = s;
+#pragma unroll
+            for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            yo[loc] = lv[0] * acc;
+        }
+        __syncthreads();
+    }
+    const double *yk = (p.k & 1) ? y1 : y0;
+    for (int i = threadIdx.x; i < nrows; i += blockDim.x) stx<ASYNC>(p.x_out + TS + i, yk[i]);
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
+// Persistent k_reg_tma: block c sweeps subdomains l = c, c + G, c + 2G, ... (G = blocks in the
+// grid) and, while it runs the k local sweeps of subdomain l, the bulk copies of subdomain
+// l + G's slices are already streaming into the other half of a double-buffered slice area —
+// the HBM stream never waits for the on-chip sweeps. One residual reduction
+// per block per launch instead of one per subdomain.
+template <bool ASYNC, int WLR>
+__global__ void __launch_bounds__(1024, 1) k_block_pers(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[2][32];
+    const int R = p.R;
+    const int wmax = p.wmax;
+    const int W = blockDim.x >> 5;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t sbb = slice_buf_bytes(wmax);
+    unsigned char *buf[2] = {smraw + (size_t)warp * sbb, smraw + (size_t)(W + warp) * sbb};
+    double *y0 = reinterpret_cast<double *>(smraw + (size_t)2 * W * sbb);
+    double *y1 = y0 + R;
+    const int64_t G = gridDim.x;
+    const int64_t q = (p.n + R - 1) / R;
+    auto nsl_of = [&](int64_t l) { return (int)((min((int64_t)R, p.n - l * R) + kSlice - 1) / kSlice); };
+    // Subdomain order. Sync-block: static round robin (the per-block partial sums, and so the
+    // residual, are then bitwise reproducible). Async: a device work queue, so subdomains are
+    // claimed in increasing order by whichever block is free — a monotone processing front, which
+    // is what lets later blocks see this iteration's values of earlier ones (eq. 4's shift
+    // s(k+1, j) < 0: the block Gauss-Seidel flavour of P:209).
+    __shared__ long long s_next;
+    if (threadIdx.x == 0) s_next = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)blockIdx.x;
+    __syncthreads();
+    int64_t l = s_next;
+    if (lane == 0) {
+        mbar_init(&bars[0][warp], 1);
+        mbar_init(&bars[1][warp], 1);
+        fence_mbar_init();
+        if (l < q && warp < nsl_of(l)) {
+            const int64_t sl = l * p.spb + warp;
+            const int sw = p.sw[sl];
+            issue_slice(p, sl, (sw & 0xffff) + (sw >> 16), buf[0], &bars[0][warp], wmax);
+        }
+    }
+    constexpr int NP = WLR / 2;
+    double rr = 0.0, bb = 0.0;
+    int i = 0;
+    for (int64_t ln; l < q; l = ln, ++i) {
+        const int st = i & 1;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        if (threadIdx.x == 0) s_next = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)(l + G);
+        __syncthreads();
+        ln = s_next;
+        if (lane == 0 && ln < q && warp < nsl_of(ln)) {  // prefetch the next subdomain's slice
+            fence_proxy_async_smem();
+            const int64_t sl = ln * p.spb + warp;
+            const int sw = p.sw[sl];
+            issue_slice(p, sl, (sw & 0xffff) + (sw >> 16), buf[st ^ 1], &bars[st ^ 1][warp], wmax);
+        }
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) y0[r] = ldx<ASYNC>(p.x_in + TS + r);
+        __syncthreads();
+        double lv[WLR];
+        uint32_t lc[NP];
+        double s = 0.0;
+        const int loc = warp * kSlice + lane;
+        const bool has_slice = warp < nsl;
+        const bool ok = has_slice && loc < nrows;
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+        for (int e = 0; e < NP; ++e) lc[e] = 0;
+        if (has_slice) {
+            const int sw = p.sw[l * p.spb + warp];
+            const int wl = sw & 0xffff, wo = sw >> 16;
+            mbar_wait(&bars[st][warp], (i >> 1) & 1);
+            const double *sv = reinterpret_cast<const double *>(buf[st]) + lane;
+            const int32_t *sc =
+                reinterpret_cast<const int32_t *>(buf[st] + (size_t)wmax * kSlice * sizeof(double)) + lane;
+            if (ok) {
+                const double bi = p.b[TS + loc];
+                bb += bi * bi;
+                double acc = bi;
+                for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                    double xv[2 * U];
+#pragma unroll
+                    for (int u = 0; u < 2 * U; ++u)
+                        if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                    for (int u = 0; u < 2 * U; ++u)
+                        if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+                }
+                s = acc;
+#pragma unroll
+                for (int e = 0; e < WLR; ++e) {
+                    if (e < wl) {
+                        lv[e] = sv[(wo + e) * kSlice];
+                        lc[e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                    }
+                }
+#pragma unroll
+                for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                lv[0] = 1.0 / lv[0];
+                rr += acc * acc;
+                y1[loc] = y0[loc] + lv[0] * acc;
+            }
+        }
+        __syncthreads();
+        for (int t = 1; t < p.k; ++t) {
+            const double *yi = (t & 1) ? y1 : y0;
+            double *yo = (t & 1) ? y0 : y1;
+            if (ok) {
+                double acc = s;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                yo[loc] = lv[0] * acc;
+            }
+            __syncthreads();
+        }
+        const double *yk = (p.k & 1) ? y1 : y0;
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
+        __syncthreads();
+    }
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
+// Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
+// g, g + G, g + 2G, ... (G = warps in the grid) and keeps the next slice's bulk copy in flight
+// (two slice buffers per warp) while computing the current one.
+template <bool RESIDUAL_ONLY>
+__global__ void __launch_bounds__(256, 4) k_rowwise_tma(KP p) {
+    if (!RESIDUAL_ONLY && *(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[8][2];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int wmax = p.wmax;
+    const uint32_t bb_bytes = slice_buf_bytes(wmax);
+    unsigned char *buf[2] = {smraw + (size_t)(2 * warp) * bb_bytes, smraw + (size_t)(2 * warp + 1) * bb_bytes};
+    const int64_t G = (int64_t)gridDim.x * 8;
+    int64_t sl = (int64_t)blockIdx.x * 8 + warp;
+    if (lane == 0) {
+        mbar_init(&bars[warp][0], 1);
+        mbar_init(&bars[warp][1], 1);
+        fence_mbar_init();
+        if (sl < p.nslices) {
+            const int w = p.sw[sl];
+            issue_slice(p, sl, (w & 0xffff) + (w >> 16), buf[0], &bars[warp][0], wmax);
+        }
+    }
+    __syncwarp();
+    double rr = 0.0, bb = 0.0;
+    for (int i = 0; sl < p.nslices; ++i, sl += G) {
+        const int st = i & 1;
+        const int64_t nx = sl + G;
+        if (lane == 0 && nx < p.nslices) {
+            fence_proxy_async_smem();
+            const int w = p.sw[nx];
+            issue_slice(p, nx, (w & 0xffff) + (w >> 16), buf[st ^ 1], &bars[warp][st ^ 1], wmax);
+        }
+        const int sw = p.sw[sl];
+        const int wl = sw & 0xffff, wo = sw >> 16, w = wl + wo;
+        const int64_t l = sl / p.spb;
+        const int64_t TS = l * (int64_t)p.R;
+        const int64_t loc = (sl - l * p.spb) * kSlice + lane;
+        const int64_t row = TS + loc;
+        mbar_wait(&bars[warp][st], (i >> 1) & 1);
+        if (loc < p.R && row < p.n) {
+            const double *sv = reinterpret_cast<const double *>(buf[st]) + lane;
+            const int32_t *sc = reinterpret_cast<const int32_t *>(buf[st] + (size_t)wmax * kSlice * sizeof(double)) + lane;
+            const double bi = p.b[row];
+            bb += bi * bi;
+            double acc = bi, dinv = 0.0;
+            for (int e0 = 0; e0 < w; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u) {
+                    const int e = e0 + u;
+                    if (e < w) xv[u] = __ldg(p.x_in + (e < wo ? 0 : TS) + sc[e * kSlice]);
+                }
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u) {
+                    const int e = e0 + u;
+                    if (e < w) {
+                        const double a = sv[e * kSlice];
+                        if (e == wo) dinv = 1.0 / a;
+                        acc -= a * xv[u];
+                    }
+                }
+            }
+            rr += acc * acc;
+            if (!RESIDUAL_ONLY) p.x_out[row] = __ldg(p.x_in + row) + dinv * acc;
+        }
+        __syncwarp();
+    }
+    reduce_finalize<RESIDUAL_ONLY ? kResidual : kSync>(rr, bb, p);
 }
 
 // Jacobi (eq. 2) and the standalone residual: one warp per 32-row slice, 8 slices per block.
@@ -234,16 +697,11 @@ __global__ void __launch_bounds__(256) k_rowwise(KP p) {
             const int wl = w & 0xffff, wo = w >> 16;
             const double bi = p.b[row];
             bb = bi * bi;
-            double acc = bi;
-            const double *vo = p.val + base + (int64_t)wl * kSlice;
-            const int32_t *co = p.col + base + (int64_t)wl * kSlice;
-            for (int e = 0; e < wo; ++e) acc -= __ldg(vo + e * kSlice) * __ldg(p.x_in + __ldg(co + e * kSlice));
-            const double *vl = p.val + base;
-            const int32_t *cl = p.col + base;
-            const double *xJ = p.x_in + TS;
-            for (int e = 0; e < wl; ++e) acc -= __ldg(vl + e * kSlice) * __ldg(xJ + __ldg(cl + e * kSlice));
-            rr = acc * acc;
-            if (!RESIDUAL_ONLY) p.x_out[row] = __ldg(p.x_in + row) + (1.0 / __ldg(vl)) * acc;
+            double s, res, dinv;
+            row_pass<false, false, false>(p.val + base, p.col + base, wo, wo + wl, p.x_in, p.x_in + TS, bi, s, res,
+                                          dinv, nullptr, nullptr, 0);
+            rr = res * res;
+            if (!RESIDUAL_ONLY) p.x_out[row] = __ldg(p.x_in + row) + dinv * res;
         }
     }
     reduce_finalize<RESIDUAL_ONLY ? kResidual : kSync>(rr, bb, p);
@@ -258,6 +716,7 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->tol = tol;
     S->last_rel = -1.0;
     S->exact_rel = -1.0;
+    S->work = 0;
 }
 
 KP make_kp(const Layout &L) {
@@ -273,35 +732,162 @@ KP make_kp(const Layout &L) {
     return p;
 }
 
-template <int MAXR, bool ASYNC>
+template <bool ASYNC, bool STAGE>
 cudaError_t launch_block_t(const KP &p, int threads, size_t smem, unsigned grid, cudaStream_t st) {
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_block<MAXR, ASYNC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             2 * BAR_MAX_ROWS_PER_BLOCK * (int)sizeof(double));
+    static size_t attr = 0;
+    if (smem > attr) {
+        cudaError_t e =
+            cudaFuncSetAttribute(k_block<ASYNC, STAGE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr_set = true;
+        attr = smem;
     }
-    k_block<MAXR, ASYNC><<<grid, threads, smem, st>>>(p);
+    k_block<ASYNC, STAGE><<<grid, threads, smem, st>>>(p);
     return cudaGetLastError();
 }
 
+
+// Block geometry: one 32-row slice per warp and pass; local entries staged in shared memory
+// when they fit (otherwise re-read through L1/L2 in every sweep).
+template <bool ASYNC, int WLR, int RPT>
+cudaError_t launch_reg_t(const KP &p, const Layout &L, cudaStream_t st) {
+    const int W = (L.spb + RPT - 1) / RPT;
+    k_reg<ASYNC, WLR, RPT><<<(unsigned)L.q, W * kSlice, 2 * (size_t)L.R * sizeof(double), st>>>(p);
+    return cudaGetLastError();
+}
+
+template <bool ASYNC, int RPT>
+cudaError_t launch_reg_w(const KP &p, const Layout &L, cudaStream_t st) {
+    if (L.max_wl <= 4) return launch_reg_t<ASYNC, 4, RPT>(p, L, st);
+    if (L.max_wl <= 6) return launch_reg_t<ASYNC, 6, RPT>(p, L, st);
+    return launch_reg_t<ASYNC, 8, RPT>(p, L, st);
+}
+
+template <bool ASYNC, int WLR>
+cudaError_t launch_reg_tma_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    static size_t attr = 0;
+    if (smem > attr) {
+        cudaError_t e =
+            cudaFuncSetAttribute(k_reg_tma<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr = smem;
+    }
+    k_reg_tma<ASYNC, WLR><<<(unsigned)L.q, L.spb * kSlice, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+// Persistent grid of k_block_pers: every block that fits on the device at once.
+template <bool ASYNC, int WLR>
+int64_t pers_grid(const Layout &L, size_t smem) {
+    static size_t attr = 0;
+    if (smem > attr) {
+        if (cudaFuncSetAttribute(k_block_pers<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+            cudaSuccess)
+            return -1;
+        attr = smem;
+    }
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_block_pers<ASYNC, WLR>, L.spb * kSlice, smem) !=
+            cudaSuccess ||
+        per_sm < 1)
+        per_sm = 1;
+    const int64_t g = (int64_t)per_sm * L.sms;
+    return g < L.q ? g : L.q;
+}
+
+template <bool ASYNC, int WLR>
+cudaError_t launch_pers_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    const int64_t g = pers_grid<ASYNC, WLR>(L, smem);
+    if (g < 0) return cudaGetLastError();
+    k_block_pers<ASYNC, WLR><<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+// Kernel choice for one block-sweep launch (async / sync-block):
+//   k_block_pers  persistent, double-buffered TMA slice stream (default when it fits)
+//   k_reg_tma  subdomains of <= 1024 rows with <= 8 local entries per row (every stencil
+//              config): TMA-streamed slices, register-resident local entries
+//   k_reg      same without TMA (BAR_KERNEL=r, for comparison)
+//   k_block    anything else: local entries staged in shared memory when they fit, else
+//              re-read through L1/L2 each sweep (BAR_KERNEL=s forces it)
 template <bool ASYNC>
-cudaError_t launch_block(const KP &p, const Layout &L, cudaStream_t st) {
-    const int W = L.spb < 32 ? L.spb : 32;
-    const int need = (L.spb + W - 1) / W;
-    const size_t smem = 2 * (size_t)L.R * sizeof(double);
-    const unsigned grid = (unsigned)L.q;
-    if (need <= 1) return launch_block_t<1, ASYNC>(p, W * 32, smem, grid, st);
-    if (need <= 2) return launch_block_t<2, ASYNC>(p, W * 32, smem, grid, st);
-    if (need <= 4) return launch_block_t<4, ASYNC>(p, W * 32, smem, grid, st);
-    return launch_block_t<8, ASYNC>(p, W * 32, smem, grid, st);
+cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
+    const char *kv = getenv("BAR_KERNEL");
+    const char kind = kv ? kv[0] : 't';
+    p.wlmax = L.max_wl;
+    p.wmax = L.max_w;
+    const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
+    const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
+    if (kind == 't' && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
+        if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
+        if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
+        return launch_pers_t<ASYNC, 8>(p, L, pers_smem, st);
+    }
+    if ((kind == 't' || kind == 'n') && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
+        if (L.max_wl <= 4) return launch_reg_tma_t<ASYNC, 4>(p, L, tma_smem, st);
+        if (L.max_wl <= 6) return launch_reg_tma_t<ASYNC, 6>(p, L, tma_smem, st);
+        return launch_reg_tma_t<ASYNC, 8>(p, L, tma_smem, st);
+    }
+    if (kind != 's' && L.spb <= 32 && L.max_wl <= 8) return launch_reg_w<ASYNC, 1>(p, L, st);
+    const size_t row_bytes = 3 * (size_t)L.R * sizeof(double);  // y0, y1, s
+    const size_t stage_bytes = (size_t)L.max_wl * L.spb * kSlice * (sizeof(double) + sizeof(int32_t));
+    const bool stage = row_bytes + stage_bytes <= kSmemBudget;
+    const size_t smem = row_bytes + (stage ? stage_bytes : 0);
+    int W = L.spb < 32 ? L.spb : 32;
+    if (const char *ev = getenv("BAR_WARPS")) {
+        int w = atoi(ev);
+        if (w >= 1 && w <= 32) W = w < L.spb ? w : L.spb;
+    }
+    if (stage) return launch_block_t<ASYNC, true>(p, W * 32, smem, (unsigned)L.q, st);
+    return launch_block_t<ASYNC, false>(p, W * 32, smem, (unsigned)L.q, st);
+}
+
+// Persistent grid for the rowwise kernels: as many 256-thread blocks as fit on the device at
+// once (two slice buffers per warp), capped by the number of 8-slice groups.
+bool rowwise_tma_ok(const Layout &L) { return 16 * (size_t)slice_buf_bytes(L.max_w) <= kSmemBudget; }
+
+template <bool RES>
+cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
+    p.wmax = L.max_w;
+    const char *kv = getenv("BAR_KERNEL");
+    if (!rowwise_tma_ok(L) || (kv && kv[0] == 'r')) {
+        k_rowwise<RES><<<(unsigned)((L.nslices + 7) / 8), 256, 0, st>>>(p);
+        return cudaGetLastError();
+    }
+    const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
+    static size_t attr = 0;
+    if (smem > attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_rowwise_tma<RES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr = smem;
+    }
+    k_rowwise_tma<RES><<<(unsigned)rowwise_grid(L), 256, smem, st>>>(p);
+    return cudaGetLastError();
 }
 
 }  // namespace
 
+int64_t rowwise_grid(const Layout &L) {
+    const int64_t groups = (L.nslices + 7) / 8;
+    if (!rowwise_tma_ok(L)) return groups;
+    const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
+    int a = 0, b = 0;
+    cudaFuncSetAttribute(k_rowwise_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBudget);
+    cudaFuncSetAttribute(k_rowwise_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBudget);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_rowwise_tma<true>, 256, smem) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_rowwise_tma<false>, 256, smem) != cudaSuccess) {
+        cudaGetLastError();
+        a = b = 1;
+    }
+    int64_t per_sm = a < b ? a : b;  // the same grid for both (deterministic reductions)
+    if (per_sm < 1) per_sm = 1;
+    const int64_t g = per_sm * L.sms;
+    return g < groups ? g : groups;
+}
+
 int64_t num_blocks_for(const Layout &L, bar_mode mode) {
-    int64_t rowwise = (L.nslices + 7) / 8;
+    int64_t rowwise = rowwise_grid(L);
+    int64_t legacy = (L.nslices + 7) / 8;
+    if (legacy > rowwise) rowwise = legacy;
     if (mode == BAR_MODE_JACOBI) return rowwise;
     return L.q > rowwise ? L.q : rowwise;
 }
@@ -315,10 +901,7 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.state = a.state;
     p.partials = a.partials;
     p.hist = a.hist;
-    if (mode == BAR_MODE_JACOBI) {
-        k_rowwise<false><<<(unsigned)((a.L->nslices + 7) / 8), 256, 0, st>>>(p);
-        return cudaGetLastError();
-    }
+    if (mode == BAR_MODE_JACOBI) return launch_rowwise<false>(p, *a.L, st);
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
     return launch_block<false>(p, *a.L, st);
 }
@@ -330,8 +913,7 @@ cudaError_t launch_residual(const Layout &L, const double *b, const double *x, D
     p.x_in = x;
     p.state = state;
     p.partials = partials;
-    k_rowwise<true><<<(unsigned)((L.nslices + 7) / 8), 256, 0, st>>>(p);
-    return cudaGetLastError();
+    return launch_rowwise<true>(p, L, st);
 }
 
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st) {
