@@ -204,8 +204,11 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     BAR_ALLOC(dmalloc(&d_err, 1));
     BAR_ALLOC(dmalloc(&ssize, (size_t)nsl + 1));
     BAR_ALLOC(dmalloc(&d_sum, 2));
-    BAR_ALLOC(dmalloc(&L.sptr, (size_t)nsl + 1));
-    BAR_ALLOC(dmalloc(&L.sw, (size_t)nsl));
+    // +4 entries of slack: bulk copies round metadata ranges up to 16 bytes
+    BAR_ALLOC(dmalloc(&L.sptr, (size_t)nsl + 5));
+    BAR_ALLOC(dmalloc(&L.sw, (size_t)nsl + 4));
+    BAR_CK(cudaMemsetAsync(L.sw + nsl, 0, 4 * sizeof(int32_t), st));
+    BAR_CK(cudaMemsetAsync(L.sptr + nsl + 1, 0, 4 * sizeof(int64_t), st));
     BAR_CK(cudaMemsetAsync(d_err, 0, sizeof(int), st));
 
     k_validate_count<<<(unsigned)((n + TB - 1) / TB), TB, 0, st>>>(n, nnz, d_rowptr, d_col, d_val, R, nloc, noff,

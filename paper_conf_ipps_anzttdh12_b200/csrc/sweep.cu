@@ -48,6 +48,7 @@ struct KP {
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
 
 constexpr size_t kSmemBudget = 200 * 1024;  // dynamic smem per block; leaves room for static scratch
+constexpr size_t kSmemMax = 227 * 1024 - 1024;  // hardware limit per block minus static scratch
 
 template <bool ASYNC>
 __device__ __forceinline__ double ldx(const double *p) {
@@ -608,6 +609,188 @@ __global__ void __launch_bounds__(1024, 1) k_block_pers(KP p) {
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+// ---------------------------------------------------------------------------------------------
+// k_block_stage: the default block sweep. Persistent blocks; everything one subdomain needs —
+// its slices' values and columns (one contiguous range of the layout), b_J, x_J (= y^0), and
+// the slices' metadata — arrives in one shared-memory STAGE through six bulk copies (TMA) that
+// complete on one mbarrier. Two stages: while the block sweeps subdomain l out of one stage,
+// the next subdomain streams into the other. Block thread 0 claims subdomains and loads the
+// range bounds one subdomain further ahead, so no thread ever waits on a dependent global load
+// except the off-block x gathers (a3). x_J may be bulk-copied early even in async mode: within
+// one launch only the block that claimed subdomain l writes x_J.
+// Requirements (host checks): rows_per_block % 128 == 0 (spb % 4 == 0), spb <= 32, <= WLR
+// local entries per row, 16-byte aligned b / x.
+struct StageGeom {
+    uint32_t vcap;    // entries per stage (spb * 32 * wmax)
+    uint32_t o_col, o_b, o_x, o_sptr, o_sw, bytes;
+};
+
+__host__ __device__ __forceinline__ StageGeom stage_geom(int R, int spb, int wmax) {
+    StageGeom g;
+    g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
+    g.o_col = g.vcap * 8;
+    g.o_b = g.o_col + g.vcap * 4;
+    g.o_x = g.o_b + (uint32_t)R * 8;
+    g.o_sptr = g.o_x + (uint32_t)R * 8;
+    g.o_sw = g.o_sptr + (uint32_t)spb * 8;
+    g.bytes = (g.o_sw + (uint32_t)spb * 4 + 127) & ~127u;
+    return g;
+}
+
+template <bool ASYNC, int WLR>
+__global__ void __launch_bounds__(1024, 1) k_block_stage(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[2];
+    __shared__ long long stage_l[2];
+    const int R = p.R, spb = p.spb;
+    const StageGeom g = stage_geom(R, spb, p.wmax);
+    double *y1 = reinterpret_cast<double *>(smraw + 2 * (size_t)g.bytes);
+    const int64_t q = (p.n + R - 1) / R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t G = gridDim.x;
+
+    // ---- thread 0: subdomain claims and stage issue ----
+    long long claims = 0;
+    auto claim = [&]() -> long long {
+        if (ASYNC) return (long long)atomicAdd(&p.state->work, 1ull);
+        return (long long)blockIdx.x + (claims++) * G;
+    };
+    auto issue = [&](long long l, int st, int64_t E0, int64_t E1) {
+        stage_l[st] = l;
+        if (l >= q) return;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        const uint32_t trows = (uint32_t)nrows & ~1u;
+        const uint32_t nb_sptr = ((uint32_t)nsl * 8 + 15) & ~15u, nb_sw = ((uint32_t)nsl * 4 + 15) & ~15u;
+        const uint32_t ne = (uint32_t)(E1 - E0);
+        unsigned char *S = smraw + (size_t)st * g.bytes;
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&bars[st], ne * 12 + trows * 16 + nb_sptr + nb_sw);
+        bulk_g2s(S, p.val + E0, ne * 8, &bars[st]);
+        bulk_g2s(S + g.o_col, p.col + E0, ne * 4, &bars[st]);
+        if (trows) {
+            bulk_g2s(S + g.o_b, p.b + TS, trows * 8, &bars[st]);
+            bulk_g2s(S + g.o_x, p.x_in + TS, trows * 8, &bars[st]);
+        }
+        bulk_g2s(S + g.o_sptr, p.sptr + l * spb, nb_sptr, &bars[st]);
+        bulk_g2s(S + g.o_sw, p.sw + l * spb, nb_sw, &bars[st]);
+    };
+    auto bounds = [&](long long l, int64_t &E0, int64_t &E1) {
+        if (l >= q) return;
+        const int nsl = (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice);
+        E0 = p.sptr[l * spb];
+        E1 = p.sptr[l * spb + nsl];
+    };
+    // Thread 0 keeps a three-deep claim pipeline so neither the work-queue atomic nor the range
+    // loads are waited on in the iteration that issues them: at iteration i it issues the stage
+    // of l_next (bounds loaded during i-1), loads the bounds of l_next2 (claimed during i-1) and
+    // claims a new subdomain.
+    long long l_next = 0, l_next2 = 0;
+    int64_t e0n = 0, e1n = 0;
+    if (threadIdx.x == 0) {
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        fence_mbar_init();
+        const long long l0 = claim();
+        int64_t e0 = 0, e1 = 0;
+        bounds(l0, e0, e1);
+        issue(l0, 0, e0, e1);
+        l_next = claim();
+        bounds(l_next, e0n, e1n);
+        l_next2 = claim();
+    }
+    __syncthreads();
+
+    constexpr int NP = WLR / 2;
+    double rr = 0.0, bb = 0.0;
+    for (int i = 0;; ++i) {
+        const int st = i & 1;
+        const long long l = stage_l[st];
+        if (l >= q) break;
+        if (threadIdx.x == 0) {  // stream the next subdomain into the other stage
+            issue(l_next, st ^ 1, e0n, e1n);
+            l_next = l_next2;
+            bounds(l_next, e0n, e1n);
+            l_next2 = l_next < q ? claim() : q;
+        }
+        unsigned char *S = smraw + (size_t)st * g.bytes;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        double *y0 = reinterpret_cast<double *>(S + g.o_x);
+        const double *sb = reinterpret_cast<const double *>(S + g.o_b);
+        mbar_wait(&bars[st], (i >> 1) & 1);
+        if (nrows & 1) {  // odd tail of the last subdomain: not bulk-copied
+            if (threadIdx.x == 0) y0[nrows - 1] = ldx<ASYNC>(p.x_in + TS + nrows - 1);
+            __syncthreads();
+        }
+        double lv[WLR];
+        uint32_t lc[NP];
+        double s = 0.0;
+        const int loc = warp * kSlice + lane;
+        const bool ok = warp < nsl && loc < nrows;
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+        for (int e = 0; e < NP; ++e) lc[e] = 0;
+        if (ok) {
+            const int64_t *ssp = reinterpret_cast<const int64_t *>(S + g.o_sptr);
+            const int sw = reinterpret_cast<const int32_t *>(S + g.o_sw)[warp];
+            const int wl = sw & 0xffff, wo = sw >> 16;
+            const int64_t off = ssp[warp] - ssp[0] + lane;
+            const double *sv = reinterpret_cast<const double *>(S) + off;
+            const int32_t *sc = reinterpret_cast<const int32_t *>(S + g.o_col) + off;
+            const double bi = loc < (nrows & ~1) ? sb[loc] : p.b[TS + loc];
+            bb += bi * bi;
+            double acc = bi;
+            // a3: off-block part, x as it stands (gathers batched)
+            for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+            }
+            s = acc;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[e] = sv[(wo + e) * kSlice];
+                    lc[e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                }
+            }
+            // first local sweep; its correction numerator is the residual (a5)
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[0] = 1.0 / lv[0];
+            rr += acc * acc;
+            y1[loc] = y0[loc] + lv[0] * acc;
+        }
+        __syncthreads();
+        // a4: sweeps 2..k, direct form, off-block part frozen
+        for (int t = 1; t < p.k; ++t) {
+            const double *yi = (t & 1) ? y1 : y0;
+            double *yo = (t & 1) ? y0 : y1;
+            if (ok) {
+                double acc = s;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                yo[loc] = lv[0] * acc;
+            }
+            __syncthreads();
+        }
+        // a6: write back
+        const double *yk = (p.k & 1) ? y1 : y0;
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
+        __syncthreads();
+    }
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
 // g, g + G, g + 2G, ... (G = warps in the grid) and keeps the next slice's bulk copy in flight
 // (two slice buffers per warp) while computing the current one.
@@ -802,7 +985,33 @@ cudaError_t launch_pers_t(const KP &p, const Layout &L, size_t smem, cudaStream_
     return cudaGetLastError();
 }
 
+template <bool ASYNC, int WLR>
+cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    static size_t attr = 0;
+    static size_t c_smem = 0;
+    static int c_threads = 0, per_sm = 0;
+    if (smem > attr) {
+        cudaError_t e =
+            cudaFuncSetAttribute(k_block_stage<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr = smem;
+    }
+    if (c_smem != smem || c_threads != L.spb * kSlice) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_block_stage<ASYNC, WLR>, L.spb * kSlice,
+                                                          smem) != cudaSuccess ||
+            per_sm < 1)
+            per_sm = 1;
+        c_smem = smem;
+        c_threads = L.spb * kSlice;
+    }
+    int64_t g = (int64_t)per_sm * L.sms;
+    if (g > L.q) g = L.q;
+    k_block_stage<ASYNC, WLR><<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
 // Kernel choice for one block-sweep launch (async / sync-block):
+//   k_block_stage persistent, whole-subdomain TMA stages (default when it fits)
 //   k_block_pers  persistent, double-buffered TMA slice stream (default when it fits)
 //   k_reg_tma  subdomains of <= 1024 rows with <= 8 local entries per row (every stencil
 //              config): TMA-streamed slices, register-resident local entries
@@ -817,7 +1026,14 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     p.wmax = L.max_w;
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
-    if (kind == 't' && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
+    const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
+    const bool aligned = ((uintptr_t)p.b % 16 == 0) && ((uintptr_t)p.x_in % 16 == 0);
+    if (kind == 't' && L.spb <= 32 && L.spb % 4 == 0 && L.max_wl <= 8 && aligned && stage_smem <= kSmemMax) {
+        if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
+        if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
+        return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
+    }
+    if ((kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
         if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
         if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
         return launch_pers_t<ASYNC, 8>(p, L, pers_smem, st);
