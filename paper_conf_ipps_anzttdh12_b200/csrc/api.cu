@@ -77,6 +77,15 @@ bar_status ensure_buf(double **p, int64_t n) {
 
 double model_bytes(const Layout &L) { return (double)L.nnz * (8 + 4) + (double)L.n * (8 + 8 + 8 + 4); }
 
+// Async driver choice. The fully asynchronous single-launch kernel removes per-iteration
+// launches and host round trips, which dominate when one global iteration moves little data;
+// for large systems the per-launch kernel streams faster (fewer registers on the hot path).
+// BAR_ASYNC_MULTI=1/0 forces either.
+bool use_async_multi(const Layout &L) {
+    if (const char *ev = getenv("BAR_ASYNC_MULTI")) return ev[0] == '1';
+    return model_bytes(L) < 256e6;
+}
+
 bar_status read_state(bar_matrix A, cudaStream_t st) {
     BAR_CUDA(cudaMemcpyAsync(A->W.h_state, A->W.state, sizeof(DevState), cudaMemcpyDeviceToHost, st));
     BAR_CUDA(cudaStreamSynchronize(st));
@@ -249,6 +258,15 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
         buf1 = A->W.xbuf;
     }
     BAR_CUDA(launch_init_state(A->W.state, -1.0, st));
+    if (mode == BAR_MODE_ASYNC && nsweeps > 0) {  // the fully asynchronous kernel when it applies
+        SweepArgs a{&A->L, b, x, x, k, A->W.state, A->W.partials, nullptr};
+        if (use_async_multi(A->L)) {
+            cudaError_t e = launch_async_multi(a, (long long)nsweeps * A->L.q, st);
+            if (e == cudaSuccess) return BAR_OK;
+            if (e != cudaErrorNotSupported) return cuda_fail(e, "launch_async_multi");
+            cudaGetLastError();
+        }
+    }
     for (int64_t m = 1; m <= nsweeps; ++m) {
         const double *xi = (m & 1) ? x : buf1;
         double *xo = (mode == BAR_MODE_ASYNC) ? x : ((m & 1) ? buf1 : x);
@@ -314,7 +332,7 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
     ++launches;
 
     DevState &H = *W.h_state;
-    int64_t iters = 0;
+    int64_t iters = 0, cta_max = -1;
     double rel = 0.0;
     int converged = 0;
     bool diverged = false, nonfinite = false, bzero = false;
@@ -367,7 +385,45 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
         if (H.bnorm == 0.0) bzero = true;
         else if (!std::isfinite(rel)) diverged = true;
         else if (rel <= tol) converged = 1;
-        while (!converged && !bzero && !diverged && H.iter < max_global_iters) {
+        // Fully asynchronous persistent solve (one launch for all global iterations); a stop
+        // request raised by the fused estimate is confirmed by an exact residual, else resumed.
+        bool multi = use_async_multi(L);
+        bool used_multi = false;
+        const long long w_end = (long long)max_global_iters * (long long)L.q;
+        while (multi && !converged && !bzero && !diverged && max_global_iters > 0) {
+            SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+            cudaError_t e = launch_async_multi(a, w_end, st);
+            if (e == cudaErrorNotSupported) {
+                cudaGetLastError();
+                multi = false;
+                break;
+            }
+            BAR_CUDA(e);
+            used_multi = true;
+            ++launches;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            if (H.diverged == 1) {
+                diverged = true;
+                break;
+            }
+            BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+            ++launches;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            rel = H.exact_rel;
+            if (!std::isfinite(rel) || rel > 1e30) diverged = true;
+            else if (rel <= tol) converged = 1;
+            else if (!H.stop || (long long)H.work_resume >= w_end) break;  // max_global_iters reached
+            else BAR_CUDA(launch_resume_queue(W.state, st));
+        }
+        if (used_multi) {
+            // global iterations needed: the iteration whose fused estimate met tol (the returned
+            // x has that many complete global iterations plus the sweeps still in flight when
+            // the queue closed, counted in cta_iters_max)
+            iters = (converged && H.stop_iter > 0) ? H.stop_iter : H.iters_done;
+            const unsigned long long claimed = H.stop ? H.work_resume : H.work;
+            cta_max = (int64_t)((claimed + L.q - 1) / L.q);
+        }
+        while (!multi && !converged && !bzero && !diverged && H.iter < max_global_iters) {
             const int64_t c = std::min<int64_t>(chunk, max_global_iters - (int64_t)H.iter);
             for (int64_t i = 0; i < c; ++i) {
                 SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
@@ -390,7 +446,7 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
                 else if (H.stop) BAR_CUDA(cudaMemsetAsync(&W.state->stop, 0, sizeof(int), st));
             }
         }
-        iters = H.iter;
+        if (!used_multi) iters = H.iter;
         result = buf0;
     }
     if (bzero) {
@@ -409,7 +465,7 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
         info->rel_res = rel;
         info->converged = converged;
         info->cta_iters_min = iters;
-        info->cta_iters_max = iters;
+        info->cta_iters_max = cta_max >= iters ? cta_max : iters;
         info->model_bytes_per_iter = model_bytes(L);
         info->kernel_launches = launches;
     }

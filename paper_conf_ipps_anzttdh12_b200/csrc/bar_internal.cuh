@@ -38,8 +38,16 @@ struct DevState {
     double last_rel;        // latest fused relative residual
     double exact_rel;       // latest standalone residual (bar_residual / confirmation)
     double exact_ss;        // its sum of squares
-    unsigned long long work;// async work queue: next subdomain to claim in this launch
+    unsigned long long work;// async work queue: next claim (subdomain w mod q of iteration w / q)
+    long long iters_done;   // async persistent: completed global iterations
+    long long stop_iter;    // async persistent: iteration whose residual estimate met tol
+    unsigned long long work_resume;  // async persistent: first unclaimed w when the queue closed
+    // async persistent: per-iteration accumulators (ring of kSlots iterations)
+    unsigned int done[64];  // subdomains of iteration m finished (slot m % 64)
+    double ss[64];          // sum of r_i^2 of those subdomains (x as it stood)
+    double bs[64];          // sum of b_i^2
 };
+constexpr int kSlots = 64;
 
 struct Layout {
     int64_t n = 0, nnz = 0;
@@ -107,10 +115,14 @@ struct SweepArgs {
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);
 cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st);
+// Fully asynchronous persistent solve: claims [work, w_end) = global iterations up to w_end / q
+// in ONE launch; cudaErrorNotSupported when the layout/vectors do not fit the staged kernel.
+cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t st);
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state,
                             double *partials, cudaStream_t st);
 cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
+cudaError_t launch_resume_queue(DevState *state, cudaStream_t st);  // reopen a closed async queue
 
 }  // namespace bar

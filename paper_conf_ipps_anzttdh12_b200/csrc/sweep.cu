@@ -43,6 +43,8 @@ struct KP {
     double *hist;
     int wlmax;
     int wmax;  // widest slice (local + off-block entries)
+    long long w_end;  // async persistent: claims [0, w_end) = global iterations [0, w_end / q)
+    int fresh_xj;     // async persistent with q < 4 * grid: read x_J when a subdomain starts
 };
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
@@ -127,9 +129,9 @@ __device__ __forceinline__ void reduce_finalize(double rr, double bb, const KP &
     }
     DevState *S = p.state;
     S->counter = 0;
-    S->work = 0;
     double bn = sqrt(bsq);
     S->bnorm = bn;
+    if (KIND != kResidual) S->work = 0;  // per-launch async queue (not the persistent one)
     if (KIND == kResidual) {
         S->exact_ss = ss;
         S->exact_rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
@@ -210,7 +212,7 @@ __device__ __forceinline__ void row_pass(const double *__restrict__ v, const int
 template <bool ASYNC, bool STAGE>
 __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
     if (*(volatile int *)&p.state->stop) return;
-    extern __shared__ __align__(16) unsigned char smraw[];
+    extern __shared__ __align__(128) unsigned char smraw[];
     const int R = p.R;
     const int sstride = p.spb * kSlice;
     double *y0 = reinterpret_cast<double *>(smraw);  // y^t, double-buffered
@@ -291,7 +293,7 @@ __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
 template <bool ASYNC, int WLR, int RPT>
 __global__ void __launch_bounds__(1024, 1) k_reg(KP p) {
     if (*(volatile int *)&p.state->stop) return;
-    extern __shared__ __align__(16) unsigned char smraw[];
+    extern __shared__ __align__(128) unsigned char smraw[];
     const int R = p.R;
     double *y0 = reinterpret_cast<double *>(smraw);
     double *y1 = y0 + R;
@@ -637,8 +639,62 @@ __host__ __device__ __forceinline__ StageGeom stage_geom(int R, int spb, int wma
     return g;
 }
 
+// Thread 0 of a block that finished a subdomain of global iteration m (MULTI): add its
+// residual contribution to iteration m's accumulators; the block finishing the q-th subdomain
+// of iteration m evaluates rel_res_m (an estimate: each subdomain saw x as it stood) and
+// applies the stopping rule (a7).
+// A block's claims increase monotonically, so it is done with iteration m when its next claim
+// belongs to a later iteration: it then publishes its (count, sum r^2, sum b^2) for m once —
+// three atomics and one fence per block per global iteration, not per subdomain.
+__device__ __forceinline__ void iteration_publish(const KP &p, long long m, unsigned int cnt, double t0, double t1,
+                                                  int64_t q) {
+    DevState *S = p.state;
+    const int slot = (int)(m % kSlots);
+    atomicAdd(&S->ss[slot], t0);
+    atomicAdd(&S->bs[slot], t1);
+    __threadfence();
+    const unsigned int c = atomicAdd(&S->done[slot], cnt);
+    if (c + cnt != (unsigned int)q) return;
+    __threadfence();
+    const double ss = __longlong_as_double(
+        (long long)atomicExch(reinterpret_cast<unsigned long long *>(&S->ss[slot]), 0ull));
+    const double bsq = __longlong_as_double(
+        (long long)atomicExch(reinterpret_cast<unsigned long long *>(&S->bs[slot]), 0ull));
+    atomicExch(&S->done[slot], 0u);
+    const double bn = sqrt(bsq);
+    const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+    atomicMax(&S->iters_done, m + 1);
+    S->bnorm = bn;
+    S->last_rel = rel;
+    if (p.hist) p.hist[m] = rel;
+    bool stop = false;
+    if (bn == 0.0) {
+        S->diverged = 2;
+        stop = true;
+    } else if (!isfinite(rel) || rel > 1e30) {
+        S->diverged = 1;
+        stop = true;
+    } else if (rel <= S->tol && S->stop == 0) {
+        S->stop_iter = m + 1;
+        stop = true;
+    }
+    if (stop && S->stop == 0) {
+        S->stop = 1;
+        // close the queue: later claims see w >= w_end; remember where to resume
+        const unsigned long long old = atomicMax(&S->work, (unsigned long long)p.w_end);
+        if (old < (unsigned long long)p.w_end) S->work_resume = old;
+    }
+}
+
+// MULTI (async only): the fully asynchronous solver — ONE launch runs every global iteration.
+// Claim w from the device queue means subdomain w mod q of global iteration w / q (R7); there
+// is no grid-wide synchronisation at all, so a block may sweep subdomain l of iteration m+1
+// while another still sweeps a neighbour in iteration m (eq. 3's bounded shift).
+// When the last subdomain of iteration m finishes, its block turns the accumulated residual
+// estimate into rel_res_m and raises the stop flag if it meets tol; blocks stop claiming.
+// Per-launch staged sweep (one global iteration per launch).
 template <bool ASYNC, int WLR>
-__global__ void __launch_bounds__(1024, 1) k_block_stage(KP p) {
+__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[2];
@@ -791,6 +847,233 @@ __global__ void __launch_bounds__(1024, 1) k_block_stage(KP p) {
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+
+// w = m*q + l without a 64-bit integer division (a long dependent chain on the critical warp):
+// w < 2^53 is exact in fp64, the quotient estimate is off by at most one and is corrected.
+__device__ __forceinline__ void divmod_q(long long w, int64_t q, double inv_q, long long &m, long long &l) {
+    m = (long long)((double)w * inv_q);
+    l = w - m * q;
+    if (l < 0) {
+        --m;
+        l += q;
+    } else if (l >= q) {
+        ++m;
+        l -= q;
+    }
+}
+
+// State of the block's thread 0 (claims, stage issue, residual publication). Kept in shared
+// memory, not registers: every thread would otherwise reserve the registers it occupies.
+struct T0State {
+    long long claims, pub_m;
+    double pub_ss, pub_bs;
+    unsigned int pub_cnt;
+};
+
+template <bool ASYNC, int WLR, bool MULTI>
+__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage_m(KP p) {
+    if (!MULTI && *(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[2];
+    __shared__ long long stage_w[2];    // claim held by each stage (>= wend: none)
+    __shared__ long long stage_sub[2];  // its subdomain index
+    __shared__ long long stage_m[2];    // its global iteration (MULTI)
+    __shared__ double sred[2][32];
+    __shared__ T0State t0;
+    const int R = p.R, spb = p.spb;
+    const StageGeom g = stage_geom(R, spb, p.wmax);
+    double *y1 = reinterpret_cast<double *>(smraw + 2 * (size_t)g.bytes);
+    const int64_t q = (p.n + R - 1) / R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const long long wend = MULTI ? p.w_end : q;  // claims >= wend end the launch
+    const double inv_q = MULTI ? 1.0 / (double)q : 0.0;
+
+    // ---- thread 0 only: subdomain claims and stage issue ----
+    auto claim = [&]() -> long long {
+        if (MULTI) {  // a stop request moves the queue to w_end, so no flag needs to be polled
+            const long long w = (long long)atomicAdd(&p.state->work, 1ull);
+            return w < wend ? w : wend;
+        }
+        if (ASYNC) return (long long)atomicAdd(&p.state->work, 1ull);
+        return (long long)blockIdx.x + (t0.claims++) * (long long)gridDim.x;
+    };
+    auto issue = [&](long long w, int st, int64_t E0, int64_t E1) {
+        stage_w[st] = w;
+        if (w >= wend) return;
+        long long l = w, m = 0;
+        if (MULTI) divmod_q(w, q, inv_q, m, l);
+        stage_sub[st] = l;
+        stage_m[st] = m;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        const uint32_t trows = (uint32_t)nrows & ~1u;
+        const uint32_t nb_sptr = ((uint32_t)nsl * 8 + 15) & ~15u, nb_sw = ((uint32_t)nsl * 4 + 15) & ~15u;
+        const uint32_t ne = (uint32_t)(E1 - E0);
+        unsigned char *S = smraw + (size_t)st * g.bytes;
+        const bool bulk_x = !(MULTI && p.fresh_xj);
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&bars[st], ne * 12 + trows * (bulk_x ? 16 : 8) + nb_sptr + nb_sw);
+        bulk_g2s(S, p.val + E0, ne * 8, &bars[st]);
+        bulk_g2s(S + g.o_col, p.col + E0, ne * 4, &bars[st]);
+        if (trows) {
+            bulk_g2s(S + g.o_b, p.b + TS, trows * 8, &bars[st]);
+            if (bulk_x) bulk_g2s(S + g.o_x, p.x_in + TS, trows * 8, &bars[st]);
+        }
+        bulk_g2s(S + g.o_sptr, p.sptr + l * spb, nb_sptr, &bars[st]);
+        bulk_g2s(S + g.o_sw, p.sw + l * spb, nb_sw, &bars[st]);
+    };
+    auto bounds = [&](long long w, int64_t &E0, int64_t &E1) {
+        if (w >= wend) return;
+        long long l = w, m = 0;
+        if (MULTI) divmod_q(w, q, inv_q, m, l);
+        const int nsl = (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice);
+        E0 = p.sptr[l * spb];
+        E1 = p.sptr[l * spb + nsl];
+    };
+    // Thread 0 keeps a three-deep claim pipeline so neither the work-queue atomic nor the range
+    // loads are waited on in the iteration that issues them: at iteration i it issues the stage
+    // of l_next (bounds loaded during i-1), loads the bounds of l_next2 (claimed during i-1) and
+    // claims a new subdomain. These four stay in registers: storing a load or atomic result to
+    // shared memory would wait for it.
+    long long l_next = 0, l_next2 = 0;
+    int64_t e0n = 0, e1n = 0;
+    if (threadIdx.x == 0) {
+        t0.claims = 0;
+        t0.pub_m = -1;
+        t0.pub_cnt = 0;
+        t0.pub_ss = t0.pub_bs = 0.0;
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        fence_mbar_init();
+        const long long l0 = claim();
+        int64_t e0 = 0, e1 = 0;
+        bounds(l0, e0, e1);
+        issue(l0, 0, e0, e1);
+        l_next = claim();
+        bounds(l_next, e0n, e1n);
+        l_next2 = claim();
+    }
+    __syncthreads();
+
+    constexpr int NP = WLR / 2;
+    double rr = 0.0, bb = 0.0;
+    for (int i = 0;; ++i) {
+        const int st = i & 1;
+        const long long wcur = stage_w[st];
+        if (wcur >= wend) break;
+        const long long l = MULTI ? stage_sub[st] : wcur;
+        if (MULTI) rr = bb = 0.0;  // per-subdomain residual contribution
+        if (threadIdx.x == 0) {  // stream the next subdomain into the other stage
+            issue(l_next, st ^ 1, e0n, e1n);
+            l_next = l_next2;
+            bounds(l_next, e0n, e1n);
+            l_next2 = l_next < wend ? claim() : wend;
+        }
+        unsigned char *S = smraw + (size_t)st * g.bytes;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        double *y0 = reinterpret_cast<double *>(S + g.o_x);
+        const double *sb = reinterpret_cast<const double *>(S + g.o_b);
+        mbar_wait(&bars[st], (i >> 1) & 1);
+        if (MULTI && p.fresh_xj) {  // few subdomains per block: x_J must not be prefetched
+            for (int r = threadIdx.x; r < nrows; r += blockDim.x) y0[r] = ldx<ASYNC>(p.x_in + TS + r);
+            __syncthreads();
+        } else if (nrows & 1) {  // odd tail of the last subdomain: not bulk-copied
+            if (threadIdx.x == 0) y0[nrows - 1] = ldx<ASYNC>(p.x_in + TS + nrows - 1);
+            __syncthreads();
+        }
+        double lv[WLR];
+        uint32_t lc[NP];
+        double s = 0.0;
+        const int loc = warp * kSlice + lane;
+        const bool ok = warp < nsl && loc < nrows;
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+        for (int e = 0; e < NP; ++e) lc[e] = 0;
+        if (ok) {
+            const int64_t *ssp = reinterpret_cast<const int64_t *>(S + g.o_sptr);
+            const int sw = reinterpret_cast<const int32_t *>(S + g.o_sw)[warp];
+            const int wl = sw & 0xffff, wo = sw >> 16;
+            const int64_t off = ssp[warp] - ssp[0] + lane;
+            const double *sv = reinterpret_cast<const double *>(S) + off;
+            const int32_t *sc = reinterpret_cast<const int32_t *>(S + g.o_col) + off;
+            const double bi = loc < (nrows & ~1) ? sb[loc] : p.b[TS + loc];
+            bb += bi * bi;
+            double acc = bi;
+            // a3: off-block part, x as it stands (gathers batched)
+            for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+            }
+            s = acc;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[e] = sv[(wo + e) * kSlice];
+                    lc[e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                }
+            }
+            // first local sweep; its correction numerator is the residual (a5)
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[0] = 1.0 / lv[0];
+            rr += acc * acc;
+            y1[loc] = y0[loc] + lv[0] * acc;
+        }
+        __syncthreads();
+        // a4: sweeps 2..k, direct form, off-block part frozen
+        for (int t = 1; t < p.k; ++t) {
+            const double *yi = (t & 1) ? y1 : y0;
+            double *yo = (t & 1) ? y0 : y1;
+            if (ok) {
+                double acc = s;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                yo[loc] = lv[0] * acc;
+            }
+            __syncthreads();
+        }
+        // a6: write back
+        const double *yk = (p.k & 1) ? y1 : y0;
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
+        if (MULTI) {
+            const double wr = warp_sum(rr), wb = warp_sum(bb);
+            if (lane == 0) {
+                sred[0][warp] = wr;
+                sred[1][warp] = wb;
+            }
+        }
+        __syncthreads();
+        if (MULTI && warp == 0) {
+            const int W = blockDim.x >> 5;
+            const double a0 = warp_sum(lane < W ? sred[0][lane] : 0.0);
+            const double a1 = warp_sum(lane < W ? sred[1][lane] : 0.0);
+            if (lane == 0) {
+                const long long m = stage_m[st];
+                if (m != t0.pub_m && t0.pub_cnt) {
+                    iteration_publish(p, t0.pub_m, t0.pub_cnt, t0.pub_ss, t0.pub_bs, q);
+                    t0.pub_cnt = 0;
+                    t0.pub_ss = t0.pub_bs = 0.0;
+                }
+                t0.pub_m = m;
+                ++t0.pub_cnt;
+                t0.pub_ss += a0;
+                t0.pub_bs += a1;
+            }
+        }
+    }
+    if (MULTI && threadIdx.x == 0 && t0.pub_cnt) iteration_publish(p, t0.pub_m, t0.pub_cnt, t0.pub_ss, t0.pub_bs, q);
+    if (!MULTI) reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
 // g, g + G, g + 2G, ... (G = warps in the grid) and keeps the next slice's bulk copy in flight
 // (two slice buffers per warp) while computing the current one.
@@ -900,6 +1183,14 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->last_rel = -1.0;
     S->exact_rel = -1.0;
     S->work = 0;
+    S->iters_done = 0;
+    S->stop_iter = -1;
+    S->work_resume = 0;
+    for (int i = 0; i < kSlots; ++i) {
+        S->done[i] = 0;
+        S->ss[i] = 0.0;
+        S->bs[i] = 0.0;
+    }
 }
 
 KP make_kp(const Layout &L) {
@@ -985,20 +1276,19 @@ cudaError_t launch_pers_t(const KP &p, const Layout &L, size_t smem, cudaStream_
     return cudaGetLastError();
 }
 
-template <bool ASYNC, int WLR>
-cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+template <bool ASYNC, int WLR, bool MULTI>
+cudaError_t launch_stage_m(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     static size_t attr = 0;
     static size_t c_smem = 0;
     static int c_threads = 0, per_sm = 0;
+    auto kfn = MULTI ? k_block_stage_m<true, WLR, true> : k_block_stage<ASYNC, WLR>;
     if (smem > attr) {
-        cudaError_t e =
-            cudaFuncSetAttribute(k_block_stage<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr = smem;
     }
     if (c_smem != smem || c_threads != L.spb * kSlice) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_block_stage<ASYNC, WLR>, L.spb * kSlice,
-                                                          smem) != cudaSuccess ||
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, L.spb * kSlice, smem) != cudaSuccess ||
             per_sm < 1)
             per_sm = 1;
         c_smem = smem;
@@ -1006,8 +1296,18 @@ cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream
     }
     int64_t g = (int64_t)per_sm * L.sms;
     if (g > L.q) g = L.q;
-    k_block_stage<ASYNC, WLR><<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
+    KP pp = p;
+    // a block prefetches x_J two claims ahead; with fewer than ~3 claims of other blocks in
+    // between, that could predate the subdomain's own previous update
+    pp.fresh_xj = MULTI && L.q < 4 * g;
+    kfn<<<(unsigned)g, L.spb * kSlice, smem, st>>>(pp);
     return cudaGetLastError();
+}
+
+template <bool ASYNC, int WLR>
+cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    if (ASYNC && p.w_end > 0) return launch_stage_m<true, WLR, true>(p, L, smem, st);
+    return launch_stage_m<ASYNC, WLR, false>(p, L, smem, st);
 }
 
 // Kernel choice for one block-sweep launch (async / sync-block):
@@ -1028,11 +1328,16 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
     const bool aligned = ((uintptr_t)p.b % 16 == 0) && ((uintptr_t)p.x_in % 16 == 0);
-    if (kind == 't' && L.spb <= 32 && L.spb % 4 == 0 && L.max_wl <= 8 && aligned && stage_smem <= kSmemMax) {
+    // bulk-copy sources must be 16-byte aligned: b/x at l*R rows (R even), ptr/sw at l*spb
+    const bool geom_ok = L.spb % 4 == 0 && L.R % 2 == 0 &&
+                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
+    if (kind == 't' && geom_ok && aligned && stage_smem <= kSmemMax) {
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
         if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
-        return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
+        if (L.max_wl <= 8) return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
+        return launch_stage_t<ASYNC, 16>(p, L, stage_smem, st);  // <= 256 threads per block
     }
+    if (p.w_end > 0) return cudaErrorNotSupported;  // no persistent multi-iteration kernel here
     if ((kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
         if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
         if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
@@ -1117,9 +1422,23 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.state = a.state;
     p.partials = a.partials;
     p.hist = a.hist;
+    p.w_end = 0;
     if (mode == BAR_MODE_JACOBI) return launch_rowwise<false>(p, *a.L, st);
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
     return launch_block<false>(p, *a.L, st);
+}
+
+cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t st) {
+    KP p = make_kp(*a.L);
+    p.b = a.b;
+    p.x_in = a.x_in;
+    p.x_out = a.x_out;
+    p.k = a.k;
+    p.state = a.state;
+    p.partials = a.partials;
+    p.hist = a.hist;
+    p.w_end = w_end > 0 ? w_end : 1;
+    return launch_block<true>(p, *a.L, st);
 }
 
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state, double *partials,
@@ -1130,6 +1449,16 @@ cudaError_t launch_residual(const Layout &L, const double *b, const double *x, D
     p.state = state;
     p.partials = partials;
     return launch_rowwise<true>(p, L, st);
+}
+
+__global__ void k_resume_queue(DevState *S) {
+    S->stop = 0;
+    S->work = S->work_resume;
+}
+
+cudaError_t launch_resume_queue(DevState *state, cudaStream_t st) {
+    k_resume_queue<<<1, 1, 0, st>>>(state);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st) {

@@ -122,7 +122,8 @@ def test_residual_parity(bar, name, R):
 @pytest.mark.parametrize("name", list(MATS))
 @pytest.mark.parametrize("mode,k,R", [("jacobi", 1, 128), ("sync-block", 1, 128), ("sync-block", 2, 100),
                                       ("sync-block", 5, 128), ("sync-block", 5, 448), ("sync-block", 9, 1024),
-                                      ("sync-block", 3, 1), ("sync-block", 5, 8192), ("sync-block", 4, 4000)])
+                                      ("sync-block", 3, 1), ("sync-block", 5, 8192), ("sync-block", 4, 4000),
+                                      ("sync-block", 5, 99), ("sync-block", 2, 256), ("sync-block", 5, 512)])
 def test_iterates_match_oracle(bar, name, mode, k, R):
     A = MATS[name]()
     b = np.ones(A.n)

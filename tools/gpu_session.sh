@@ -1,6 +1,3 @@
-timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -4
-timeout 900 python bench.py > gpurun_out/bench_c5.json 2> gpurun_out/bench_c5.err; tail -c 3000 gpurun_out/bench_c5.json
-timeout 600 python bench.py --workload c4 --no-cpu-baseline > gpurun_out/bench_c4.json 2>&1
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:k_ --csv --log-file gpurun_out/launches_c5.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_block_stage -s 3 -c 1 -o gpurun_out/prof_c5_async python tools/profile_sweep.py --workload c5 > gpurun_out/ncu_c5.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_block_stage -s 3 -c 1 -o gpurun_out/prof_c4_async python tools/profile_sweep.py --workload c4 > gpurun_out/ncu_c4.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+for w in c1 c2 c3; do timeout 300 python tools/sweep_R.py --workload $w --R 128 --modes async,sync-block 2>&1 | grep '^{'; done
+timeout 300 python tools/sweep_R.py --workload c2 --R 448 --k 1,2,5,9 --modes async 2>&1 | grep '^{'
