@@ -216,57 +216,94 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        raise SystemExit("multi-GPU bench: not built yet (DESIGN.md §Multi-GPU)")
     torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=dev)
     from paper_conf_ipps_anzttdh12_b200 import bar
 
-    dev = torch.device("cuda", local_rank)
-    n, nnz = matrix_dims(args.workload)
-    t0 = time.time()
-    A = make_matrix(args.workload)
-    t_gen = time.time() - t0
-    t0 = time.time()
-    M = bar.Matrix.from_csr(A, rows_per_block=args.R, device=local_rank)
-    t_setup = time.time() - t0
-    del A
-    minfo = M.info()
-    model_bytes = minfo["model_bytes_per_iter"]
-    stream = torch.cuda.current_stream(dev)
-    b = torch.ones(n, dtype=torch.float64, device=dev)
-    x = torch.empty(n, dtype=torch.float64, device=dev)
+    def barrier():
+        if dist is not None:
+            dist.barrier()
 
-    def step():
-        _, info = M.solve(b, None, x, k=args.k, max_global_iters=20000, tol=args.tol, mode=args.mode, stream=stream)
+    def reduce(v, op):
+        if dist is None:
+            return v
+        t = torch.tensor([float(v)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=op)
+        return float(t.item())
+
+    MAX = dist.ReduceOp.MAX if dist is not None else None
+    SUM = dist.ReduceOp.SUM if dist is not None else None
+    n, nnz = matrix_dims(args.workload)
+    stream = torch.cuda.current_stream(dev)
+    t0 = time.time()
+    if world == 1:
+        A = make_matrix(args.workload)
+        t_gen = time.time() - t0
+        t0 = time.time()
+        M = bar.Matrix.from_csr(A, rows_per_block=args.R, device=local_rank)
+        t_setup = time.time() - t0
+        del A
+        minfo = M.info()
+        n_loc, rows = n, (0, n)
+        local_bytes = minfo["model_bytes_per_iter"]
+    else:
+        from paper_conf_ipps_anzttdh12_b200 import dist as bdist
+
+        rows = bdist.partition(n, args.R, world)[rank]
+        A = make_matrix(args.workload, rows[0], rows[1])
+        t_gen = time.time() - t0
+        t0 = time.time()
+        M = bdist.DistMatrix(A, n, args.R, local_rank)
+        t_setup = time.time() - t0
+        n_loc = rows[1] - rows[0]
+        local_bytes = A.nnz * 12.0 + n_loc * 28.0
+        minfo = {"n_local": n_loc, "row_range": list(rows), "nnz_local": A.nnz, "ranks": world}
+        del A
+    total_bytes = nnz * 12.0 + n * 28.0
+    b = torch.ones(n_loc, dtype=torch.float64, device=dev)
+    x = torch.empty(n_loc, dtype=torch.float64, device=dev)
+
+    def step(bv=b, x0v=None, xv=x):
+        _, info = M.solve(bv, x0v, xv, k=args.k, max_global_iters=20000, tol=args.tol, mode=args.mode, stream=stream)
         return info
 
     for _ in range(args.warmup):
-        info = step()
+        step()
     torch.cuda.synchronize(dev)
     infos = []
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local_rank) as clk:
+        barrier()
         torch.cuda.synchronize(dev)
         ev0.record(stream)
         for _ in range(args.steps):
             infos.append(step())
         ev1.record(stream)
         torch.cuda.synchronize(dev)
-    ms_total = ev0.elapsed_time(ev1)
-    ms_per_step = ms_total / args.steps
+        barrier()
+    ms_per_step = reduce(ev0.elapsed_time(ev1), MAX) / args.steps  # max over ranks
     iters = [i["iters"] for i in infos]
-    launches = sum(i["kernel_launches"] for i in infos)
+    launches = int(reduce(sum(i["kernel_launches"] for i in infos), SUM))
     assert all(i["converged"] for i in infos), infos
     mean_iters = sum(iters) / len(iters)
 
-    # dominant kernel: per-launch duration of the sweep kernel, by the slope of back-to-back
-    # launch batches timed with CUDA events on the launching stream (cancels fixed overheads)
-    xs = torch.zeros(n, dtype=torch.float64, device=dev)
+    # dominant kernel: per-launch duration of the block-sweep kernel, from the slope of
+    # back-to-back launch batches timed with CUDA events on the launching stream (cancels fixed
+    # overheads); multi-GPU: the local kernel of each rank (no exchange), max over ranks
+    xs = torch.zeros(n_loc, dtype=torch.float64, device=dev)
 
     def timed_sweeps(nsw):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        M.sweep(b, xs, k=args.k, nsweeps=nsw, mode=args.mode, stream=stream)
+        if world == 1:
+            M.sweep(b, xs, k=args.k, nsweeps=nsw, mode=args.mode, stream=stream)
+        else:
+            M.sweep(k=args.k, nsweeps=nsw, mode=args.mode, stream=stream)
         e1.record(stream)
         torch.cuda.synchronize(dev)
         return e0.elapsed_time(e1)
@@ -275,16 +312,16 @@ def main():
     lo, hi = 8, 40
     t_lo = min(timed_sweeps(lo) for _ in range(3))
     t_hi = min(timed_sweeps(hi) for _ in range(3))
-    kernel_ms = (t_hi - t_lo) / (hi - lo)
+    kernel_ms = reduce((t_hi - t_lo) / (hi - lo), MAX)
     peak, peak_src = load_peaks()
-    achieved = model_bytes / (kernel_ms * 1e-3) / 1e9
+    achieved = local_bytes / (kernel_ms * 1e-3) / 1e9  # per GPU
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": None,
                 "kernel": f"k_block_stage<{args.mode}>" if args.mode != "jacobi" else "k_rowwise_tma<jacobi>",
-                "kernel_ms": round(kernel_ms, 5),
-                "algorithmic_bytes_per_launch": model_bytes, "peak_source": peak_src}
+                "kernel_ms": round(kernel_ms, 5), "algorithmic_bytes_per_launch": local_bytes,
+                "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
     prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")
-    if os.path.exists(prof):
+    if world == 1 and os.path.exists(prof):
         try:
             roofline["traffic"] = json.load(open(prof))["dram_bytes_per_launch"]
         except Exception:
@@ -293,25 +330,26 @@ def main():
     # end-to-end through the public API with HOST (pinned) buffers: H2D of b and x0, D2H of x
     e2e = None
     if not args.no_e2e:
-        bh = torch.ones(n, dtype=torch.float64).pin_memory()
-        x0h = torch.zeros(n, dtype=torch.float64).pin_memory()
-        xh = torch.empty(n, dtype=torch.float64).pin_memory()
-        M.solve(bh, x0h, xh, k=args.k, tol=args.tol, mode=args.mode, stream=stream)
+        bh = torch.ones(n_loc, dtype=torch.float64).pin_memory()
+        x0h = torch.zeros(n_loc, dtype=torch.float64).pin_memory()
+        xh = torch.empty(n_loc, dtype=torch.float64).pin_memory()
+        step(bh, x0h, xh)
         torch.cuda.synchronize(dev)
+        barrier()
         t0 = time.perf_counter()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for _ in range(args.steps):
-            _, ie = M.solve(bh, x0h, xh, k=args.k, tol=args.tol, mode=args.mode, stream=stream)
-            assert ie["converged"]
+            assert step(bh, x0h, xh)["converged"]
         e1.record(stream)
         torch.cuda.synchronize(dev)
-        e2e_s = e0.elapsed_time(e1) / 1e3 / args.steps
+        barrier()
+        e2e_s = reduce(e0.elapsed_time(e1), MAX) / 1e3 / args.steps
         e2e = {"value": e2e_s, "unit": "s", "h2d_bytes_per_step": 2 * 8 * n, "d2h_bytes_per_step": 8 * n,
                "wall_s": (time.perf_counter() - t0) / args.steps}
 
     cpu = None
-    if not args.no_cpu_baseline and rank == 0:
+    if not args.no_cpu_baseline and rank == 0 and world == 1:
         cores, model = cpu_info()
         s_iter, desc = oracle_sample(args.workload, args.k, args.R, args.mode,
                                      min(n, 4_000_000 if n > 4_000_000 else n))
@@ -326,16 +364,20 @@ def main():
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload][0]}", "n": n, "nnz": nnz,
                    "mode": args.mode, "k": args.k, "rows_per_block": args.R, "tol": args.tol, "b": "ones",
-                   "x0": "zeros", "parallelism": f"rows/{world}", "l2": "inputs > L2 (no flush needed)"
-                   if model_bytes > 126e6 else "inputs L2-resident (latency-bound config)"},
+                   "x0": "zeros", "parallelism": f"rows/{world}" + (" (NCCL halo send/recv)" if world > 1 else ""),
+                   "l2": "inputs > L2 (no flush needed)" if total_bytes / world > 126e6
+                   else "inputs L2-resident (latency-bound config)"},
         "global_iters": mean_iters, "global_iters_minmax": [min(iters), max(iters)],
-        "global_iters_per_s": mean_iters / value, "hbm_gbs_contract": model_bytes * mean_iters / value / 1e9,
+        "global_iters_per_s": mean_iters / value, "hbm_gbs_contract": total_bytes * mean_iters / value / 1e9,
         "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
         "clocks": clk.summary(), "setup_s": {"generate": round(t_gen, 2), "bar_create_csr": round(t_setup, 2)},
         "layout": minfo,
     }
     if rank == 0:
         print(json.dumps(line), flush=True)
+    if dist is not None:
+        M.close()
+        dist.destroy_process_group()
 
 
 if __name__ == "__main__":

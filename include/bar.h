@@ -148,6 +148,87 @@ bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info);
 /* bar_destroy — free the handle and its device memory (NULL-safe). */
 void bar_destroy(bar_matrix A);
 
+/* ===================== multi-GPU: row-partitioned solve =====================
+ * One process per GPU. Rank r owns the contiguous rows [row_begin, row_end) of the global
+ * system — the paper's "blocks addressed to the different devices, again split into ... blocks
+ * of rows ... assigned to the different thread blocks" (§3.4). row_begin must be a
+ * multiple of rows_per_block, so subdomains never straddle ranks and the per-row arithmetic
+ * is identical to the one-GPU solve (sync-block / Jacobi iterates are bitwise independent of
+ * the number of ranks). Columns a rank reads but does not own ("ghosts") are refreshed once
+ * per global iteration: halo exchange by NCCL grouped send/recv over NVLink, replacing the
+ * paper's AMC / DC / DK host- or master-GPU transfers. Local numbering is
+ * order-preserving: [ghosts below row_begin | owned rows | ghosts above], stored relative to
+ * the owned block (ghosts below are negative), so a row's entries keep their global order.
+ *
+ * Planning (host only, no GPU, usable before any device exists):
+ *   bar_dist_ghosts    sorted distinct ghost columns of the local rows: the n_ghost_lo ones
+ *                      below row_begin, then the n_ghost_hi ones at or above row_end. Call with
+ *                      ghosts = NULL for the counts. rowptr is relative (rowptr[0] = 0), col global.
+ *   bar_dist_localize  col_local[e] = col[e] - row_begin for owned columns, -n_ghost_lo + j for
+ *                      the j-th ghost below, (row_end - row_begin) + j for the j-th ghost above.
+ * The caller exchanges ghost lists with its process group (tests: gloo; bench: NCCL) to get
+ *   recv_counts[p]  how many of this rank's ghosts rank p owns (they are consecutive in ghost order)
+ *   send_counts[p]  how many owned rows rank p needs, and send_idx (their local row indices, in p's
+ *                   ghost order, concatenated by p).
+ */
+typedef struct bar_dist_s *bar_dist; /* opaque, one per rank */
+
+bar_status bar_dist_ghosts(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
+                           const int32_t *col, int64_t *n_ghost_lo, int64_t *n_ghost_hi, int32_t *ghosts);
+bar_status bar_dist_localize(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
+                             const int32_t *col, int64_t n_ghost_lo, int64_t n_ghost_hi, const int32_t *ghosts,
+                             int32_t *col_local);
+
+/* bar_nccl_unique_id — rank 0 creates the NCCL id (128 bytes) that every rank passes to
+ * bar_dist_create (broadcast it with the caller's process group). BAR_ERR_NCCL without NCCL. */
+bar_status bar_nccl_unique_id(void *id128);
+
+/*
+ * bar_dist_create — this rank's share: the local CSR (n_local = row_end - row_begin rows,
+ * col_local from bar_dist_localize, values), the exchange plan, and the transport.
+ *   nccl_id   128-byte ncclUniqueId from bar_nccl_unique_id, or NULL for the in-process
+ *             LOOPBACK transport (several ranks in one process on one device, linked with
+ *             bar_dist_link_loopback and driven by bar_dist_solve_loopback — for testing the
+ *             partitioned path on a single GPU).
+ *   send_idx  int32[sum send_counts] local row indices; send/recv_counts int64[nranks].
+ * Arrays may be host or device memory and are copied. Errors as bar_create_csr, plus
+ * BAR_ERR_NCCL, BAR_ERR_INVALID_ARG (row_begin not a multiple of R, inconsistent counts).
+ */
+bar_status bar_dist_create(int64_t n_global, int64_t row_begin, int64_t row_end, int64_t nnz_local,
+                           const int32_t *rowptr, const int32_t *col_local, const double *val, int64_t n_ghost_lo,
+                           int64_t n_ghost_hi, int nranks, int rank, const int64_t *recv_counts,
+                           const int64_t *send_counts, const int32_t *send_idx, int32_t rows_per_block, int device,
+                           const void *nccl_id, bar_dist *out);
+
+/* bar_dist_link_loopback — connect the loopback ranks of one process (ranks[r] has rank r). */
+bar_status bar_dist_link_loopback(bar_dist *ranks, int nranks);
+
+/*
+ * bar_dist_solve — the collective solve (every rank calls it with the same k, limits and mode):
+ * b, x0, x are this rank's owned rows (device or host, as bar_solve). Each global iteration:
+ * pack the rows peers need, NCCL grouped send/recv into the ghost slots, one block sweep on the
+ * local subdomains, all-gather of the per-rank [sum r^2, sum b^2] and a rank-ordered sum, so all
+ * ranks take the same stopping decision. Async mode: blocks of a rank run asynchronously
+ * (async-(k) within the GPU) and read the ghosts of the latest exchange.
+ */
+bar_status bar_dist_solve(bar_dist D, const double *b, const double *x0, double *x, int32_t k,
+                          int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
+                          bar_solve_info *info);
+
+/* bar_dist_solve_loopback — the same solve for all loopback ranks of this process, on one
+ * stream, with device-to-device copies as the exchange. b[r], x0[r], x[r] are rank r's rows. */
+bar_status bar_dist_solve_loopback(bar_dist *ranks, int nranks, const double *const *b, const double *const *x0,
+                                   double *const *x, int32_t k, int64_t max_global_iters, double tol,
+                                   bar_mode mode, void *cuda_stream, bar_solve_info *info);
+
+/* bar_dist_sweep — measurement entry point: enqueue exactly nsweeps launches of this rank's local
+ * block-sweep kernel on its current iterate (no halo exchange, no convergence control, no sync;
+ * ghost values are whatever the last exchange left). Local, not collective. */
+bar_status bar_dist_sweep(bar_dist D, int32_t k, int64_t nsweeps, bar_mode mode, void *cuda_stream);
+
+/* bar_dist_destroy — free one rank's share (NULL-safe; also destroys its NCCL communicator). */
+void bar_dist_destroy(bar_dist D);
+
 /* bar_last_error — text of the last failure on the calling thread ("" if none). */
 const char *bar_last_error(void);
 

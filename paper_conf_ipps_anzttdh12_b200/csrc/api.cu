@@ -27,21 +27,7 @@ bar_status cuda_fail(cudaError_t e, const char *what) {
     return e == cudaErrorMemoryAllocation ? BAR_ERR_OOM : BAR_ERR_CUDA;
 }
 
-namespace {
-
-// RAII: switch to the handle's device for the duration of a call.
-struct DeviceGuard {
-    int prev = -1;
-    bool ok = true;
-    explicit DeviceGuard(int dev) {
-        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
-        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
-    }
-    ~DeviceGuard() {
-        int cur = -1;
-        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
-    }
-};
+// Helpers shared with dist.cu (declared in bar_internal.cuh).
 
 bool is_device_ptr(const void *p) {
     cudaPointerAttributes a;
@@ -92,7 +78,6 @@ bar_status read_state(bar_matrix A, cudaStream_t st) {
     return BAR_OK;
 }
 
-}  // namespace
 }  // namespace bar
 
 using namespace bar;

@@ -90,6 +90,28 @@ namespace bar {
 void set_error(const std::string &msg);
 bar_status cuda_fail(cudaError_t e, const char *what);
 
+// RAII: switch to a handle's device for the duration of a call.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+// api.cu helpers
+bool is_device_ptr(const void *p);
+bar_status ensure_workspace(bar_matrix A);
+bar_status ensure_buf(double **p, int64_t n);
+double model_bytes(const Layout &L);
+bool use_async_multi(const Layout &L);
+bar_status read_state(bar_matrix A, cudaStream_t st);
+
 #define BAR_CUDA(call)                                              \
     do {                                                            \
         cudaError_t _e = (call);                                    \
@@ -97,8 +119,9 @@ bar_status cuda_fail(cudaError_t e, const char *what);
     } while (0)
 
 // Layout construction (layout.cu). rowptr/col/val are DEVICE pointers.
+// Columns in [col_lo, col_hi) (default [0, n)); row i's diagonal is column i.
 bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowptr, const int32_t *d_col,
-                        const double *d_val, int32_t R, cudaStream_t st);
+                        const double *d_val, int32_t R, cudaStream_t st, int64_t col_lo = 0, int64_t col_hi = -1);
 void free_layout(Layout &L);
 
 // Kernel launchers (sweep.cu). All pointers are device pointers.
@@ -111,6 +134,7 @@ struct SweepArgs {
     DevState *state;
     double *partials;
     double *hist;  // nullable device array: hist[m-1] = rel_res(x^(m-1)) (sync modes)
+    double *dist_out = nullptr;  // multi-GPU: receives this rank's [sum r^2, sum b^2]
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);
@@ -119,7 +143,12 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st);
 // in ONE launch; cudaErrorNotSupported when the layout/vectors do not fit the staged kernel.
 cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t st);
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state,
-                            double *partials, cudaStream_t st);
+                            double *partials, cudaStream_t st, double *dist_out = nullptr);
+// Multi-GPU helpers (sweep.cu): gather the values peers need; apply the stopping rule to the
+// rank-ordered sum of every rank's [sum r^2, sum b^2] (identical decision on every rank).
+cudaError_t launch_pack(const double *x_own, const int32_t *idx, int64_t cnt, double *out, cudaStream_t st);
+cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nranks, bool residual_only,
+                               cudaStream_t st);
 cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);

@@ -1,0 +1,564 @@
+// dist.cu — multi-GPU row-partitioned solve (include/bar.h "multi-GPU").
+//
+// Paper: §3.4 splits the system into row blocks per device, then per thread block,
+// with an asynchronous iteration between devices; its data paths (AMC through host memory,
+// DC/DK through a master GPU) were PCIe workarounds. Here every rank keeps its own rows and
+// refreshes the x values it reads but does not own (ghosts) once per global iteration with an
+// NCCL grouped send/recv over NVLink; the per-rank residual sums are all-gathered and summed
+// in rank order, so every rank applies the same stopping rule to the same bits.
+//
+// Local vector ("extended x"): [pad | ghosts below | owned rows | ghosts above]; the owned
+// block starts 16-byte aligned and every kernel indexes it with columns relative to the owned
+// block (ghosts below negative), which keeps each row's entries in their global order: the
+// per-row arithmetic, and so every sync-block / Jacobi iterate, is bitwise the one-GPU result.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "bar_internal.cuh"
+
+#ifdef BAR_WITH_NCCL
+#include <nccl.h>
+#endif
+
+struct bar_dist_s {
+    bar_matrix A = nullptr;  // local layout: n_local rows, columns [-n_glo, n_local + n_ghi)
+    int rank = 0, nranks = 1, device = 0;
+    int64_t n_global = 0, row_begin = 0, row_end = 0, n_local = 0, n_glo = 0, n_ghi = 0;
+    int64_t glo_pad = 0, ext = 0;  // owned block offset in the extended vector; its length
+    double *xa = nullptr, *xb = nullptr;  // extended iterate buffers
+    double *bbuf = nullptr;               // owned b (device)
+    double *xio = nullptr;                // owned x0 / x staging for host pointers
+    int32_t *send_idx = nullptr;          // device, local row indices
+    double *send_buf = nullptr;           // device
+    int64_t n_send = 0;
+    std::vector<int64_t> send_cnt, send_off, recv_cnt, recv_pos;  // recv_pos: owned-relative index
+    double *part = nullptr;      // device [2]: this rank's [sum r^2, sum b^2]
+    double *gathered = nullptr;  // device [2 * nranks]
+    bool loopback = true;
+    std::vector<bar_dist> peers;  // loopback group (peers[r] is rank r)
+#ifdef BAR_WITH_NCCL
+    ncclComm_t comm = nullptr;
+#endif
+};
+
+namespace bar {
+namespace {
+
+bar_status nccl_fail(int code, const char *what) {
+#ifdef BAR_WITH_NCCL
+    set_error(std::string(what) + ": " + ncclGetErrorString((ncclResult_t)code));
+#else
+    (void)code;
+    set_error(std::string(what) + ": libbar was built without NCCL");
+#endif
+    return BAR_ERR_NCCL;
+}
+
+#ifdef BAR_WITH_NCCL
+#define BAR_NCCL(call)                                                \
+    do {                                                              \
+        ncclResult_t _r = (call);                                     \
+        if (_r != ncclSuccess) return ::bar::nccl_fail((int)_r, #call); \
+    } while (0)
+#endif
+
+template <class T>
+bar_status to_device(const T *src, int64_t count, T **dst) {
+    BAR_CUDA(cudaMalloc((void **)dst, sizeof(T) * (size_t)(count > 0 ? count : 1)));
+    if (count > 0) BAR_CUDA(cudaMemcpy(*dst, src, sizeof(T) * (size_t)count, cudaMemcpyDefault));
+    return BAR_OK;
+}
+
+double *own(const bar_dist D, double *ext) { return ext + D->glo_pad; }
+
+// Refresh the ghost slots of the extended vector `ext` of every rank in `ranks` (NCCL: the
+// calling rank only; loopback: all ranks of the process, in order, on one stream).
+bar_status exchange(bar_dist *ranks, int nr, double *const *ext, cudaStream_t st) {
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        BAR_CUDA(launch_pack(own(D, ext[i]), D->send_idx, D->n_send, D->send_buf, st));
+    }
+    if (!ranks[0]->loopback) {
+#ifdef BAR_WITH_NCCL
+        bar_dist D = ranks[0];
+        double *xo = own(D, ext[0]);
+        BAR_NCCL(ncclGroupStart());
+        for (int p = 0; p < D->nranks; ++p) {
+            if (p == D->rank) continue;
+            if (D->send_cnt[p])
+                BAR_NCCL(ncclSend(D->send_buf + D->send_off[p], (size_t)D->send_cnt[p], ncclDouble, p, D->comm, st));
+            if (D->recv_cnt[p])
+                BAR_NCCL(ncclRecv(xo + D->recv_pos[p], (size_t)D->recv_cnt[p], ncclDouble, p, D->comm, st));
+        }
+        BAR_NCCL(ncclGroupEnd());
+        return BAR_OK;
+#else
+        return nccl_fail(0, "exchange");
+#endif
+    }
+    for (int i = 0; i < nr; ++i) {  // loopback: receiver i pulls from every sender p
+        bar_dist D = ranks[i];
+        for (int p = 0; p < nr; ++p) {
+            if (p == i || !D->recv_cnt[p]) continue;
+            bar_dist S = ranks[p];
+            if (S->send_cnt[i] != D->recv_cnt[p]) {
+                set_error("loopback plan mismatch: send/recv counts differ");
+                return BAR_ERR_INVALID_ARG;
+            }
+            BAR_CUDA(cudaMemcpyAsync(own(D, ext[i]) + D->recv_pos[p], S->send_buf + S->send_off[i],
+                                     sizeof(double) * (size_t)D->recv_cnt[p], cudaMemcpyDeviceToDevice, st));
+        }
+    }
+    return BAR_OK;
+}
+
+// All-gather the per-rank partial sums and apply the stopping rule on every rank.
+bar_status reduce_decide(bar_dist *ranks, int nr, bool residual_only, cudaStream_t st) {
+    if (!ranks[0]->loopback) {
+#ifdef BAR_WITH_NCCL
+        bar_dist D = ranks[0];
+        BAR_NCCL(ncclAllGather(D->part, D->gathered, 2, ncclDouble, D->comm, st));
+        BAR_CUDA(launch_dist_decide(D->A->W.state, D->gathered, D->nranks, residual_only, st));
+        return BAR_OK;
+#else
+        return nccl_fail(0, "reduce");
+#endif
+    }
+    bar_dist D0 = ranks[0];
+    for (int i = 0; i < nr; ++i)
+        BAR_CUDA(cudaMemcpyAsync(D0->gathered + 2 * i, ranks[i]->part, 2 * sizeof(double), cudaMemcpyDeviceToDevice,
+                                 st));
+    for (int i = 0; i < nr; ++i) {
+        if (i) BAR_CUDA(cudaMemcpyAsync(ranks[i]->gathered, D0->gathered, 2 * sizeof(double) * nr,
+                                        cudaMemcpyDeviceToDevice, st));
+        BAR_CUDA(launch_dist_decide(ranks[i]->A->W.state, ranks[i]->gathered, nr, residual_only, st));
+    }
+    return BAR_OK;
+}
+
+// The collective solve for the ranks this process drives (1 with NCCL, all with loopback).
+bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const double *const *x0, double *const *x,
+                      int32_t k, int64_t max_iters, double tol, bar_mode mode, cudaStream_t st,
+                      bar_solve_info *info) {
+    if ((mode != BAR_MODE_JACOBI && k < 1) || max_iters < 0 || !(tol >= 0.0) ||
+        (mode != BAR_MODE_ASYNC && mode != BAR_MODE_SYNC_BLOCK && mode != BAR_MODE_JACOBI)) {
+        set_error("need k >= 1, max_global_iters >= 0, tol >= 0, a valid mode");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if (mode == BAR_MODE_JACOBI) k = 1;
+    bar_status r;
+    DeviceGuard g(ranks[0]->device);
+    std::vector<double *> xa(nr), xb(nr);
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        if ((r = ensure_workspace(D->A)) != BAR_OK) return r;
+        const size_t nb = sizeof(double) * (size_t)D->n_local;
+        BAR_CUDA(cudaMemcpyAsync(D->bbuf, b[i], nb, cudaMemcpyDefault, st));
+        BAR_CUDA(cudaMemsetAsync(D->xa, 0, sizeof(double) * (size_t)D->ext, st));
+        BAR_CUDA(cudaMemsetAsync(D->xb, 0, sizeof(double) * (size_t)D->ext, st));
+        if (x0 && x0[i]) BAR_CUDA(cudaMemcpyAsync(own(D, D->xa), x0[i], nb, cudaMemcpyDefault, st));
+        BAR_CUDA(launch_init_state(D->A->W.state, tol, st));
+        xa[i] = D->xa;
+        xb[i] = D->xb;
+    }
+    int64_t launches = nr;
+    bar_dist D0 = ranks[0];
+    DevState &H = *D0->A->W.h_state;
+    int64_t issued = 0, chunk = 8;
+    int64_t iters = 0;
+    double rel = 0.0;
+    int converged = 0;
+    bool diverged = false, bzero = false;
+    std::vector<double *> res(nr);
+    for (;;) {
+        bool stopped = false;
+        // global iteration m: x^(m-1) in (m odd ? xa : xb) (async: always xa, in place)
+        while (issued < max_iters && !stopped) {
+            const int64_t c = std::min(chunk, max_iters - issued);
+            for (int64_t it = 0; it < c; ++it) {
+                const int64_t m = issued + it + 1;
+                const bool odd = (m & 1) || mode == BAR_MODE_ASYNC;
+                const std::vector<double *> &vin = odd ? xa : xb;
+                const std::vector<double *> &vout = mode == BAR_MODE_ASYNC ? xa : (odd ? xb : xa);
+                if ((r = exchange(ranks, nr, vin.data(), st)) != BAR_OK) return r;
+                for (int i = 0; i < nr; ++i) {
+                    bar_dist D = ranks[i];
+                    SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state,
+                                D->A->W.partials, nullptr, D->part};
+                    BAR_CUDA(launch_sweep(a, mode, st));
+                }
+                if ((r = reduce_decide(ranks, nr, false, st)) != BAR_OK) return r;
+                launches += 2 * nr;
+            }
+            issued += c;
+            if ((r = read_state(D0->A, st)) != BAR_OK) return r;
+            stopped = H.stop != 0;
+            chunk = std::min<int64_t>(chunk * 2, 256);
+        }
+        if (stopped && mode != BAR_MODE_ASYNC) {
+            iters = H.conv_iter;
+            rel = H.last_rel;
+            if (H.diverged == 2) bzero = true;
+            else if (H.diverged == 1) diverged = true;
+            else converged = 1;
+            for (int i = 0; i < nr; ++i) res[i] = (iters & 1) ? xb[i] : xa[i];
+            break;
+        }
+        // async (its fused estimate mixed old and new values) or max_global_iters reached:
+        // exact residual of the returned iterate, after a fresh exchange
+        iters = stopped ? (int64_t)H.iter : max_iters;
+        const bool est_diverged = stopped && H.diverged == 1;
+        for (int i = 0; i < nr; ++i) res[i] = mode == BAR_MODE_ASYNC ? xa[i] : ((iters & 1) ? xb[i] : xa[i]);
+        if ((r = exchange(ranks, nr, res.data(), st)) != BAR_OK) return r;
+        for (int i = 0; i < nr; ++i) {
+            bar_dist D = ranks[i];
+            BAR_CUDA(launch_residual(D->A->L, D->bbuf, own(D, res[i]), D->A->W.state, D->A->W.partials, st, D->part));
+        }
+        if ((r = reduce_decide(ranks, nr, true, st)) != BAR_OK) return r;
+        if ((r = read_state(D0->A, st)) != BAR_OK) return r;
+        rel = H.exact_rel;
+        if (H.bnorm == 0.0) bzero = true;
+        else if (est_diverged || !std::isfinite(rel) || rel > 1e30) diverged = true;
+        else converged = rel <= tol;
+        if (converged || diverged || bzero || !stopped || issued >= max_iters) break;
+        // the async estimate met tol but the exact residual did not: resume
+        for (int i = 0; i < nr; ++i)
+            BAR_CUDA(cudaMemsetAsync(&ranks[i]->A->W.state->stop, 0, sizeof(int), st));
+    }
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        const size_t nb = sizeof(double) * (size_t)D->n_local;
+        if (bzero) BAR_CUDA(cudaMemsetAsync(x[i], 0, nb, st));
+        else BAR_CUDA(cudaMemcpyAsync(x[i], own(D, res[i]), nb, cudaMemcpyDefault, st));
+    }
+    BAR_CUDA(cudaStreamSynchronize(st));
+    if (bzero) {
+        iters = 0;
+        rel = 0.0;
+        converged = 1;
+        diverged = false;
+    }
+    if (info) {
+        info->iters = iters;
+        info->rel_res = rel;
+        info->converged = converged;
+        info->cta_iters_min = iters;
+        info->cta_iters_max = iters;
+        double mb = 0.0;
+        for (int i = 0; i < nr; ++i) mb += model_bytes(ranks[i]->A->L);
+        info->model_bytes_per_iter = mb;
+        info->kernel_launches = launches;
+    }
+    if (diverged) {
+        set_error("relative residual became non-finite or exceeded 1e30");
+        return BAR_ERR_DIVERGED;
+    }
+    return BAR_OK;
+}
+
+}  // namespace
+}  // namespace bar
+
+using namespace bar;
+
+extern "C" {
+
+bar_status bar_dist_ghosts(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
+                           const int32_t *col, int64_t *n_ghost_lo, int64_t *n_ghost_hi, int32_t *ghosts) {
+    if (!rowptr || (!col && nnz_local > 0) || !n_ghost_lo || !n_ghost_hi || row_end < row_begin || row_begin < 0) {
+        set_error("invalid argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    const int64_t nl = row_end - row_begin;
+    if (rowptr[0] != 0 || rowptr[nl] != nnz_local) {
+        set_error("rowptr[0] != 0 or rowptr[n_local] != nnz_local");
+        return BAR_ERR_BAD_CSR;
+    }
+    std::vector<int32_t> lo, hi;
+    for (int64_t e = 0; e < nnz_local; ++e) {
+        const int64_t c = col[e];
+        if (c < row_begin) lo.push_back((int32_t)c);
+        else if (c >= row_end) hi.push_back((int32_t)c);
+    }
+    std::sort(lo.begin(), lo.end());
+    lo.erase(std::unique(lo.begin(), lo.end()), lo.end());
+    std::sort(hi.begin(), hi.end());
+    hi.erase(std::unique(hi.begin(), hi.end()), hi.end());
+    *n_ghost_lo = (int64_t)lo.size();
+    *n_ghost_hi = (int64_t)hi.size();
+    if (ghosts) {
+        std::copy(lo.begin(), lo.end(), ghosts);
+        std::copy(hi.begin(), hi.end(), ghosts + lo.size());
+    }
+    return BAR_OK;
+}
+
+bar_status bar_dist_localize(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
+                             const int32_t *col, int64_t n_ghost_lo, int64_t n_ghost_hi, const int32_t *ghosts,
+                             int32_t *col_local) {
+    if (!rowptr || !col_local || (nnz_local > 0 && !col) || ((n_ghost_lo + n_ghost_hi) > 0 && !ghosts)) {
+        set_error("invalid argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    const int64_t nl = row_end - row_begin;
+    const int32_t *lo = ghosts, *hi = ghosts + n_ghost_lo;
+    for (int64_t e = 0; e < nnz_local; ++e) {
+        const int64_t c = col[e];
+        if (c < row_begin) {
+            const int32_t *it = std::lower_bound(lo, lo + n_ghost_lo, (int32_t)c);
+            if (it == lo + n_ghost_lo || *it != c) {
+                set_error("column missing from the ghost list");
+                return BAR_ERR_INVALID_ARG;
+            }
+            col_local[e] = (int32_t)(-n_ghost_lo + (it - lo));
+        } else if (c >= row_end) {
+            const int32_t *it = std::lower_bound(hi, hi + n_ghost_hi, (int32_t)c);
+            if (it == hi + n_ghost_hi || *it != c) {
+                set_error("column missing from the ghost list");
+                return BAR_ERR_INVALID_ARG;
+            }
+            col_local[e] = (int32_t)(nl + (it - hi));
+        } else {
+            col_local[e] = (int32_t)(c - row_begin);
+        }
+    }
+    (void)rowptr;
+    return BAR_OK;
+}
+
+bar_status bar_nccl_unique_id(void *id128) {
+    if (!id128) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+#ifdef BAR_WITH_NCCL
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    ncclUniqueId id;
+    ncclResult_t rc = ncclGetUniqueId(&id);
+    if (rc != ncclSuccess) return nccl_fail((int)rc, "ncclGetUniqueId");
+    std::memcpy(id128, &id, sizeof(id));
+    return BAR_OK;
+#else
+    return nccl_fail(0, "ncclGetUniqueId");
+#endif
+}
+
+bar_status bar_dist_create(int64_t n_global, int64_t row_begin, int64_t row_end, int64_t nnz_local,
+                           const int32_t *rowptr, const int32_t *col_local, const double *val, int64_t n_ghost_lo,
+                           int64_t n_ghost_hi, int nranks, int rank, const int64_t *recv_counts,
+                           const int64_t *send_counts, const int32_t *send_idx, int32_t rows_per_block, int device,
+                           const void *nccl_id, bar_dist *out) {
+    if (!out) {
+        set_error("out is NULL");
+        return BAR_ERR_INVALID_ARG;
+    }
+    *out = nullptr;
+    const int64_t nl = row_end - row_begin;
+    if (nranks < 1 || rank < 0 || rank >= nranks || nl < 1 || row_begin < 0 || row_end > n_global ||
+        rows_per_block < 1 || rows_per_block > BAR_MAX_ROWS_PER_BLOCK || row_begin % rows_per_block != 0 ||
+        n_ghost_lo < 0 || n_ghost_hi < 0 || !recv_counts || !send_counts) {
+        set_error("invalid partition (row_begin must be a multiple of rows_per_block) or argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    int64_t nrecv = 0, nsend = 0;
+    for (int p = 0; p < nranks; ++p) {
+        if (recv_counts[p] < 0 || send_counts[p] < 0 || (p == rank && (recv_counts[p] || send_counts[p]))) {
+            set_error("invalid send/recv counts");
+            return BAR_ERR_INVALID_ARG;
+        }
+        nrecv += recv_counts[p];
+        nsend += send_counts[p];
+    }
+    if (nrecv != n_ghost_lo + n_ghost_hi || (nsend > 0 && !send_idx)) {
+        set_error("recv counts must add up to the ghost count");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(device);
+    if (!g.ok) return cuda_fail(cudaGetLastError(), "cudaSetDevice");
+    auto *D = new bar_dist_s();
+    D->rank = rank;
+    D->nranks = nranks;
+    D->device = device;
+    D->n_global = n_global;
+    D->row_begin = row_begin;
+    D->row_end = row_end;
+    D->n_local = nl;
+    D->n_glo = n_ghost_lo;
+    D->n_ghi = n_ghost_hi;
+    D->glo_pad = (n_ghost_lo + 1) & ~(int64_t)1;  // owned block 16-byte aligned
+    D->ext = D->glo_pad + nl + n_ghost_hi + 2;
+    D->send_cnt.assign(send_counts, send_counts + nranks);
+    D->recv_cnt.assign(recv_counts, recv_counts + nranks);
+    D->send_off.assign(nranks, 0);
+    D->recv_pos.assign(nranks, 0);
+    for (int p = 1; p < nranks; ++p) D->send_off[p] = D->send_off[p - 1] + D->send_cnt[p - 1];
+    {
+        int64_t pos = -n_ghost_lo;  // ghosts of ranks below, then (skipping the owned block) above
+        for (int p = 0; p < nranks; ++p) {
+            if (p == rank) pos = nl;
+            D->recv_pos[p] = pos;
+            pos += D->recv_cnt[p];
+        }
+    }
+    D->n_send = nsend;
+    bar_status st = BAR_OK;
+    // local layout: rows [0, nl), columns [-n_glo, nl + n_ghi)
+    {
+        const int32_t *d_rp = rowptr, *d_col = col_local;
+        const double *d_val = val;
+        int32_t *t_rp = nullptr, *t_col = nullptr;
+        double *t_val = nullptr;
+        if (!is_device_ptr(rowptr)) st = to_device(rowptr, nl + 1, &t_rp), d_rp = t_rp;
+        if (st == BAR_OK && !is_device_ptr(col_local)) st = to_device(col_local, nnz_local, &t_col), d_col = t_col;
+        if (st == BAR_OK && !is_device_ptr(val)) st = to_device(val, nnz_local, &t_val), d_val = t_val;
+        if (st == BAR_OK) {
+            D->A = new bar_matrix_s();
+            D->A->device = device;
+            st = build_layout(D->A->L, nl, nnz_local, d_rp, d_col, d_val, rows_per_block, nullptr, -n_ghost_lo,
+                              nl + n_ghost_hi);
+            if (st != BAR_OK) {
+                delete D->A;
+                D->A = nullptr;
+            }
+        }
+        cudaFree(t_rp);
+        cudaFree(t_col);
+        cudaFree(t_val);
+    }
+    if (st == BAR_OK) {
+        std::vector<int32_t> hidx(nsend);
+        if (nsend) {
+            if (is_device_ptr(send_idx)) {
+                if (cudaMemcpy(hidx.data(), send_idx, sizeof(int32_t) * nsend, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    st = cuda_fail(cudaGetLastError(), "send_idx");
+            } else {
+                std::memcpy(hidx.data(), send_idx, sizeof(int32_t) * nsend);
+            }
+        }
+        for (int64_t i = 0; st == BAR_OK && i < nsend; ++i)
+            if (hidx[i] < 0 || hidx[i] >= nl) {
+                set_error("send_idx out of the owned rows");
+                st = BAR_ERR_INVALID_ARG;
+            }
+        if (st == BAR_OK) st = to_device(hidx.data(), nsend, &D->send_idx);
+    }
+    auto dalloc = [&](double **p, int64_t n) {
+        if (st == BAR_OK && cudaMalloc((void **)p, sizeof(double) * (size_t)(n > 0 ? n : 1)) != cudaSuccess)
+            st = cuda_fail(cudaGetLastError(), "cudaMalloc");
+    };
+    dalloc(&D->xa, D->ext);
+    dalloc(&D->xb, D->ext);
+    dalloc(&D->bbuf, nl);
+    dalloc(&D->send_buf, nsend);
+    dalloc(&D->part, 2);
+    dalloc(&D->gathered, 2 * (int64_t)nranks);
+    D->loopback = nccl_id == nullptr;
+    if (st == BAR_OK && !D->loopback) {
+#ifdef BAR_WITH_NCCL
+        ncclUniqueId id;
+        std::memcpy(&id, nccl_id, sizeof(id));
+        ncclResult_t rc = ncclCommInitRank(&D->comm, nranks, id, rank);
+        if (rc != ncclSuccess) st = nccl_fail((int)rc, "ncclCommInitRank");
+#else
+        st = nccl_fail(0, "ncclCommInitRank");
+#endif
+    }
+    if (st != BAR_OK) {
+        bar_dist_destroy(D);
+        return st;
+    }
+    if (D->loopback) D->peers.assign(1, D);
+    *out = D;
+    return BAR_OK;
+}
+
+bar_status bar_dist_link_loopback(bar_dist *ranks, int nranks) {
+    if (!ranks || nranks < 1) {
+        set_error("invalid argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    for (int i = 0; i < nranks; ++i) {
+        if (!ranks[i] || !ranks[i]->loopback || ranks[i]->rank != i || ranks[i]->nranks != nranks ||
+            ranks[i]->device != ranks[0]->device) {
+            set_error("loopback ranks must be 0..nranks-1 of one group on one device, created with nccl_id = NULL");
+            return BAR_ERR_INVALID_ARG;
+        }
+    }
+    for (int i = 0; i < nranks; ++i) ranks[i]->peers.assign(ranks, ranks + nranks);
+    return BAR_OK;
+}
+
+bar_status bar_dist_solve(bar_dist D, const double *b, const double *x0, double *x, int32_t k,
+                          int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
+                          bar_solve_info *info) {
+    if (!D || !b || !x) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    if (D->loopback && D->nranks > 1) {
+        set_error("loopback ranks are driven together by bar_dist_solve_loopback");
+        return BAR_ERR_INVALID_ARG;
+    }
+    const double *bb[1] = {b};
+    const double *xx0[1] = {x0};
+    double *xx[1] = {x};
+    return dist_solve(&D, 1, bb, xx0, xx, k, max_global_iters, tol, mode, (cudaStream_t)cuda_stream, info);
+}
+
+bar_status bar_dist_solve_loopback(bar_dist *ranks, int nranks, const double *const *b, const double *const *x0,
+                                   double *const *x, int32_t k, int64_t max_global_iters, double tol,
+                                   bar_mode mode, void *cuda_stream, bar_solve_info *info) {
+    if (!ranks || nranks < 1 || !b || !x) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    for (int i = 0; i < nranks; ++i)
+        if (!ranks[i] || !ranks[i]->loopback || (int)ranks[i]->peers.size() != nranks || ranks[i]->peers[0] != ranks[0]) {
+            set_error("ranks are not a linked loopback group");
+            return BAR_ERR_INVALID_ARG;
+        }
+    return dist_solve(ranks, nranks, b, x0, x, k, max_global_iters, tol, mode, (cudaStream_t)cuda_stream, info);
+}
+
+bar_status bar_dist_sweep(bar_dist D, int32_t k, int64_t nsweeps, bar_mode mode, void *cuda_stream) {
+    if (!D || nsweeps < 0 || (mode != BAR_MODE_JACOBI && k < 1)) {
+        set_error("invalid argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(D->device);
+    bar_status r = ensure_workspace(D->A);
+    if (r != BAR_OK) return r;
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    BAR_CUDA(launch_init_state(D->A->W.state, -1.0, st));
+    for (int64_t m = 1; m <= nsweeps; ++m) {
+        double *xi = (mode == BAR_MODE_ASYNC || (m & 1)) ? D->xa : D->xb;
+        double *xo = mode == BAR_MODE_ASYNC ? D->xa : ((m & 1) ? D->xb : D->xa);
+        SweepArgs a{&D->A->L, D->bbuf, own(D, xi), own(D, xo), mode == BAR_MODE_JACOBI ? 1 : k, D->A->W.state,
+                    D->A->W.partials, nullptr, D->part};
+        BAR_CUDA(launch_sweep(a, mode, st));
+    }
+    return BAR_OK;
+}
+
+void bar_dist_destroy(bar_dist D) {
+    if (!D) return;
+    DeviceGuard g(D->device);
+#ifdef BAR_WITH_NCCL
+    if (D->comm) ncclCommDestroy(D->comm);
+#endif
+    bar_destroy(D->A);
+    cudaFree(D->xa);
+    cudaFree(D->xb);
+    cudaFree(D->bbuf);
+    cudaFree(D->xio);
+    cudaFree(D->send_idx);
+    cudaFree(D->send_buf);
+    cudaFree(D->part);
+    cudaFree(D->gathered);
+    delete D;
+}
+
+}  // extern "C"

@@ -25,9 +25,12 @@ __device__ __forceinline__ void slice_row(int64_t s, int32_t R, int32_t spb, int
 
 // Per row: validate and count local (column inside the row's subdomain, diagonal included)
 // and off-block entries.
+// Columns may range over [col_lo, col_hi) with col_lo <= 0: a multi-GPU rank numbers its
+// ghost columns below its first row negatively (order-preserving local numbering, dist.cu).
 __global__ void k_validate_count(int64_t n, int64_t nnz, const int32_t *__restrict__ rowptr,
                                  const int32_t *__restrict__ col, const double *__restrict__ val, int32_t R,
-                                 int32_t *__restrict__ nloc, int32_t *__restrict__ noff, int *__restrict__ err) {
+                                 int64_t col_lo, int64_t col_hi, int32_t *__restrict__ nloc,
+                                 int32_t *__restrict__ noff, int *__restrict__ err) {
     int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
     int32_t a = rowptr[i], e = rowptr[i + 1];
@@ -41,11 +44,11 @@ __global__ void k_validate_count(int64_t n, int64_t nnz, const int32_t *__restri
     int64_t TE = min(TS + (int64_t)R, n);
     int cl = 0, co = 0, bad = 0;
     bool diag = false;
-    int64_t prev = -1;
+    int64_t prev = col_lo - 1;
     for (int32_t p = a; p < e; ++p) {
         int64_t c = col[p];
         double v = val[p];
-        if (c < 0 || c >= n || c <= prev) bad |= kErrBadCsr;
+        if (c < col_lo || c >= col_hi || c <= prev) bad |= kErrBadCsr;
         prev = c;
         if (!isfinite(v)) bad |= kErrNonFinite;
         if (c == i) {
@@ -174,7 +177,8 @@ static bar_status alloc_fail(cudaError_t e, const char *what) {
     } while (0)
 
 bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowptr, const int32_t *d_col,
-                        const double *d_val, int32_t R, cudaStream_t st) {
+                        const double *d_val, int32_t R, cudaStream_t st, int64_t col_lo, int64_t col_hi) {
+    if (col_hi < 0) col_hi = n;
     bar_status st_ = BAR_OK;
     int32_t *nloc = nullptr, *noff = nullptr;
     int *d_err = nullptr;
@@ -211,8 +215,8 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     BAR_CK(cudaMemsetAsync(L.sptr + nsl + 1, 0, 4 * sizeof(int64_t), st));
     BAR_CK(cudaMemsetAsync(d_err, 0, sizeof(int), st));
 
-    k_validate_count<<<(unsigned)((n + TB - 1) / TB), TB, 0, st>>>(n, nnz, d_rowptr, d_col, d_val, R, nloc, noff,
-                                                                  d_err);
+    k_validate_count<<<(unsigned)((n + TB - 1) / TB), TB, 0, st>>>(n, nnz, d_rowptr, d_col, d_val, R, col_lo,
+                                                                  col_hi, nloc, noff, d_err);
     BAR_CK(cudaGetLastError());
     BAR_CK(cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, st));
     BAR_CK(cudaStreamSynchronize(st));

@@ -45,6 +45,7 @@ struct KP {
     int wmax;  // widest slice (local + off-block entries)
     long long w_end;  // async persistent: claims [0, w_end) = global iterations [0, w_end / q)
     int fresh_xj;     // async persistent with q < 4 * grid: read x_J when a subdomain starts
+    double *dist_out; // multi-GPU: [sum r^2, sum b^2] of this rank (no stopping decision here)
 };
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
@@ -76,6 +77,35 @@ __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     return v;
+}
+
+// The stopping rule (R2/R6/R14) on the global sums of r_i^2 and b_i^2.
+// A sweep launch that produced x^(m) reports rel_res(x^(m-1)).
+__device__ __forceinline__ void apply_stop_rule(DevState *S, double ss, double bsq, bool residual_only,
+                                                double *hist) {
+    const double bn = sqrt(bsq);
+    S->bnorm = bn;
+    if (residual_only) {
+        S->exact_ss = ss;
+        S->exact_rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+        return;
+    }
+    const long long m = ++S->iter;  // this launch produced x^(m) from x^(m-1)
+    const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+    S->last_rel = rel;
+    if (hist) hist[m - 1] = rel;
+    if (bn == 0.0) {  // b = 0: x = 0 is the answer (DESIGN.md reading R2)
+        S->stop = 1;
+        S->conv_iter = 0;
+        S->diverged = 2;
+    } else if (!isfinite(rel) || rel > 1e30) {
+        S->stop = 1;
+        S->diverged = 1;
+        S->conv_iter = m - 1;
+    } else if (rel <= S->tol) {
+        S->stop = 1;
+        S->conv_iter = m - 1;  // sync: x^(m-1) (still in the input buffer) is the answer
+    }
 }
 
 // Deterministic two-level reduction of (rr, bb) over the grid: fixed shuffle tree per warp,
@@ -129,30 +159,13 @@ __device__ __forceinline__ void reduce_finalize(double rr, double bb, const KP &
     }
     DevState *S = p.state;
     S->counter = 0;
-    double bn = sqrt(bsq);
-    S->bnorm = bn;
     if (KIND != kResidual) S->work = 0;  // per-launch async queue (not the persistent one)
-    if (KIND == kResidual) {
-        S->exact_ss = ss;
-        S->exact_rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+    if (p.dist_out) {  // multi-GPU: this rank's sums; the stopping rule runs after the exchange
+        p.dist_out[0] = ss;
+        p.dist_out[1] = bsq;
         return;
     }
-    long long m = ++S->iter;  // this launch produced x^(m) from x^(m-1)
-    double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
-    S->last_rel = rel;
-    if (p.hist) p.hist[m - 1] = rel;
-    if (bn == 0.0) {  // b = 0: x = 0 is the answer (DESIGN.md reading R2)
-        S->stop = 1;
-        S->conv_iter = 0;
-        S->diverged = 2;
-    } else if (!isfinite(rel) || rel > 1e30) {
-        S->stop = 1;
-        S->diverged = 1;
-        S->conv_iter = m - 1;
-    } else if (rel <= S->tol) {
-        S->stop = 1;
-        S->conv_iter = m - 1;  // sync: x^(m-1) (still in the input buffer) is the answer
-    }
+    apply_stop_rule(S, ss, bsq, KIND == kResidual, p.hist);
 }
 
 constexpr int U = 4;  // stored entries of a row loaded together (loads in flight per thread)
@@ -1422,6 +1435,7 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.state = a.state;
     p.partials = a.partials;
     p.hist = a.hist;
+    p.dist_out = a.dist_out;
     p.w_end = 0;
     if (mode == BAR_MODE_JACOBI) return launch_rowwise<false>(p, *a.L, st);
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
@@ -1437,18 +1451,52 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
     p.state = a.state;
     p.partials = a.partials;
     p.hist = a.hist;
+    p.dist_out = a.dist_out;
     p.w_end = w_end > 0 ? w_end : 1;
     return launch_block<true>(p, *a.L, st);
 }
 
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state, double *partials,
-                            cudaStream_t st) {
+                            cudaStream_t st, double *dist_out) {
     KP p = make_kp(L);
     p.b = b;
     p.x_in = x;
     p.state = state;
     p.partials = partials;
+    p.dist_out = dist_out;
     return launch_rowwise<true>(p, L, st);
+}
+
+__global__ void k_pack(const double *__restrict__ x_own, const int32_t *__restrict__ idx, int64_t cnt,
+                       double *__restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = x_own[idx[i]];
+}
+
+cudaError_t launch_pack(const double *x_own, const int32_t *idx, int64_t cnt, double *out, cudaStream_t st) {
+    if (cnt <= 0) return cudaSuccess;
+    int64_t blocks = (cnt + 255) / 256;
+    if (blocks > 4096) blocks = 4096;
+    k_pack<<<(unsigned)blocks, 256, 0, st>>>(x_own, idx, cnt, out);
+    return cudaGetLastError();
+}
+
+// Rank-ordered sum of the gathered per-rank [sum r^2, sum b^2]: every rank computes the same
+// bits, so every rank takes the same stopping decision.
+__global__ void k_dist_decide(DevState *S, const double *__restrict__ g, int nranks, int residual_only) {
+    if (!residual_only && S->stop) return;  // queued iterations after the stop: sweeps were skipped
+    double ss = 0.0, bsq = 0.0;
+    for (int r = 0; r < nranks; ++r) {
+        ss += g[2 * r];
+        bsq += g[2 * r + 1];
+    }
+    apply_stop_rule(S, ss, bsq, residual_only != 0, nullptr);
+}
+
+cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nranks, bool residual_only,
+                               cudaStream_t st) {
+    k_dist_decide<<<1, 1, 0, st>>>(state, gathered, nranks, residual_only ? 1 : 0);
+    return cudaGetLastError();
 }
 
 __global__ void k_resume_queue(DevState *S) {

@@ -1,0 +1,97 @@
+"""The partitioned (multi-GPU) device path on ONE GPU: P loopback ranks in one process, the
+exchange done by device-to-device copies (the NCCL path differs only in the transport call).
+
+Sync-block and Jacobi iterates over P ranks must be bitwise identical to the one-GPU solve
+(the order-preserving local numbering leaves every row's arithmetic unchanged), the stopping
+iteration equal, and async must converge.
+"""
+import numpy as np
+import pytest
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+def _split(gen, args, n, R, P):
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    return [gen(*args, row_lo=a, row_hi=b) for a, b in D.partition(n, R, P)]
+
+
+def _single(bar, A, b, R, k, mode, iters, tol, x0):
+    import torch
+
+    M = bar.Matrix.from_csr(A, R)
+    x = torch.empty(A.n, dtype=torch.float64, device="cuda")
+    _, info = M.solve(torch.from_numpy(b).cuda(), torch.from_numpy(x0).cuda(), x, k=k, max_global_iters=iters,
+                      tol=tol, mode=mode)
+    M.close()
+    return x.cpu().numpy(), info
+
+
+def _loop(blocks, n, R, b, k, mode, iters, tol, x0):
+    import torch
+
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    G = D.LoopbackGroup(blocks, n, R)
+    bs = [torch.from_numpy(b[a:c].copy()).cuda() for a, c in G.ranges]
+    x0s = [torch.from_numpy(x0[a:c].copy()).cuda() for a, c in G.ranges]
+    xs, info = G.solve(bs, x0s, None, k=k, max_global_iters=iters, tol=tol, mode=mode)
+    G.close()
+    return np.concatenate([x.cpu().numpy() for x in xs]), info
+
+
+MATS = [("s7", W.stencil7_3d, (16,), 128), ("s9", W.stencil9_2d, (98,), 128), ("tref", W.trefethen, (2000,), 128),
+        ("s7big", W.stencil7_3d, (64,), 1024)]
+
+
+@pytest.mark.parametrize("name,gen,args,R", MATS)
+@pytest.mark.parametrize("P", [1, 2, 3, 4])
+@pytest.mark.parametrize("mode,k", [("sync-block", 5), ("jacobi", 1)])
+def test_partitioned_iterates_bitwise(bar, name, gen, args, R, P, mode, k):
+    A = gen(*args)
+    n = A.n
+    b = np.ones(n)
+    x0 = np.random.default_rng(5).uniform(-1, 1, n)
+    blocks = _split(gen, args, n, R, P)
+    for m in (1, 4):
+        xs, i1 = _single(bar, A, b, R, k, mode, m, 0.0, x0)
+        xp, i2 = _loop(blocks, n, R, b, k, mode, m, 0.0, x0)
+        assert np.array_equal(xs, xp), (m, np.abs(xs - xp).max())
+        assert i2["iters"] == m
+    # same stopping iteration at tol 1e-10; the returned iterate is the same bits
+    xs, i1 = _single(bar, A, b, R, k, mode, 20000, 1e-10, np.zeros(n))
+    xp, i2 = _loop(blocks, n, R, b, k, mode, 20000, 1e-10, np.zeros(n))
+    assert i1["iters"] == i2["iters"] and i2["converged"]
+    assert np.array_equal(xs, xp)
+    assert abs(i1["rel_res"] - i2["rel_res"]) <= 1e-12 * i1["rel_res"]
+
+
+@pytest.mark.parametrize("name,gen,args,R", MATS)
+@pytest.mark.parametrize("P", [2, 4])
+def test_partitioned_async_converges(bar, name, gen, args, R, P):
+    A = gen(*args)
+    n = A.n
+    b = np.ones(n)
+    blocks = _split(gen, args, n, R, P)
+    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n))
+    assert info["converged"] and info["rel_res"] <= 1e-10
+    assert O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+def test_plan_errors(bar):
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    A = W.stencil7_3d(8)
+    blk = W.stencil7_3d(8, row_lo=128, row_hi=256)
+    lo, hi = D.ghosts(blk)
+    z = np.zeros(2, dtype=np.int64)
+    rc = np.array([len(lo), len(hi)], dtype=np.int64)
+    idx = np.zeros(0, dtype=np.int32)
+    with pytest.raises(D.BarError):  # row_begin = 128 is not a multiple of R = 96
+        D._create(A.n, blk, 96, 0, 2, 1, rc[::-1].copy(), z, idx, lo, hi, None)
+    with pytest.raises(D.BarError):  # a rank cannot receive from itself
+        D._create(A.n, blk, 64, 0, 2, 1, np.array([0, len(lo) + len(hi)], dtype=np.int64), z, idx, lo, hi, None)

@@ -1,3 +1,3 @@
 timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
-for w in c1 c2 c3; do timeout 300 python tools/sweep_R.py --workload $w --R 128 --modes async,sync-block 2>&1 | grep '^{'; done
-timeout 300 python tools/sweep_R.py --workload c2 --R 448 --k 1,2,5,9 --modes async 2>&1 | grep '^{'
+timeout 900 python bench.py > gpurun_out/bench_c5.json 2> gpurun_out/bench_c5.err; tail -c 2500 gpurun_out/bench_c5.json
+for w in c1 c2 c3 c4; do timeout 600 python bench.py --workload $w --no-cpu-baseline > gpurun_out/bench_$w.json 2>&1; tail -c 400 gpurun_out/bench_$w.json; echo; done
