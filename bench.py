@@ -205,6 +205,7 @@ def main():
     ap.add_argument("--ref-iters", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-p2p", action="store_true", help="multi-GPU async: NCCL halo exchange instead of P2P")
     args = ap.parse_args()
     if args.R is None:
         args.R = WORKLOADS[args.workload][2]
@@ -259,10 +260,24 @@ def main():
         t_gen = time.time() - t0
         t0 = time.time()
         M = bdist.DistMatrix(A, n, args.R, local_rank)
+        p2p = False
+        if args.mode == "async" and not args.no_p2p:
+            # async across GPUs reads peers' x over NVLink (CUDA IPC), no per-iteration collective;
+            # fall back to the NCCL halo exchange on every rank if any rank cannot map its peers
+            try:
+                M.enable_p2p()
+                ok = 1.0
+            except bar.BarError:
+                ok = 0.0
+            p2p = reduce(ok, dist.ReduceOp.MIN) > 0.5
+            if not p2p:
+                M.close()
+                M = bdist.DistMatrix(A, n, args.R, local_rank)
         t_setup = time.time() - t0
         n_loc = rows[1] - rows[0]
         local_bytes = A.nnz * 12.0 + n_loc * 28.0
-        minfo = {"n_local": n_loc, "row_range": list(rows), "nnz_local": A.nnz, "ranks": world}
+        minfo = {"n_local": n_loc, "row_range": list(rows), "nnz_local": A.nnz, "ranks": world,
+                 "exchange": "peer-memory pull (CUDA IPC over NVLink)" if p2p else "NCCL grouped send/recv"}
         del A
     total_bytes = nnz * 12.0 + n * 28.0
     b = torch.ones(n_loc, dtype=torch.float64, device=dev)
@@ -364,7 +379,7 @@ def main():
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload][0]}", "n": n, "nnz": nnz,
                    "mode": args.mode, "k": args.k, "rows_per_block": args.R, "tol": args.tol, "b": "ones",
-                   "x0": "zeros", "parallelism": f"rows/{world}" + (" (NCCL halo send/recv)" if world > 1 else ""),
+                   "x0": "zeros", "parallelism": f"rows/{world}" + (f" ({minfo['exchange']})" if world > 1 else ""),
                    "l2": "inputs > L2 (no flush needed)" if total_bytes / world > 126e6
                    else "inputs L2-resident (latency-bound config)"},
         "global_iters": mean_iters, "global_iters_minmax": [min(iters), max(iters)],

@@ -221,6 +221,24 @@ bar_status bar_dist_solve_loopback(bar_dist *ranks, int nranks, const double *co
                                    double *const *x, int32_t k, int64_t max_global_iters, double tol,
                                    bar_mode mode, void *cuda_stream, bar_solve_info *info);
 
+/*
+ * Asynchronous multi-GPU mode over peer memory (north star: "an async mode reads peers' x over
+ * NVLink P2P with no barrier"; the paper's DK idea, without a master GPU). After
+ * bar_dist_enable_p2p, bar_dist_solve / bar_dist_solve_loopback in BAR_MODE_ASYNC no longer
+ * exchange halos collectively: before every local sweep each rank PULLS its ghost values from
+ * the owners' live iterates with relaxed system-scope loads (x "as it stands", eq. 3) and
+ * pushes its residual partial into every peer's board; ranks only synchronise at chunk
+ * boundaries (a one-int all-reduce of the stop requests) and for the exact confirming residual.
+ *   bar_dist_p2p_handles  128 bytes: CUDA IPC handles of this rank's iterate and board (publish
+ *                         them to the group), and *own_offset (its owned-block offset, in doubles).
+ *   bar_dist_enable_p2p   ghost_src_idx[j] = owner-local row of ghost j (ghost order); handles =
+ *                         nranks * 128 bytes and own_offsets = nranks offsets gathered from every
+ *                         rank, or both NULL for linked loopback ranks (same process).
+ */
+bar_status bar_dist_p2p_handles(bar_dist D, void *handles128, int64_t *own_offset);
+bar_status bar_dist_enable_p2p(bar_dist D, const int32_t *ghost_src_idx, const void *handles,
+                               const int64_t *own_offsets);
+
 /* bar_dist_sweep — measurement entry point: enqueue exactly nsweeps launches of this rank's local
  * block-sweep kernel on its current iterate (no halo exchange, no convergence control, no sync;
  * ghost values are whatever the last exchange left). Local, not collective. */

@@ -33,7 +33,7 @@ MAX_ROWS_PER_BLOCK = 8192
 EXPORTS = ("bar_create_csr", "bar_solve", "bar_sweep", "bar_residual", "bar_matrix_get_info", "bar_destroy",
            "bar_last_error", "bar_dist_ghosts", "bar_dist_localize", "bar_nccl_unique_id", "bar_dist_create",
            "bar_dist_link_loopback", "bar_dist_solve", "bar_dist_solve_loopback", "bar_dist_sweep",
-           "bar_dist_destroy")
+           "bar_dist_p2p_handles", "bar_dist_enable_p2p", "bar_dist_destroy")
 
 
 class SolveInfo(ctypes.Structure):

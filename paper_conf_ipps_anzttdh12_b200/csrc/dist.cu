@@ -37,6 +37,14 @@ struct bar_dist_s {
     std::vector<int64_t> send_cnt, send_off, recv_cnt, recv_pos;  // recv_pos: owned-relative index
     double *part = nullptr;      // device [2]: this rank's [sum r^2, sum b^2]
     double *gathered = nullptr;  // device [2 * nranks]
+    // async over peer memory (bar_dist_enable_p2p)
+    bool p2p = false;
+    int32_t *g_rank = nullptr, *g_idx = nullptr;     // device, per ghost: owner rank, owner-local row
+    double **d_peer_own = nullptr;                  // device [nranks]: owned block of each rank's x
+    double **d_peer_board = nullptr;                // device [nranks]: each rank's board
+    double *board = nullptr;                        // device [2 * nranks]: latest partials of every rank
+    int *d_flag = nullptr;                          // device: stop-request all-reduce
+    std::vector<void *> opened;                     // IPC mappings to close
     bool loopback = true;
     std::vector<bar_dist> peers;  // loopback group (peers[r] is rank r)
 #ifdef BAR_WITH_NCCL
@@ -139,6 +147,72 @@ bar_status reduce_decide(bar_dist *ranks, int nr, bool residual_only, cudaStream
     return BAR_OK;
 }
 
+// ---- async over peer memory ----------------------------------------------------------------
+// Pull every ghost value from its owner's live iterate: x "as it stands" (eq. 3), read over
+// NVLink with relaxed system-scope loads, no synchronisation with the owner.
+__global__ void k_pull_ghosts(double *__restrict__ x_own, int64_t n_glo, int64_t n_local, int64_t n_ghost,
+                              const int32_t *__restrict__ g_rank, const int32_t *__restrict__ g_idx,
+                              double *const *__restrict__ peer_own) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n_ghost;
+         j += (int64_t)gridDim.x * blockDim.x) {
+        const double *src = peer_own[g_rank[j]] + g_idx[j];
+        double v;
+        asm volatile("ld.relaxed.sys.global.f64 %0, [%1];" : "=d"(v) : "l"(src));
+        double *dst = j < n_glo ? x_own - n_glo + j : x_own + n_local + (j - n_glo);
+        asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(dst), "d"(v) : "memory");
+    }
+}
+
+// Push this rank's latest [sum r^2, sum b^2] into slot `rank` of every rank's board.
+__global__ void k_publish(const double *__restrict__ part, double *const *__restrict__ peer_board, int rank,
+                          int nranks) {
+    const int p = threadIdx.x;
+    if (p >= nranks) return;
+    double *dst = peer_board[p] + 2 * rank;
+    asm volatile("st.relaxed.sys.global.f64 [%0], %1;" ::"l"(dst), "d"(part[0]) : "memory");
+    asm volatile("st.relaxed.sys.global.f64 [%0], %1;" ::"l"(dst + 1), "d"(part[1]) : "memory");
+}
+
+bar_status p2p_iteration(bar_dist D, const SweepArgs &a, bar_mode mode, cudaStream_t st) {
+    const int64_t ng = D->n_glo + D->n_ghi;
+    if (ng > 0) {
+        int64_t blocks = (ng + 255) / 256;
+        if (blocks > 1024) blocks = 1024;
+        k_pull_ghosts<<<(unsigned)blocks, 256, 0, st>>>(own(D, D->xa), D->n_glo, D->n_local, ng, D->g_rank, D->g_idx,
+                                                         D->d_peer_own);
+        BAR_CUDA(cudaGetLastError());
+    }
+    BAR_CUDA(launch_sweep(a, mode, st));
+    k_publish<<<1, 32 * ((D->nranks + 31) / 32), 0, st>>>(D->part, D->d_peer_board, D->rank, D->nranks);
+    BAR_CUDA(cudaGetLastError());
+    // the board holds every rank's latest partial (others' possibly a few launches old)
+    BAR_CUDA(launch_dist_decide(D->A->W.state, D->board, D->nranks, false, st));
+    return BAR_OK;
+}
+
+// Chunk-boundary agreement on the stop requests of all ranks (the only synchronisation of the
+// asynchronous multi-GPU mode besides the exact confirming residual).
+bar_status agree_stop(bar_dist *ranks, int nr, cudaStream_t st, bool &any) {
+    any = false;
+    for (int i = 0; i < nr; ++i) {
+        bar_status r = read_state(ranks[i]->A, st);
+        if (r != BAR_OK) return r;
+        any = any || ranks[i]->A->W.h_state->stop != 0;
+    }
+    if (!ranks[0]->loopback) {
+#ifdef BAR_WITH_NCCL
+        bar_dist D = ranks[0];
+        int v = any ? 1 : 0, out = 0;
+        BAR_CUDA(cudaMemcpyAsync(D->d_flag, &v, sizeof(int), cudaMemcpyHostToDevice, st));
+        BAR_NCCL(ncclAllReduce(D->d_flag, D->d_flag, 1, ncclInt32, ncclMax, D->comm, st));
+        BAR_CUDA(cudaMemcpyAsync(&out, D->d_flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+        BAR_CUDA(cudaStreamSynchronize(st));
+        any = out != 0;
+#endif
+    }
+    return BAR_OK;
+}
+
 // The collective solve for the ranks this process drives (1 with NCCL, all with loopback).
 bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const double *const *x0, double *const *x,
                       int32_t k, int64_t max_iters, double tol, bar_mode mode, cudaStream_t st,
@@ -167,6 +241,19 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
     int64_t launches = nr;
     bar_dist D0 = ranks[0];
     DevState &H = *D0->A->W.h_state;
+    const bool p2p = mode == BAR_MODE_ASYNC && D0->p2p;
+    if (p2p) {  // boards start "unknown": huge partials keep the estimate above tol until published
+        std::vector<double> init(2 * (size_t)D0->nranks, 1e300);
+        for (int i = 0; i < nr; ++i)
+            BAR_CUDA(cudaMemcpy(ranks[i]->board, init.data(), sizeof(double) * init.size(), cudaMemcpyHostToDevice));
+        if (!D0->loopback) {
+#ifdef BAR_WITH_NCCL
+            BAR_CUDA(cudaStreamSynchronize(st));  // every rank's board reset before any peer publishes
+            BAR_NCCL(ncclAllReduce(D0->d_flag, D0->d_flag, 1, ncclInt32, ncclMax, D0->comm, st));
+            BAR_CUDA(cudaStreamSynchronize(st));
+#endif
+        }
+    }
     int64_t issued = 0, chunk = 8;
     int64_t iters = 0;
     double rel = 0.0;
@@ -183,6 +270,16 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                 const bool odd = (m & 1) || mode == BAR_MODE_ASYNC;
                 const std::vector<double *> &vin = odd ? xa : xb;
                 const std::vector<double *> &vout = mode == BAR_MODE_ASYNC ? xa : (odd ? xb : xa);
+                if (p2p) {  // no collective: pull ghosts, sweep, publish, estimate — per rank
+                    for (int i = 0; i < nr; ++i) {
+                        bar_dist D = ranks[i];
+                        SweepArgs a{&D->A->L, D->bbuf, own(D, D->xa), own(D, D->xa), k, D->A->W.state,
+                                    D->A->W.partials, nullptr, D->part};
+                        if ((r = p2p_iteration(D, a, mode, st)) != BAR_OK) return r;
+                    }
+                    launches += 4 * nr;
+                    continue;
+                }
                 if ((r = exchange(ranks, nr, vin.data(), st)) != BAR_OK) return r;
                 for (int i = 0; i < nr; ++i) {
                     bar_dist D = ranks[i];
@@ -194,8 +291,12 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                 launches += 2 * nr;
             }
             issued += c;
-            if ((r = read_state(D0->A, st)) != BAR_OK) return r;
-            stopped = H.stop != 0;
+            if (p2p) {
+                if ((r = agree_stop(ranks, nr, st, stopped)) != BAR_OK) return r;
+            } else {
+                if ((r = read_state(D0->A, st)) != BAR_OK) return r;
+                stopped = H.stop != 0;
+            }
             chunk = std::min<int64_t>(chunk * 2, 256);
         }
         if (stopped && mode != BAR_MODE_ASYNC) {
@@ -523,6 +624,81 @@ bar_status bar_dist_solve_loopback(bar_dist *ranks, int nranks, const double *co
     return dist_solve(ranks, nranks, b, x0, x, k, max_global_iters, tol, mode, (cudaStream_t)cuda_stream, info);
 }
 
+bar_status bar_dist_p2p_handles(bar_dist D, void *handles128, int64_t *own_offset) {
+    if (!D || !handles128 || !own_offset) {
+        set_error("NULL argument");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(D->device);
+    if (!D->board) BAR_CUDA(cudaMalloc(&D->board, sizeof(double) * 2 * (size_t)D->nranks));
+    cudaIpcMemHandle_t hx, hb;
+    BAR_CUDA(cudaIpcGetMemHandle(&hx, D->xa));
+    BAR_CUDA(cudaIpcGetMemHandle(&hb, D->board));
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+    std::memcpy(handles128, &hx, 64);
+    std::memcpy((char *)handles128 + 64, &hb, 64);
+    *own_offset = D->glo_pad;
+    return BAR_OK;
+}
+
+bar_status bar_dist_enable_p2p(bar_dist D, const int32_t *ghost_src_idx, const void *handles,
+                               const int64_t *own_offsets) {
+    const int64_t ng = D ? D->n_glo + D->n_ghi : 0;
+    if (!D || (ng > 0 && !ghost_src_idx) || ((handles == nullptr) != (own_offsets == nullptr)) ||
+        (handles == nullptr && !D->loopback) || (D->loopback && (int)D->peers.size() != D->nranks)) {
+        set_error("invalid argument (loopback ranks must be linked first; NCCL ranks need handles)");
+        return BAR_ERR_INVALID_ARG;
+    }
+    DeviceGuard g(D->device);
+    if (!D->board) BAR_CUDA(cudaMalloc(&D->board, sizeof(double) * 2 * (size_t)D->nranks));
+    if (!D->d_flag) BAR_CUDA(cudaMalloc(&D->d_flag, sizeof(int)));
+    BAR_CUDA(cudaMemset(D->d_flag, 0, sizeof(int)));
+    // ghost j's owner: ghosts are ordered by owner (recv_counts), owners' ranges are contiguous
+    std::vector<int32_t> grank(ng), gidx(ng);
+    {
+        int64_t j = 0;
+        for (int p = 0; p < D->nranks; ++p)
+            for (int64_t c = 0; c < D->recv_cnt[p]; ++c, ++j) grank[j] = p;
+    }
+    for (int64_t j = 0; j < ng; ++j) gidx[j] = ghost_src_idx[j];
+    std::vector<double *> pown(D->nranks), pboard(D->nranks);
+    for (int p = 0; p < D->nranks; ++p) {
+        if (handles == nullptr) {  // loopback: the peers live in this process
+            bar_dist P = D->peers[p];
+            if (!P->board) BAR_CUDA(cudaMalloc(&P->board, sizeof(double) * 2 * (size_t)P->nranks));
+            pown[p] = own(P, P->xa);
+            pboard[p] = P->board;
+        } else if (p == D->rank) {
+            pown[p] = own(D, D->xa);
+            pboard[p] = D->board;
+        } else {
+            cudaIpcMemHandle_t hx, hb;
+            std::memcpy(&hx, (const char *)handles + 128 * (size_t)p, 64);
+            std::memcpy(&hb, (const char *)handles + 128 * (size_t)p + 64, 64);
+            void *px = nullptr, *pb = nullptr;
+            BAR_CUDA(cudaIpcOpenMemHandle(&px, hx, cudaIpcMemLazyEnablePeerAccess));
+            D->opened.push_back(px);
+            BAR_CUDA(cudaIpcOpenMemHandle(&pb, hb, cudaIpcMemLazyEnablePeerAccess));
+            D->opened.push_back(pb);
+            pown[p] = (double *)px + own_offsets[p];
+            pboard[p] = (double *)pb;
+        }
+    }
+    cudaFree(D->g_rank);
+    cudaFree(D->g_idx);
+    cudaFree(D->d_peer_own);
+    cudaFree(D->d_peer_board);
+    D->g_rank = D->g_idx = nullptr;
+    D->d_peer_own = D->d_peer_board = nullptr;
+    bar_status r;
+    if ((r = to_device(grank.data(), ng, &D->g_rank)) != BAR_OK) return r;
+    if ((r = to_device(gidx.data(), ng, &D->g_idx)) != BAR_OK) return r;
+    if ((r = to_device(pown.data(), D->nranks, &D->d_peer_own)) != BAR_OK) return r;
+    if ((r = to_device(pboard.data(), D->nranks, &D->d_peer_board)) != BAR_OK) return r;
+    D->p2p = true;
+    return BAR_OK;
+}
+
 bar_status bar_dist_sweep(bar_dist D, int32_t k, int64_t nsweeps, bar_mode mode, void *cuda_stream) {
     if (!D || nsweeps < 0 || (mode != BAR_MODE_JACOBI && k < 1)) {
         set_error("invalid argument");
@@ -549,6 +725,13 @@ void bar_dist_destroy(bar_dist D) {
 #ifdef BAR_WITH_NCCL
     if (D->comm) ncclCommDestroy(D->comm);
 #endif
+    for (void *p : D->opened) cudaIpcCloseMemHandle(p);
+    cudaFree(D->g_rank);
+    cudaFree(D->g_idx);
+    cudaFree(D->d_peer_own);
+    cudaFree(D->d_peer_board);
+    cudaFree(D->board);
+    cudaFree(D->d_flag);
     bar_destroy(D->A);
     cudaFree(D->xa);
     cudaFree(D->xb);

@@ -37,6 +37,10 @@ _lib.bar_dist_solve_loopback.restype = ctypes.c_int
 _lib.bar_dist_solve_loopback.argtypes = [ctypes.POINTER(_vp), ctypes.c_int, ctypes.POINTER(_vp), ctypes.POINTER(_vp),
                                          ctypes.POINTER(_vp), _i32, _i64, _f64, ctypes.c_int, _vp,
                                          ctypes.POINTER(SolveInfo)]
+_lib.bar_dist_p2p_handles.restype = ctypes.c_int
+_lib.bar_dist_p2p_handles.argtypes = [_vp, _vp, ctypes.POINTER(_i64)]
+_lib.bar_dist_enable_p2p.restype = ctypes.c_int
+_lib.bar_dist_enable_p2p.argtypes = [_vp, _vp, _vp, _vp]
 _lib.bar_dist_sweep.restype = ctypes.c_int
 _lib.bar_dist_sweep.argtypes = [_vp, _i32, _i64, ctypes.c_int, _vp]
 _lib.bar_dist_destroy.restype = None
@@ -103,6 +107,17 @@ def make_plan(rank: int, ranges, ghost_lists):
     return recv_counts, send_counts, np.ascontiguousarray(send_idx, dtype=np.int32)
 
 
+def ghost_sources(ranges, ghost_cols):
+    """Owner-local row of every ghost column (ghost order), for bar_dist_enable_p2p."""
+    g = np.asarray(ghost_cols, dtype=np.int64)
+    if len(g) == 0:
+        return np.zeros(0, dtype=np.int32)
+    starts = np.array([r[0] for r in ranges])
+    ends = np.array([r[1] for r in ranges])
+    o = np.searchsorted(ends, g, side="right")
+    return np.ascontiguousarray(g - starts[o], dtype=np.int32)
+
+
 def _create(n_global, A_rows, R, device, nranks, rank, recv_counts, send_counts, send_idx, lo, hi, nccl_id):
     col_local = localize(A_rows, lo, hi)
     rp = np.ascontiguousarray(A_rows.rowptr, dtype=np.int32)
@@ -146,6 +161,21 @@ class DistMatrix:
                               hi, nid[0])
         self.rank, self.nranks, self.n_local = r, P, A_rows.row_hi - A_rows.row_lo
         self.row_lo, self.row_hi = A_rows.row_lo, A_rows.row_hi
+        self.ranges, self.ghost_cols, self.group = ranges, np.concatenate([lo, hi]), group
+
+    def enable_p2p(self):
+        """Async over peer memory: exchange CUDA IPC handles of every rank's iterate and board."""
+        import torch.distributed as dist
+
+        buf = ctypes.create_string_buffer(128)
+        off = _i64()
+        _check(_lib.bar_dist_p2p_handles(self.handle, buf, ctypes.byref(off)))
+        allh = [None] * self.nranks
+        dist.all_gather_object(allh, (buf.raw, off.value), group=self.group)
+        handles = ctypes.create_string_buffer(b"".join(h for h, _ in allh), 128 * self.nranks)
+        offs = np.array([o for _, o in allh], dtype=np.int64)
+        src = ghost_sources(self.ranges, self.ghost_cols)
+        _check(_lib.bar_dist_enable_p2p(self.handle, _ptr(src), handles, _ptr(offs)))
 
     def solve(self, b, x0=None, x=None, k=5, max_global_iters=20000, tol=1e-10, mode="async", stream=None,
               raise_on_error=True):
@@ -195,6 +225,13 @@ class LoopbackGroup:
         _check(_lib.bar_dist_link_loopback(self._arr, P))
         self.ranges = ranges
         self.nranks = P
+        self.ghost_cols = glists
+
+    def enable_p2p(self):
+        """Async mode pulls ghosts from the other ranks' live iterates (no exchange, no barrier)."""
+        for r, h in enumerate(self.handles):
+            src = ghost_sources(self.ranges, self.ghost_cols[r])
+            _check(_lib.bar_dist_enable_p2p(h, _ptr(src), None, None))
 
     def solve(self, bs, x0s=None, xs=None, k=5, max_global_iters=20000, tol=1e-10, mode="async", stream=None,
               raise_on_error=True):
