@@ -57,6 +57,14 @@ def _load():
     lib.oracle_solve.restype = ctypes.c_int
     lib.oracle_solve.argtypes = [i32, i64, i32p, i32p, f64p, f64p, f64p, f64p, i64, i32, i64, ctypes.c_double,
                                  ctypes.POINTER(i64), f64p, ctypes.POINTER(i32), f64p]
+    u8p = ctypes.POINTER(ctypes.c_uint8)
+    lib.oracle_solve_ex.restype = ctypes.c_int
+    lib.oracle_solve_ex.argtypes = lib.oracle_solve.argtypes + [ctypes.c_double, u8p, i64, i64]
+    lib.oracle_jacobi_step_ex.restype = ctypes.c_int
+    lib.oracle_jacobi_step_ex.argtypes = [i64, i32p, i32p, f64p, f64p, f64p, f64p, ctypes.c_double, u8p]
+    lib.oracle_block_jacobi_step_ex.restype = ctypes.c_int
+    lib.oracle_block_jacobi_step_ex.argtypes = [i64, i32p, i32p, f64p, f64p, i64, i32, f64p, f64p, ctypes.c_double,
+                                                u8p]
     _lib = lib
     return lib
 
@@ -179,8 +187,12 @@ class SolveResult:
 
 
 def solve(A, b, x0=None, method: int = BLOCK_JACOBI, R: int = 128, k: int = 5,
-          max_iters: int = 20000, tol: float = 1e-10) -> SolveResult:
-    """O5: iterate until rel_res(x^m) <= tol (first such m) or max_iters."""
+          max_iters: int = 20000, tol: float = 1e-10, tau: float = 1.0, frozen=None,
+          fail_start: int = 0, fail_stop: int = -1) -> SolveResult:
+    """O5: iterate until rel_res(x^m) <= tol (first such m) or max_iters.
+
+    N3: ``tau`` scales every update (B = I - tau D^-1 A). N1: components with
+    ``frozen[i]`` do not update in global iterations fail_start <= m < fail_stop."""
     lib = _load()
     n = len(A.rowptr) - 1
     rp, prp = _i32(A.rowptr)
@@ -195,9 +207,38 @@ def solve(A, b, x0=None, method: int = BLOCK_JACOBI, R: int = 128, k: int = 5,
     iters = ctypes.c_int64()
     rel = ctypes.c_double()
     conv = ctypes.c_int32()
-    st = lib.oracle_solve(method, n, prp, pc, pv, pb, px0, out.ctypes.data_as(ctypes.POINTER(ctypes.c_double)),
-                          R, k, max_iters, tol, ctypes.byref(iters), ctypes.byref(rel), ctypes.byref(conv),
-                          hist.ctypes.data_as(ctypes.POINTER(ctypes.c_double)))
+    fz = None
+    pfz = None
+    if frozen is not None:
+        fz = np.ascontiguousarray(frozen, dtype=np.uint8)
+        pfz = fz.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+    st = lib.oracle_solve_ex(method, n, prp, pc, pv, pb, px0, out.ctypes.data_as(ctypes.POINTER(ctypes.c_double)),
+                             R, k, max_iters, tol, ctypes.byref(iters), ctypes.byref(rel), ctypes.byref(conv),
+                             hist.ctypes.data_as(ctypes.POINTER(ctypes.c_double)), tau, pfz, fail_start, fail_stop)
     if st == ERR:
         raise ValueError("oracle_solve failed")
     return SolveResult(out, iters.value, rel.value, bool(conv.value), st, hist[: iters.value + 1])
+
+
+def step_ex(A, b, x_old, method: int = BLOCK_JACOBI, R: int = 128, k: int = 5, tau: float = 1.0, frozen=None):
+    """One global iteration of O1/O2 with the N1/N3 options."""
+    lib = _load()
+    n = len(A.rowptr) - 1
+    rp, prp = _i32(A.rowptr)
+    c, pc = _i32(A.col)
+    v, pv = _f64(A.val)
+    bb, pb = _f64(b)
+    xo, pxo = _f64(x_old)
+    out = np.empty(n)
+    po = out.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+    pfz = None
+    if frozen is not None:
+        fz = np.ascontiguousarray(frozen, dtype=np.uint8)
+        pfz = fz.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+    if method == JACOBI:
+        rc = lib.oracle_jacobi_step_ex(n, prp, pc, pv, pb, pxo, po, tau, pfz)
+    else:
+        rc = lib.oracle_block_jacobi_step_ex(n, prp, pc, pv, pb, R, k, pxo, po, tau, pfz)
+    if rc:
+        raise ValueError("step failed")
+    return out

@@ -24,6 +24,9 @@
  *   oracle_block_jacobi_subdomain  one subdomain of O2 (for sampled checks at full size).
  *   oracle_gauss_seidel_step  O3  forward Gauss-Seidel, in place, natural order.
  *   oracle_residual_norm      O4  ||b - A x||_2 ("residuals ... always in the l2-norm").
+ *   oracle_*_step_ex / oracle_solve_ex  N1 failure injection (§4.5: frozen components)
+ *                                 and N3 tau-scaled relaxation (B = I - tau D^-1 A),
+ *                                 DESIGN.md readings R17/R18.
  *   oracle_solve              O5  stopping rule of DESIGN.md reading R2/R6: check x^0, then
  *                                 return the first x^m with ||b-Ax^m||/||b|| <= tol, else
  *                                 x^{max_iters} with converged = 0; divergence => status 2.
@@ -175,6 +178,67 @@ int oracle_gauss_seidel_step(int64_t n, const int32_t *rowptr, const int32_t *co
     return 0;
 }
 
+/* ------------------------------------------- N1 / N3 extensions (oracle) ---- */
+/* tau-scaled relaxation (B = I - tau D^-1 A) applied to every update of O1/O2:    */
+/*   x_new = x_old + tau * (v - x_old), v the unscaled update; tau == 1 gives v exactly.       */
+/* Failure injection (§4.5): components with frozen[i] != 0 keep their value.         */
+static double relax(double xold, double v, double tau) { return tau == 1.0 ? v : xold + tau * (v - xold); }
+
+int oracle_jacobi_step_ex(int64_t n, const int32_t *rowptr, const int32_t *col, const double *val,
+                          const double *b, const double *x_old, double *x_new, double tau,
+                          const uint8_t *frozen) {
+    int rc = oracle_jacobi_step(n, rowptr, col, val, b, x_old, x_new);
+    if (rc) return rc;
+    for (int64_t i = 0; i < n; ++i) {
+        if (frozen && frozen[i]) x_new[i] = x_old[i];
+        else x_new[i] = relax(x_old[i], x_new[i], tau);
+    }
+    return 0;
+}
+
+int oracle_block_jacobi_step_ex(int64_t n, const int32_t *rowptr, const int32_t *col, const double *val,
+                                const double *b, int64_t R, int32_t k, const double *x_old, double *x_new,
+                                double tau, const uint8_t *frozen) {
+    if (R < 1 || k < 1) return -2;
+    for (int64_t TS = 0; TS < n; TS += R) {
+        int64_t TE = TS + R < n ? TS + R : n, nl = TE - TS;
+        double *y = (double *)malloc(sizeof(double) * (size_t)nl);
+        double *yn = (double *)malloc(sizeof(double) * (size_t)nl);
+        double *s = (double *)malloc(sizeof(double) * (size_t)nl);
+        if (!y || !yn || !s) { free(y); free(yn); free(s); return -3; }
+        for (int64_t i = 0; i < nl; ++i) {
+            double acc = b[TS + i];
+            for (int32_t e = rowptr[TS + i]; e < rowptr[TS + i + 1]; ++e) {
+                int64_t j = col[e];
+                if (j >= TS && j < TE) continue;
+                double t = val[e] * x_old[j];
+                acc = acc - t;
+            }
+            s[i] = acc;
+            y[i] = x_old[TS + i];
+        }
+        for (int32_t t = 0; t < k; ++t) {
+            for (int64_t i = 0; i < nl; ++i) {
+                int64_t gi = TS + i;
+                if (frozen && frozen[gi]) { yn[i] = y[i]; continue; }
+                double acc = s[i], aii = 0.0;
+                for (int32_t e = rowptr[gi]; e < rowptr[gi + 1]; ++e) {
+                    int64_t j = col[e];
+                    if (j < TS || j >= TE) continue;
+                    if (j == gi) { aii = val[e]; continue; }
+                    double tt = val[e] * y[j - TS];
+                    acc = acc - tt;
+                }
+                yn[i] = relax(y[i], acc / aii, tau);
+            }
+            memcpy(y, yn, sizeof(double) * (size_t)nl);
+        }
+        memcpy(x_new + TS, y, sizeof(double) * (size_t)nl);
+        free(y); free(yn); free(s);
+    }
+    return 0;
+}
+
 /* ---------------------------------------------------------------- O5 ---- */
 enum { ORACLE_JACOBI = 0, ORACLE_BLOCK_JACOBI = 1, ORACLE_GAUSS_SEIDEL = 2 };
 enum { ORACLE_OK = 0, ORACLE_ERR = 1, ORACLE_DIVERGED = 2 };
@@ -182,10 +246,14 @@ enum { ORACLE_OK = 0, ORACLE_ERR = 1, ORACLE_DIVERGED = 2 };
 /* Solve A x = b from x0 with the chosen relaxation until rel_res <= tol or       */
 /* max_iters global iterations. res_hist (nullable) gets rel_res(x^m) for          */
 /* m = 0..iters (length >= max_iters + 1).                                          */
-int oracle_solve(int32_t method, int64_t n, const int32_t *rowptr, const int32_t *col, const double *val,
-                 const double *b, const double *x0, double *x_out, int64_t R, int32_t k,
-                 int64_t max_iters, double tol, int64_t *iters_out, double *rel_res_out,
-                 int32_t *converged_out, double *res_hist) {
+/* oracle_solve_ex: O5 with the N1/N3 options: tau-scaling of every update, and components with */
+/* frozen[i] != 0 not updated in global iterations m with fail_start <= m < fail_stop            */
+/* (fail_stop < 0: never recover). tau = 1, frozen = NULL gives oracle_solve.                    */
+int oracle_solve_ex(int32_t method, int64_t n, const int32_t *rowptr, const int32_t *col, const double *val,
+                    const double *b, const double *x0, double *x_out, int64_t R, int32_t k,
+                    int64_t max_iters, double tol, int64_t *iters_out, double *rel_res_out,
+                    int32_t *converged_out, double *res_hist, double tau, const uint8_t *frozen,
+                    int64_t fail_start, int64_t fail_stop) {
     double bn = oracle_norm2(n, b);
     *iters_out = 0; *converged_out = 0; *rel_res_out = 0.0;
     if (bn == 0.0) {                       /* b = 0 => x = 0 (reading R2) */
@@ -205,10 +273,14 @@ int oracle_solve(int32_t method, int64_t n, const int32_t *rowptr, const int32_t
     if (!(rel <= tol)) {
         for (m = 1; m <= max_iters; ++m) {
             int rc = 0;
+            const uint8_t *fr = (frozen && m >= fail_start && (fail_stop < 0 || m < fail_stop)) ? frozen : NULL;
+            const int plain = tau == 1.0 && fr == NULL;
             if (method == ORACLE_JACOBI) {
-                rc = oracle_jacobi_step(n, rowptr, col, val, b, xa, xb);
+                rc = plain ? oracle_jacobi_step(n, rowptr, col, val, b, xa, xb)
+                           : oracle_jacobi_step_ex(n, rowptr, col, val, b, xa, xb, tau, fr);
             } else if (method == ORACLE_BLOCK_JACOBI) {
-                rc = oracle_block_jacobi_step(n, rowptr, col, val, b, R, k, xa, xb);
+                rc = plain ? oracle_block_jacobi_step(n, rowptr, col, val, b, R, k, xa, xb)
+                           : oracle_block_jacobi_step_ex(n, rowptr, col, val, b, R, k, xa, xb, tau, fr);
             } else if (method == ORACLE_GAUSS_SEIDEL) {
                 memcpy(xb, xa, sizeof(double) * (size_t)n);
                 rc = oracle_gauss_seidel_step(n, rowptr, col, val, b, xb);
@@ -230,4 +302,12 @@ int oracle_solve(int32_t method, int64_t n, const int32_t *rowptr, const int32_t
     *converged_out = (status == ORACLE_OK && rel <= tol) ? 1 : 0;
     free(xa); free(xb);
     return status;
+}
+
+int oracle_solve(int32_t method, int64_t n, const int32_t *rowptr, const int32_t *col, const double *val,
+                 const double *b, const double *x0, double *x_out, int64_t R, int32_t k,
+                 int64_t max_iters, double tol, int64_t *iters_out, double *rel_res_out,
+                 int32_t *converged_out, double *res_hist) {
+    return oracle_solve_ex(method, n, rowptr, col, val, b, x0, x_out, R, k, max_iters, tol, iters_out,
+                           rel_res_out, converged_out, res_hist, 1.0, NULL, 0, -1);
 }

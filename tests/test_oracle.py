@@ -289,3 +289,83 @@ def test_max_iters_not_converged():
     r = O.solve(A, np.ones(2000), method=O.JACOBI, tol=1e-10, max_iters=20)
     assert r.iters == 20 and not r.converged and r.rel_res > 1e-10
     assert abs(r.rel_res - O.rel_res(A, np.ones(2000), r.x)) == 0
+
+
+# ------------------------------------------------ N3: tau-scaled relaxation
+def test_tau_jacobi_matches_matrix_form():
+    """x_new = x + tau D^-1 (b - A x)  (B = I - tau D^-1 A)."""
+    rng = np.random.default_rng(21)
+    A = W.random_dd(60, 5, seed=21)
+    Ad = _dense(A)
+    b, x = rng.standard_normal(60), rng.standard_normal(60)
+    for tau in (0.5, 0.8, 1.3):
+        ref = x + tau * (b - Ad @ x) / np.diag(Ad)
+        np.testing.assert_allclose(O.step_ex(A, b, x, O.JACOBI, tau=tau), ref, rtol=0, atol=1e-13 * np.abs(ref).max())
+    # tau = 1 is the unscaled method, bit for bit
+    assert np.array_equal(O.step_ex(A, b, x, O.JACOBI, tau=1.0), O.jacobi_step(A, b, x))
+
+
+def test_tau_block_R_ge_n_is_k_tau_jacobi():
+    A = W.random_dd(40, 5, seed=22)
+    b, x = np.ones(40), np.random.default_rng(2).standard_normal(40)
+    y = x
+    for _ in range(3):
+        y = O.step_ex(A, b, y, O.JACOBI, tau=0.7)
+    assert np.array_equal(O.step_ex(A, b, x, O.BLOCK_JACOBI, R=40, k=3, tau=0.7), y)
+
+
+def test_tau_makes_rho_gt_1_spd_converge():
+    """SPD with rho(B) > 1 (s1rmt3m1-like) diverges unscaled but converges with
+    tau = 2/(lambda_1 + lambda_n) of D^-1 A."""
+    n = 12
+    Ad = np.eye(n) + 0.3 * np.ones((n, n))
+    rp = np.arange(0, n * n + 1, n, dtype=np.int32)
+    A = W.CSR(n, rp, np.tile(np.arange(n, dtype=np.int32), n), Ad.ravel())
+    DA = Ad / np.diag(Ad)[:, None]
+    lam = np.linalg.eigvals(DA).real
+    assert np.abs(np.linalg.eigvals(np.eye(n) - DA)).max() > 1
+    tau = 2.0 / (lam.min() + lam.max())
+    b = np.arange(n, dtype=float)
+    assert O.solve(A, b, method=O.JACOBI, tol=1e-12, max_iters=5000).status == O.DIVERGED
+    # (the two-stage method with k > 1 inner tau-sweeps is not covered by this choice of tau:
+    # its iteration matrix differs; DESIGN.md reading R17)
+    for meth, R, k in [(O.JACOBI, 1, 1), (O.BLOCK_JACOBI, 4, 1)]:
+        r = O.solve(A, b, method=meth, R=R, k=k, tol=1e-12, max_iters=5000, tau=tau)
+        assert r.converged
+        np.testing.assert_allclose(r.x, np.linalg.solve(Ad, b), rtol=0, atol=1e-10)
+
+
+# ------------------------------------------------ N1: failure injection (P:1139, §4.5)
+def test_frozen_components_keep_their_value():
+    A = W.trefethen(500)
+    b, x = np.ones(500), np.random.default_rng(3).standard_normal(500)
+    frozen = (np.random.default_rng(4).random(500) < 0.25).astype(np.uint8)
+    for meth in (O.JACOBI, O.BLOCK_JACOBI):
+        y = O.step_ex(A, b, x, meth, R=64, k=5, frozen=frozen)
+        assert np.array_equal(y[frozen == 1], x[frozen == 1])
+        free = O.step_ex(A, b, x, meth, R=64, k=5)
+        if meth == O.JACOBI:  # unaffected rows are the plain update (they read x_old)
+            assert np.array_equal(y[frozen == 0], free[frozen == 0])
+    # masked Jacobi in matrix form
+    Ad = _dense(A)
+    ref = np.where(frozen == 1, x, np.linalg.solve(np.diag(np.diag(Ad)), b - (Ad - np.diag(np.diag(Ad))) @ x))
+    np.testing.assert_allclose(O.step_ex(A, b, x, O.JACOBI, frozen=frozen), ref, rtol=0, atol=1e-13)
+
+
+def test_failure_and_recovery_delay():
+    """25% of the components fail at t0 = 10 and recover after tr iterations: the solve still
+    converges to the same solution, later; without recovery it cannot converge (Fig. 10)."""
+    A = W.trefethen(2000)
+    b = np.ones(2000)
+    frozen = (np.random.default_rng(5).random(2000) < 0.25).astype(np.uint8)
+    base = O.solve(A, b, method=O.BLOCK_JACOBI, R=128, k=5, tol=1e-10)
+    prev = base.iters
+    for tr in (10, 20, 30):
+        r = O.solve(A, b, method=O.BLOCK_JACOBI, R=128, k=5, tol=1e-10, frozen=frozen, fail_start=10,
+                    fail_stop=10 + tr)
+        assert r.converged and r.iters > prev
+        assert np.abs(r.x - base.x).max() < 1e-8 * np.abs(base.x).max()
+        prev = r.iters
+    never = O.solve(A, b, method=O.BLOCK_JACOBI, R=128, k=5, tol=1e-10, frozen=frozen, fail_start=10, fail_stop=-1,
+                    max_iters=300)
+    assert not never.converged
