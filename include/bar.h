@@ -124,6 +124,34 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
                      bar_solve_info *info);
 
 /*
+ * bar_solve_ex — bar_solve with the options of SURVEY §8(f)'s next rows (opts may be NULL):
+ *   tau        N3, τ-scaled relaxation: every update x <- x + tau (v - x), i.e. the
+ *              iteration matrix B = I - tau D^-1 A (tau = 2/(lambda_1 + lambda_n) of D^-1 A makes
+ *              Jacobi converge for SPD systems with rho(B) > 1, like s1rmt3m1). 1 = the paper's methods.
+ *   fail_mask  N1, failure injection (§4.5): n bytes (host or device), nonzero = the
+ *              component "fails": it keeps its value in global iterations m (1-based: the m-th
+ *              global iteration produces x^(m)) with fail_start <= m < fail_stop; fail_stop < 0 =
+ *              never recovers. NULL = no failures.
+ *   res_history  HOST double[max_global_iters + 1] (nullable): sync modes rel_res(x^(m)) for
+ *              m = 0..iters (exact up to the summation order); async the fused per-iteration
+ *              estimate (x as each block saw it). Entries past iters are left untouched.
+ *   async_single_launch  -1 auto, 0 one launch per global iteration, 1 the fully asynchronous
+ *              single-launch kernel (falls back silently where it does not apply). Options
+ *              tau != 1, fail_mask and res_history imply 0.
+ */
+typedef struct {
+    double tau;
+    const uint8_t *fail_mask;
+    int64_t fail_start, fail_stop;
+    double *res_history;
+    int32_t async_single_launch;
+} bar_solve_opts;
+
+bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double *x, int32_t k,
+                        int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
+                        bar_solve_info *info, const bar_solve_opts *opts);
+
+/*
  * bar_residual — res_norm2 = ||b - A x||_2 (and b_norm2 = ||b||_2 if non-NULL), computed on the
  * device with a fixed-order (deterministic) reduction. b, x device or host.
  * Errors: BAR_ERR_INVALID_ARG, BAR_ERR_CUDA, BAR_ERR_OOM.

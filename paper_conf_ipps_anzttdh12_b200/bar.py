@@ -30,7 +30,7 @@ STATUS = {0: "BAR_OK", 1: "BAR_ERR_INVALID_ARG", 2: "BAR_ERR_BAD_CSR", 3: "BAR_E
 MAX_ROWS_PER_BLOCK = 8192
 
 # every symbol include/bar.h declares (tests check the export table against the header)
-EXPORTS = ("bar_create_csr", "bar_solve", "bar_sweep", "bar_residual", "bar_matrix_get_info", "bar_destroy",
+EXPORTS = ("bar_create_csr", "bar_solve", "bar_solve_ex", "bar_sweep", "bar_residual", "bar_matrix_get_info", "bar_destroy",
            "bar_last_error", "bar_dist_ghosts", "bar_dist_localize", "bar_nccl_unique_id", "bar_dist_create",
            "bar_dist_link_loopback", "bar_dist_solve", "bar_dist_solve_loopback", "bar_dist_sweep",
            "bar_dist_p2p_handles", "bar_dist_enable_p2p", "bar_dist_destroy")
@@ -43,6 +43,12 @@ class SolveInfo(ctypes.Structure):
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class SolveOpts(ctypes.Structure):
+    _fields_ = [("tau", ctypes.c_double), ("fail_mask", ctypes.c_void_p), ("fail_start", ctypes.c_int64),
+                ("fail_stop", ctypes.c_int64), ("res_history", ctypes.c_void_p),
+                ("async_single_launch", ctypes.c_int32)]
 
 
 class MatrixInfo(ctypes.Structure):
@@ -60,6 +66,9 @@ _lib.bar_create_csr.restype = ctypes.c_int
 _lib.bar_create_csr.argtypes = [_i64, _i64, _vp, _vp, _vp, _i32, ctypes.c_int, ctypes.POINTER(_vp)]
 _lib.bar_solve.restype = ctypes.c_int
 _lib.bar_solve.argtypes = [_vp, _vp, _vp, _vp, _i32, _i64, _f64, ctypes.c_int, _vp, ctypes.POINTER(SolveInfo)]
+_lib.bar_solve_ex.restype = ctypes.c_int
+_lib.bar_solve_ex.argtypes = [_vp, _vp, _vp, _vp, _i32, _i64, _f64, ctypes.c_int, _vp, ctypes.POINTER(SolveInfo),
+                              ctypes.POINTER(SolveOpts)]
 _lib.bar_sweep.restype = ctypes.c_int
 _lib.bar_sweep.argtypes = [_vp, _vp, _vp, _i32, _i64, ctypes.c_int, _vp]
 _lib.bar_residual.restype = ctypes.c_int
@@ -120,6 +129,28 @@ def bar_solve(A, b, x0, x, k, max_global_iters, tol, mode, cuda_stream=None, rai
     return st, info
 
 
+def bar_solve_ex(A, b, x0, x, k, max_global_iters, tol, mode, cuda_stream=None, raise_on_error=True, tau=1.0,
+                 fail_mask=None, fail_start=0, fail_stop=-1, history=None, async_single_launch=-1):
+    """bar_solve with the options struct (N1 failure injection, N3 tau-scaling, residual history)."""
+    info = SolveInfo()
+    if isinstance(mode, str):
+        mode = MODES[mode]
+    opts = SolveOpts(tau, None, fail_start, fail_stop, None, async_single_launch)
+    keep = []
+    if fail_mask is not None:
+        m = fail_mask if hasattr(fail_mask, "data_ptr") else np.ascontiguousarray(fail_mask, dtype=np.uint8)
+        keep.append(m)
+        opts.fail_mask = _ptr(m)
+    if history is not None:
+        assert isinstance(history, np.ndarray) and history.dtype == np.float64 and len(history) >= max_global_iters + 1
+        opts.res_history = history.ctypes.data
+    st = _lib.bar_solve_ex(A, _ptr(b), _ptr(x0), _ptr(x), k, max_global_iters, tol, mode, cuda_stream,
+                           ctypes.byref(info), ctypes.byref(opts))
+    if raise_on_error:
+        _check(st)
+    return st, info
+
+
 def bar_sweep(A, b, x, k, nsweeps, mode, cuda_stream=None):
     if isinstance(mode, str):
         mode = MODES[mode]
@@ -172,8 +203,12 @@ class Matrix:
         return bar_matrix_get_info(self.handle).as_dict()
 
     def solve(self, b, x0=None, x=None, k: int = 5, max_global_iters: int = 20000, tol: float = 1e-10,
-              mode="async", stream=None, raise_on_error=True):
-        """Solve in place into ``x`` (allocated like ``b`` if None). Returns (x, info dict)."""
+              mode="async", stream=None, raise_on_error=True, tau=1.0, fail_mask=None, fail_start=0, fail_stop=-1,
+              history=False, async_single_launch=-1):
+        """Solve in place into ``x`` (allocated like ``b`` if None). Returns (x, info dict).
+
+        Options (bar_solve_ex): ``tau`` (N3), ``fail_mask``/``fail_start``/``fail_stop`` (N1),
+        ``history`` (info["history"] = rel_res per global iteration)."""
         if x is None:
             if hasattr(b, "data_ptr"):
                 import torch
@@ -181,10 +216,18 @@ class Matrix:
                 x = torch.empty_like(b)
             else:
                 x = np.empty_like(b)
-        st, info = bar_solve(self.handle, b, x0, x, k, max_global_iters, tol, mode, _stream_handle(stream),
-                             raise_on_error)
+        ext = tau != 1.0 or fail_mask is not None or history or async_single_launch != -1
+        hist = np.full(max_global_iters + 1, np.nan) if history else None
+        if ext:
+            st, info = bar_solve_ex(self.handle, b, x0, x, k, max_global_iters, tol, mode, _stream_handle(stream),
+                                    raise_on_error, tau, fail_mask, fail_start, fail_stop, hist, async_single_launch)
+        else:
+            st, info = bar_solve(self.handle, b, x0, x, k, max_global_iters, tol, mode, _stream_handle(stream),
+                                 raise_on_error)
         d = info.as_dict()
         d["status"] = STATUS.get(st, st)
+        if hist is not None:
+            d["history"] = hist[: d["iters"] + 1]
         return x, d
 
     def sweep(self, b, x, k: int = 5, nsweeps: int = 1, mode="async", stream=None):

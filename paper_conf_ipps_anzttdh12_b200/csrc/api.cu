@@ -167,6 +167,7 @@ void bar_destroy(bar_matrix A) {
     cudaFree(W.stage_b);
     cudaFree(W.stage_x);
     cudaFree(W.partials);
+    cudaFree(W.frozen);
     cudaFree(W.state);
     cudaFreeHost(W.h_state);
     delete A;
@@ -263,8 +264,9 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
     return BAR_OK;
 }
 
-bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x, int32_t k, int64_t max_global_iters,
-                     double tol, bar_mode mode, void *cuda_stream, bar_solve_info *info) {
+bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double *x, int32_t k,
+                        int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream, bar_solve_info *info,
+                        const bar_solve_opts *opts) {
     g_err.clear();
     if (!A || !b || !x) {
         set_error("NULL argument");
@@ -279,6 +281,11 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
         return BAR_ERR_INVALID_ARG;
     }
     if (mode == BAR_MODE_JACOBI) k = 1;
+    const double tau = opts ? opts->tau : 1.0;
+    if (!(tau > 0.0) || !std::isfinite(tau)) {
+        set_error("tau must be a positive finite number");
+        return BAR_ERR_INVALID_ARG;
+    }
     DeviceGuard g(A->device);
     if (!g.ok) return cuda_fail(cudaGetLastError(), "cudaSetDevice");
     cudaStream_t st = (cudaStream_t)cuda_stream;
@@ -289,6 +296,24 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
     bar_status r = ensure_workspace(A);
     if (r != BAR_OK) return r;
     int64_t launches = 0;
+    // N1 failure mask (device copy) and the per-launch window; residual history buffer
+    const uint8_t *d_mask = nullptr;
+    const int64_t f0 = opts ? opts->fail_start : 0, f1 = opts ? opts->fail_stop : -1;
+    if (opts && opts->fail_mask) {
+        if (!W.frozen) BAR_CUDA(cudaMalloc(&W.frozen, (size_t)n));
+        BAR_CUDA(cudaMemcpyAsync(W.frozen, opts->fail_mask, (size_t)n, cudaMemcpyDefault, st));
+        d_mask = W.frozen;
+    }
+    auto mask_at = [&](int64_t m) -> const uint8_t * {
+        return (d_mask && m >= f0 && (f1 < 0 || m < f1)) ? d_mask : nullptr;
+    };
+    double *d_hist = nullptr;
+    struct HistFree {
+        double *&p;
+        ~HistFree() { cudaFree(p); }
+    } hist_free{d_hist};
+    if (opts && opts->res_history) BAR_CUDA(cudaMalloc(&d_hist, sizeof(double) * (size_t)(max_global_iters + 2)));
+    const bool ext_opts = tau != 1.0 || d_mask || d_hist;
 
     // End-to-end path: host vectors are staged through device buffers inside the call.
     const double *db = b;
@@ -331,7 +356,9 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
             const int64_t c = std::min(chunk, max_global_iters - issued);
             for (int64_t i = 0; i < c; ++i) {
                 const int64_t m = issued + i + 1;
-                SweepArgs a{&L, db, (m & 1) ? buf0 : buf1, (m & 1) ? buf1 : buf0, k, W.state, W.partials, nullptr};
+                SweepArgs a{&L, db, (m & 1) ? buf0 : buf1, (m & 1) ? buf1 : buf0, k, W.state, W.partials, d_hist};
+                a.frozen = mask_at(m);
+                a.tau = tau;
                 BAR_CUDA(launch_sweep(a, mode, st));
             }
             launches += c;
@@ -373,6 +400,8 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
         // Fully asynchronous persistent solve (one launch for all global iterations); a stop
         // request raised by the fused estimate is confirmed by an exact residual, else resumed.
         bool multi = use_async_multi(L);
+        if (opts && opts->async_single_launch >= 0) multi = opts->async_single_launch == 1;
+        if (ext_opts) multi = false;
         bool used_multi = false;
         const long long w_end = (long long)max_global_iters * (long long)L.q;
         while (multi && !converged && !bzero && !diverged && max_global_iters > 0) {
@@ -411,7 +440,11 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
         while (!multi && !converged && !bzero && !diverged && H.iter < max_global_iters) {
             const int64_t c = std::min<int64_t>(chunk, max_global_iters - (int64_t)H.iter);
             for (int64_t i = 0; i < c; ++i) {
-                SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+                // global iteration index of this launch (launches after a stop request no-op)
+                const int64_t m = (int64_t)H.iter + i + 1;
+                SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, d_hist};
+                a.frozen = mask_at(m);
+                a.tau = tau;
                 BAR_CUDA(launch_sweep(a, mode, st));
             }
             launches += c;
@@ -445,6 +478,11 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
     if (diverged && iters == 0 && !std::isfinite(rel)) nonfinite = true;
     if (result != x) BAR_CUDA(cudaMemcpyAsync(x, result, bytes, x_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
     BAR_CUDA(cudaStreamSynchronize(st));
+    if (d_hist && iters > 0) {  // the device wrote entry m-1 during global iteration m
+        const int64_t have = std::min<int64_t>(iters, max_global_iters);
+        BAR_CUDA(cudaMemcpy(opts->res_history, d_hist, sizeof(double) * (size_t)have, cudaMemcpyDeviceToHost));
+    }
+    if (d_hist) opts->res_history[iters] = rel;  // the returned iterate, exactly
     if (info) {
         info->iters = iters;
         info->rel_res = rel;
@@ -466,3 +504,9 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
 }
 
 }  // extern "C"
+
+extern "C" bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x, int32_t k,
+                                int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
+                                bar_solve_info *info) {
+    return bar_solve_ex(A, b, x0, x, k, max_global_iters, tol, mode, cuda_stream, info, nullptr);
+}

@@ -72,6 +72,7 @@ struct Workspace {
     double *stage_b = nullptr;  // n: device staging of host b (end-to-end path)
     double *stage_x = nullptr;  // n: device staging of host x0/x
     double *partials = nullptr; // per-block partial sums of squares
+    uint8_t *frozen = nullptr;  // N1 failure mask (device copy, n bytes)
     int64_t npartials = 0;
     DevState *state = nullptr;  // device
     DevState *h_state = nullptr;// pinned host mirror
@@ -135,6 +136,8 @@ struct SweepArgs {
     double *partials;
     double *hist;  // nullable device array: hist[m-1] = rel_res(x^(m-1)) (sync modes)
     double *dist_out = nullptr;  // multi-GPU: receives this rank's [sum r^2, sum b^2]
+    const uint8_t *frozen = nullptr;  // N1: rows that do not update in this launch (nullable)
+    double tau = 1.0;                 // N3: relaxation weight, B = I - tau D^-1 A
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);

@@ -46,7 +46,15 @@ struct KP {
     long long w_end;  // async persistent: claims [0, w_end) = global iterations [0, w_end / q)
     int fresh_xj;     // async persistent with q < 4 * grid: read x_J when a subdomain starts
     double *dist_out; // multi-GPU: [sum r^2, sum b^2] of this rank (no stopping decision here)
+    const uint8_t *frozen;  // N1 failure injection: rows that keep their value (nullable)
+    double tau;             // N3: every update scaled, x + tau (v - x)
 };
+
+// N1/N3 update rule (R17/R18): x_old -> v unless the row is frozen; tau-scaled.
+__device__ __forceinline__ double ext_update(double xold, double v, bool frozen, double tau) {
+    if (frozen) return xold;
+    return tau == 1.0 ? v : xold + tau * (v - xold);
+}
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
 
@@ -259,7 +267,7 @@ __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
                                          sv + loc, sc + loc, sstride);
             rr += res * res;
             ss[loc] = s;
-            y1[loc] = y0[loc] + dinv * res;
+            y1[loc] = ext_update(y0[loc], y0[loc] + dinv * res, p.frozen && p.frozen[TS + loc], p.tau);
         }
     }
     __syncthreads();
@@ -279,14 +287,14 @@ __global__ void __launch_bounds__(1024, 1) k_block(KP p) {
                     const int32_t *lc = sc + loc;
 #pragma unroll 4
                     for (int e = 1; e < wl; ++e) acc -= lv[e * sstride] * yi[lc[e * sstride]];
-                    yo[loc] = lv[0] * acc;
+                    yo[loc] = ext_update(yi[loc], lv[0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
                 } else {
                     const int64_t base = p.sptr[sl0 + j] + lane + (int64_t)(w >> 16) * kSlice;
                     const double *vl = p.val + base;
                     const int32_t *cl = p.col + base;
 #pragma unroll 4
                     for (int e = 1; e < wl; ++e) acc -= __ldg(vl + e * kSlice) * yi[__ldg(cl + e * kSlice)];
-                    yo[loc] = acc / __ldg(vl);
+                    yo[loc] = ext_update(yi[loc], acc / __ldg(vl), p.frozen && p.frozen[TS + loc], p.tau);
                 }
             }
         }
@@ -706,7 +714,7 @@ __device__ __forceinline__ void iteration_publish(const KP &p, long long m, unsi
 // When the last subdomain of iteration m finishes, its block turns the accumulated residual
 // estimate into rel_res_m and raises the stop flag if it meets tol; blocks stop claiming.
 // Per-launch staged sweep (one global iteration per launch).
-template <bool ASYNC, int WLR>
+template <bool ASYNC, int WLR, bool EXT = false>
 __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
@@ -800,6 +808,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
         double s = 0.0;
         const int loc = warp * kSlice + lane;
         const bool ok = warp < nsl && loc < nrows;
+        const bool fz = EXT && ok && p.frozen && p.frozen[TS + loc];  // N1
 #pragma unroll
         for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
 #pragma unroll
@@ -837,7 +846,8 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
             for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
             lv[0] = 1.0 / lv[0];
             rr += acc * acc;
-            y1[loc] = y0[loc] + lv[0] * acc;
+            if (EXT) y1[loc] = ext_update(y0[loc], y0[loc] + lv[0] * acc, fz, p.tau);
+            else y1[loc] = y0[loc] + lv[0] * acc;
         }
         __syncthreads();
         // a4: sweeps 2..k, direct form, off-block part frozen
@@ -848,7 +858,8 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
                 double acc = s;
 #pragma unroll
                 for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
-                yo[loc] = lv[0] * acc;
+                if (EXT) yo[loc] = ext_update(yi[loc], lv[0] * acc, fz, p.tau);
+                else yo[loc] = lv[0] * acc;
             }
             __syncthreads();
         }
@@ -1151,7 +1162,10 @@ __global__ void __launch_bounds__(256, 4) k_rowwise_tma(KP p) {
                 }
             }
             rr += acc * acc;
-            if (!RESIDUAL_ONLY) p.x_out[row] = __ldg(p.x_in + row) + dinv * acc;
+            if (!RESIDUAL_ONLY) {
+                const double xi = __ldg(p.x_in + row);
+                p.x_out[row] = ext_update(xi, xi + dinv * acc, p.frozen && p.frozen[row], p.tau);
+            }
         }
         __syncwarp();
     }
@@ -1180,7 +1194,10 @@ __global__ void __launch_bounds__(256) k_rowwise(KP p) {
             row_pass<false, false, false>(p.val + base, p.col + base, wo, wo + wl, p.x_in, p.x_in + TS, bi, s, res,
                                           dinv, nullptr, nullptr, 0);
             rr = res * res;
-            if (!RESIDUAL_ONLY) p.x_out[row] = __ldg(p.x_in + row) + dinv * res;
+            if (!RESIDUAL_ONLY) {
+                const double xi = __ldg(p.x_in + row);
+                p.x_out[row] = ext_update(xi, xi + dinv * res, p.frozen && p.frozen[row], p.tau);
+            }
         }
     }
     reduce_finalize<RESIDUAL_ONLY ? kResidual : kSync>(rr, bb, p);
@@ -1216,6 +1233,8 @@ KP make_kp(const Layout &L) {
     p.R = L.R;
     p.spb = L.spb;
     p.nslices = L.nslices;
+    p.tau = 1.0;
+    p.frozen = nullptr;
     return p;
 }
 
@@ -1291,22 +1310,26 @@ cudaError_t launch_pers_t(const KP &p, const Layout &L, size_t smem, cudaStream_
 
 template <bool ASYNC, int WLR, bool MULTI>
 cudaError_t launch_stage_m(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
-    static size_t attr = 0;
-    static size_t c_smem = 0;
-    static int c_threads = 0, per_sm = 0;
-    auto kfn = MULTI ? k_block_stage_m<true, WLR, true> : k_block_stage<ASYNC, WLR>;
-    if (smem > attr) {
+    const bool ext = !MULTI && (p.frozen != nullptr || p.tau != 1.0);  // N1 / N3 requested
+    auto kfn = MULTI ? k_block_stage_m<true, WLR, true>
+                     : (ext ? k_block_stage<ASYNC, WLR, true> : k_block_stage<ASYNC, WLR, false>);
+    static size_t attr[2] = {0, 0};
+    static size_t c_smem[2] = {0, 0};
+    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
+    const int v = ext ? 1 : 0;
+    if (smem > attr[v]) {
         cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr = smem;
+        attr[v] = smem;
     }
-    if (c_smem != smem || c_threads != L.spb * kSlice) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, L.spb * kSlice, smem) != cudaSuccess ||
-            per_sm < 1)
-            per_sm = 1;
-        c_smem = smem;
-        c_threads = L.spb * kSlice;
+    if (c_smem[v] != smem || c_threads[v] != L.spb * kSlice) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, L.spb * kSlice, smem) != cudaSuccess ||
+            occ[v] < 1)
+            occ[v] = 1;
+        c_smem[v] = smem;
+        c_threads[v] = L.spb * kSlice;
     }
+    const int per_sm = occ[v];
     int64_t g = (int64_t)per_sm * L.sms;
     if (g > L.q) g = L.q;
     KP pp = p;
@@ -1351,17 +1374,18 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         return launch_stage_t<ASYNC, 16>(p, L, stage_smem, st);  // <= 256 threads per block
     }
     if (p.w_end > 0) return cudaErrorNotSupported;  // no persistent multi-iteration kernel here
-    if ((kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
+    const bool ext = p.frozen != nullptr || p.tau != 1.0;  // N1/N3: only k_block_stage and k_block
+    if (!ext && (kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
         if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
         if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
         return launch_pers_t<ASYNC, 8>(p, L, pers_smem, st);
     }
-    if ((kind == 't' || kind == 'n') && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
+    if (!ext && (kind == 't' || kind == 'n') && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
         if (L.max_wl <= 4) return launch_reg_tma_t<ASYNC, 4>(p, L, tma_smem, st);
         if (L.max_wl <= 6) return launch_reg_tma_t<ASYNC, 6>(p, L, tma_smem, st);
         return launch_reg_tma_t<ASYNC, 8>(p, L, tma_smem, st);
     }
-    if (kind != 's' && L.spb <= 32 && L.max_wl <= 8) return launch_reg_w<ASYNC, 1>(p, L, st);
+    if (!ext && kind != 's' && L.spb <= 32 && L.max_wl <= 8) return launch_reg_w<ASYNC, 1>(p, L, st);
     const size_t row_bytes = 3 * (size_t)L.R * sizeof(double);  // y0, y1, s
     const size_t stage_bytes = (size_t)L.max_wl * L.spb * kSlice * (sizeof(double) + sizeof(int32_t));
     const bool stage = row_bytes + stage_bytes <= kSmemBudget;
@@ -1436,6 +1460,8 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.partials = a.partials;
     p.hist = a.hist;
     p.dist_out = a.dist_out;
+    p.frozen = a.frozen;
+    p.tau = a.tau;
     p.w_end = 0;
     if (mode == BAR_MODE_JACOBI) return launch_rowwise<false>(p, *a.L, st);
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
@@ -1452,6 +1478,8 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
     p.partials = a.partials;
     p.hist = a.hist;
     p.dist_out = a.dist_out;
+    p.frozen = a.frozen;
+    p.tau = a.tau;
     p.w_end = w_end > 0 ? w_end : 1;
     return launch_block<true>(p, *a.L, st);
 }
