@@ -1,0 +1,55 @@
+"""N4: cost of the local iterations on B200 — time per global iteration of
+async-(k) for k = 1..9 (CUDA-event slope of back-to-back sweep launches, as bench.py), against
+the paper's Table 4 (fv3 on a C2070: +19% at k=5, +39% at k=9 over async-(1); the
+text claims "<5%" for k=2 and "<35%" for k=9).
+
+    python tools/local_iters.py --workload c4 > profiles/r01_n4_c4.txt
+"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="c4")
+    ap.add_argument("--R", type=int, default=None)
+    ap.add_argument("--mode", default="async")
+    a = ap.parse_args()
+    import torch
+
+    import bench
+    from paper_conf_ipps_anzttdh12_b200 import bar
+
+    R = a.R or bench.WORKLOADS[a.workload][2]
+    A = bench.make_matrix(a.workload)
+    M = bar.Matrix.from_csr(A, R)
+    nb = M.info()["model_bytes_per_iter"]
+    b = torch.ones(A.n, dtype=torch.float64, device="cuda")
+    x = torch.zeros_like(b)
+    st = torch.cuda.current_stream()
+
+    def timed(k, nsw):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        M.sweep(b, x, k=k, nsweeps=nsw, mode=a.mode)
+        e1.record(st)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1)
+
+    print(f"# N4: {a.mode}-(k), {A.name}, R={R}; ms per global iteration (slope of 8 vs 40 launches)")
+    print(f"# paper Table 4 (fv3, C2070): async-(5) +19%, async-(9) +39% per global iteration over async-(1)")
+    print(f"{'k':>3} {'ms/iter':>10} {'vs k=1':>8} {'GB/s':>8}")
+    base = None
+    for k in range(1, 10):
+        timed(k, 4)
+        t = (min(timed(k, 40) for _ in range(3)) - min(timed(k, 8) for _ in range(3))) / 32
+        base = base or t
+        print(f"{k:3d} {t:10.4f} {100 * (t / base - 1):+7.1f}% {nb / (t * 1e-3) / 1e9:8.1f}")
+
+
+if __name__ == "__main__":
+    main()
