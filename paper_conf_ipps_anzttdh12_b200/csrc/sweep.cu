@@ -713,6 +713,193 @@ __device__ __forceinline__ void iteration_publish(const KP &p, long long m, unsi
 // while another still sweeps a neighbour in iteration m (eq. 3's bounded shift).
 // When the last subdomain of iteration m finishes, its block turns the accumulated residual
 // estimate into rel_res_m and raises the stop flag if it meets tol; blocks stop claiming.
+// ---------------------------------------------------------------------------------------------
+// k_block_pipe: the per-launch staged sweep with a DEEPER pipeline. The matrix slab of a
+// subdomain is only needed until its local entries are in registers (end of phase 1), so the
+// slab buffer is refilled with subdomain l+2 right then, while l's k-1 local sweeps and l+1's
+// whole sweep still run: the HBM stream stays busy through the sweeps (N4: with one subdomain
+// of look-ahead the local sweeps were not hidden, 2.2 -> 2.9 ms/iteration on C5 for k 1 -> 5).
+// Buffers: two slab buffers (values, columns) and three small row slots [b -> y1 | x -> y0 |
+// slice metadata] (b_i is read once, then its slot holds y1_i).
+struct PipeGeom {
+    uint32_t vcap, vc_bytes, o_x, o_sptr, o_sw, bx_bytes, o_bx;
+};
+
+__host__ __device__ __forceinline__ PipeGeom pipe_geom(int R, int spb, int wmax) {
+    PipeGeom g;
+    g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
+    g.vc_bytes = (g.vcap * 12 + 127) & ~127u;  // values (8 B) then columns (4 B)
+    g.o_x = (uint32_t)R * 8;
+    g.o_sptr = g.o_x + (uint32_t)R * 8;
+    g.o_sw = g.o_sptr + (uint32_t)spb * 8;
+    g.bx_bytes = (g.o_sw + (uint32_t)spb * 4 + 127) & ~127u;
+    g.o_bx = 2 * g.vc_bytes;
+    return g;
+}
+
+template <bool ASYNC, int WLR, bool EXT = false>
+__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bars[3];
+    __shared__ long long slot_l[3];
+    const int R = p.R, spb = p.spb;
+    const PipeGeom g = pipe_geom(R, spb, p.wmax);
+    const int64_t q = (p.n + R - 1) / R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    // ---- thread 0: claims (four deep) and stage issue. Only two claims stay in registers
+    // across iterations; the next stage's range bounds arrive in shared memory by cp.async, so
+    // no register holds an in-flight load (register pressure = spills on this 64-reg kernel).
+    __shared__ __align__(16) int64_t bnd[2];
+    auto claim = [&](long long j) -> long long {
+        if (ASYNC) return (long long)atomicAdd(&p.state->work, 1ull);
+        return (long long)blockIdx.x + j * (long long)gridDim.x;
+    };
+    auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
+    auto fetch_bounds = [&](long long l) {  // async: E0, E1 of subdomain l -> bnd[]
+        if (l >= q) return;
+        const unsigned s0 = smem_u32(&bnd[0]), s1 = smem_u32(&bnd[1]);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s0), "l"(p.sptr + l * spb) : "memory");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s1), "l"(p.sptr + l * spb + nsl_of(l))
+                     : "memory");
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    // subdomain of iteration j: slab buffer j % 2, row slot and barrier j % 3
+    auto issue = [&](long long l, int j, int64_t E0, int64_t E1) {
+        const int vs = j & 1, bs = j % 3;
+        slot_l[bs] = l;
+        if (l >= q) return;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        const uint32_t trows = (uint32_t)nrows & ~1u;
+        const uint32_t nb_sptr = ((uint32_t)nsl * 8 + 15) & ~15u, nb_sw = ((uint32_t)nsl * 4 + 15) & ~15u;
+        const uint32_t ne = (uint32_t)(E1 - E0);
+        unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
+        unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&bars[bs], ne * 12 + trows * 16 + nb_sptr + nb_sw);
+        bulk_g2s(V, p.val + E0, ne * 8, &bars[bs]);
+        bulk_g2s(V + (size_t)g.vcap * 8, p.col + E0, ne * 4, &bars[bs]);
+        if (trows) {
+            bulk_g2s(B, p.b + TS, trows * 8, &bars[bs]);
+            bulk_g2s(B + g.o_x, p.x_in + TS, trows * 8, &bars[bs]);
+        }
+        bulk_g2s(B + g.o_sptr, p.sptr + l * spb, nb_sptr, &bars[bs]);
+        bulk_g2s(B + g.o_sw, p.sw + l * spb, nb_sw, &bars[bs]);
+    };
+    long long l2 = 0, l3 = 0;  // claims: next to issue (bounds in flight to bnd[]), the one after
+    if (threadIdx.x == 0) {
+        for (int j = 0; j < 3; ++j) mbar_init(&bars[j], 1);
+        fence_mbar_init();
+        const long long l0 = claim(0);
+        if (l0 < q) issue(l0, 0, p.sptr[l0 * spb], p.sptr[l0 * spb + nsl_of(l0)]);
+        else slot_l[0] = q;
+        const long long l1 = l0 < q ? claim(1) : q;
+        if (l1 < q) issue(l1, 1, p.sptr[l1 * spb], p.sptr[l1 * spb + nsl_of(l1)]);
+        else slot_l[1] = q;
+        l2 = l1 < q ? claim(2) : q;
+        fetch_bounds(l2);
+        l3 = l2 < q ? claim(3) : q;
+    }
+    __syncthreads();
+
+    constexpr int NP = WLR / 2;
+    double rr = 0.0, bb = 0.0;
+    for (int i = 0;; ++i) {
+        const int vs = i & 1, bs = i % 3;
+        const long long l = slot_l[bs];
+        if (l >= q) break;
+        unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
+        unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        double *y1 = reinterpret_cast<double *>(B);  // b, then y1
+        double *y0 = reinterpret_cast<double *>(B + g.o_x);
+        mbar_wait(&bars[bs], (i / 3) & 1);
+        if (nrows & 1) {  // odd tail of the last subdomain: not bulk-copied
+            if (threadIdx.x == 0) y0[nrows - 1] = ldx<ASYNC>(p.x_in + TS + nrows - 1);
+            __syncthreads();
+        }
+        double lv[WLR];
+        uint32_t lc[NP];
+        double s = 0.0;
+        const int loc = warp * kSlice + lane;
+        const bool ok = warp < nsl && loc < nrows;
+        const bool fz = EXT && ok && p.frozen && p.frozen[TS + loc];  // N1
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+        for (int e = 0; e < NP; ++e) lc[e] = 0;
+        if (ok) {
+            const int64_t *ssp = reinterpret_cast<const int64_t *>(B + g.o_sptr);
+            const int sw = reinterpret_cast<const int32_t *>(B + g.o_sw)[warp];
+            const int wl = sw & 0xffff, wo = sw >> 16;
+            const int64_t off = ssp[warp] - ssp[0] + lane;
+            const double *sv = reinterpret_cast<const double *>(V) + off;
+            const int32_t *sc = reinterpret_cast<const int32_t *>(V + (size_t)g.vcap * 8) + off;
+            const double bi = loc < (nrows & ~1) ? y1[loc] : p.b[TS + loc];
+            bb += bi * bi;
+            double acc = bi;
+            // a3: off-block part, x as it stands (gathers batched)
+            for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+            }
+            s = acc;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[e] = sv[(wo + e) * kSlice];
+                    lc[e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                }
+            }
+            // first local sweep; its correction numerator is the residual (a5)
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[0] = 1.0 / lv[0];
+            rr += acc * acc;
+            // y1 takes b's slot: only this thread ever read b[loc]
+            if (EXT) y1[loc] = ext_update(y0[loc], y0[loc] + lv[0] * acc, fz, p.tau);
+            else y1[loc] = y0[loc] + lv[0] * acc;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {  // the slab buffer is free: stream subdomain l_{i+2} into it
+            asm volatile("cp.async.wait_all;" ::: "memory");
+            if (l2 < q) issue(l2, i + 2, bnd[0], bnd[1]);
+            else slot_l[(i + 2) % 3] = q;
+            l2 = l3;
+            fetch_bounds(l2);
+            l3 = l2 < q ? claim(i + 4) : q;
+        }
+        // a4: sweeps 2..k, direct form, off-block part frozen
+        for (int t = 1; t < p.k; ++t) {
+            const double *yi = (t & 1) ? y1 : y0;
+            double *yo = (t & 1) ? y0 : y1;
+            if (ok) {
+                double acc = s;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                if (EXT) yo[loc] = ext_update(yi[loc], lv[0] * acc, fz, p.tau);
+                else yo[loc] = lv[0] * acc;
+            }
+            __syncthreads();
+        }
+        // a6: write back
+        const double *yk = (p.k & 1) ? y1 : y0;
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
+        __syncthreads();
+    }
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
 // Per-launch staged sweep (one global iteration per launch).
 template <bool ASYNC, int WLR, bool EXT = false>
 __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
@@ -1341,9 +1528,44 @@ cudaError_t launch_stage_m(const KP &p, const Layout &L, size_t smem, cudaStream
 }
 
 template <bool ASYNC, int WLR>
+cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    const bool ext = p.frozen != nullptr || p.tau != 1.0;
+    auto kfn = ext ? k_block_pipe<ASYNC, WLR, true> : k_block_pipe<ASYNC, WLR, false>;
+    static size_t attr[2] = {0, 0};
+    static size_t c_smem[2] = {0, 0};
+    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
+    const int v = ext ? 1 : 0;
+    if (smem > attr[v]) {
+        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr[v] = smem;
+    }
+    if (c_smem[v] != smem || c_threads[v] != L.spb * kSlice) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, L.spb * kSlice, smem) != cudaSuccess ||
+            occ[v] < 1)
+            occ[v] = 1;
+        c_smem[v] = smem;
+        c_threads[v] = L.spb * kSlice;
+    }
+    int64_t g = (int64_t)occ[v] * L.sms;
+    if (g > L.q) g = L.q;
+    kfn<<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <bool ASYNC, int WLR>
 cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     if (ASYNC && p.w_end > 0) return launch_stage_m<true, WLR, true>(p, L, smem, st);
     return launch_stage_m<ASYNC, WLR, false>(p, L, smem, st);
+}
+
+// Whether the staged (TMA) block kernels apply to this layout and these vectors.
+bool staged_ok(const KP &p, const Layout &L) {
+    const bool aligned = ((uintptr_t)p.b % 16 == 0) && ((uintptr_t)p.x_in % 16 == 0);
+    const bool geom_ok = L.spb % 4 == 0 && L.R % 2 == 0 &&
+                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
+    const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
+    return aligned && geom_ok && stage_smem <= kSmemMax;
 }
 
 // Kernel choice for one block-sweep launch (async / sync-block):
@@ -1367,6 +1589,19 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // bulk-copy sources must be 16-byte aligned: b/x at l*R rows (R even), ptr/sw at l*spb
     const bool geom_ok = L.spb % 4 == 0 && L.R % 2 == 0 &&
                          ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
+    const PipeGeom pg = pipe_geom(L.R, L.spb, L.max_w);
+    const size_t pipe_smem = 2 * (size_t)pg.vc_bytes + 3 * (size_t)pg.bx_bytes;
+    // measured on B200 (round 1, tools/local_iters.py, sweep_R.py): the two-ahead pipeline wins
+    // for sync-block (C5: 2.96 vs 3.52 ms/iteration) and loses for async (3.40 vs 3.05), whose
+    // issue path (work-queue claim) sits on the critical warp; BAR_PIPE=0/1 overrides
+    const char *pe = getenv("BAR_PIPE");
+    const bool pipe_on = pe ? pe[0] == '1' : (!ASYNC && p.k >= 3);
+    if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
+        if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);
+        if (L.max_wl <= 6) return launch_pipe_t<ASYNC, 6>(p, L, pipe_smem, st);
+        if (L.max_wl <= 8) return launch_pipe_t<ASYNC, 8>(p, L, pipe_smem, st);
+        return launch_pipe_t<ASYNC, 16>(p, L, pipe_smem, st);
+    }
     if (kind == 't' && geom_ok && aligned && stage_smem <= kSmemMax) {
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
         if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
@@ -1463,7 +1698,16 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.frozen = a.frozen;
     p.tau = a.tau;
     p.w_end = 0;
-    if (mode == BAR_MODE_JACOBI) return launch_rowwise<false>(p, *a.L, st);
+    if (mode == BAR_MODE_JACOBI) {
+        // Jacobi (eq. 2) is sync-block-(1) for any R, with the same per-row arithmetic
+        // (off-block entries, then local ones, diagonal included): use the staged stream
+        const char *jv = getenv("BAR_JACOBI_ROWWISE");
+        if (!(jv && jv[0] == '1') && staged_ok(p, *a.L)) {
+            p.k = 1;
+            return launch_block<false>(p, *a.L, st);
+        }
+        return launch_rowwise<false>(p, *a.L, st);
+    }
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
     return launch_block<false>(p, *a.L, st);
 }

@@ -1,6 +1,3 @@
-timeout 900 python tools/nondeterminism.py --workload c1 --runs 200 > gpurun_out/r01_n2_c1.txt 2>&1
-timeout 900 python tools/nondeterminism.py --workload c2 --runs 100 > gpurun_out/r01_n2_c2.txt 2>&1
-timeout 900 python tools/nondeterminism.py --workload c1 --runs 100 --single-launch 0 > gpurun_out/r01_n2_c1_perlaunch.txt 2>&1
-timeout 600 python tools/local_iters.py --workload c4 > gpurun_out/r01_n4_c4.txt 2>&1
-timeout 600 python tools/local_iters.py --workload c5 > gpurun_out/r01_n4_c5.txt 2>&1
-timeout 600 python tools/local_iters.py --workload c2 --R 128 > gpurun_out/r01_n4_c2.txt 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+timeout 600 python tools/sweep_R.py --workload c5 --R 1024 --modes async,sync-block,jacobi 2>&1 | grep '^{'
+timeout 600 python tools/sweep_R.py --workload c4 --R 128 --modes async,sync-block,jacobi 2>&1 | grep '^{'
