@@ -258,3 +258,26 @@ def test_siam_constant_async(bar, golden):
     for mode in ("async", "sync-block"):
         x, info = _solve(bar, A, b, 128, 5, mode, 20000, 1e-13)
         assert info["converged"] and abs(x[0] - ref) < 1e-11
+
+
+# ------------------------------------------------------------------ every kernel generation
+@pytest.mark.parametrize("env", [{"BAR_KERNEL": "s"}, {"BAR_KERNEL": "r"}, {"BAR_KERNEL": "n"}, {"BAR_KERNEL": "p"},
+                                 {"BAR_PIPE": "1"}, {"BAR_PIPE": "0"}, {"BAR_JACOBI_ROWWISE": "1"},
+                                 {"BAR_ASYNC_MULTI": "1"}, {"BAR_ASYNC_MULTI": "0"}])
+@pytest.mark.parametrize("name,R", [("fv1", 128), ("s7_m12", 288), ("tref2000", 128)])
+def test_forced_kernel_paths(bar, monkeypatch, env, name, R):
+    """Each kernel the dispatcher can choose (fallbacks included) gives the oracle's iterates in
+    the sync modes and converges in async (the environment variables only steer dispatch)."""
+    for k_, v in env.items():
+        monkeypatch.setenv(k_, v)
+    A = MATS[name]()
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(2).uniform(-1, 1, A.n)
+    for mode, k in (("sync-block", 5), ("jacobi", 1)):
+        ref = x0
+        for _ in range(3):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x, _ = _solve(bar, A, b, R, k, mode, 3, 0.0, x0)
+        _close(x, ref)
+    x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10)
+    assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
