@@ -48,6 +48,7 @@ struct KP {
     double *dist_out; // multi-GPU: [sum r^2, sum b^2] of this rank (no stopping decision here)
     const uint8_t *frozen;  // N1 failure injection: rows that keep their value (nullable)
     double tau;             // N3: every update scaled, x + tau (v - x)
+    int static_claims;      // async: round-robin subdomain order instead of the work queue
 };
 
 // N1/N3 update rule (R17/R18): x_old -> v unless the row is frozen; tau-scaled.
@@ -753,7 +754,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     // no register holds an in-flight load (register pressure = spills on this 64-reg kernel).
     __shared__ __align__(16) int64_t bnd[2];
     auto claim = [&](long long j) -> long long {
-        if (ASYNC) return (long long)atomicAdd(&p.state->work, 1ull);
+        if (ASYNC && !p.static_claims) return (long long)atomicAdd(&p.state->work, 1ull);
         return (long long)blockIdx.x + j * (long long)gridDim.x;
     };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
@@ -917,7 +918,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
     // ---- thread 0: subdomain claims and stage issue ----
     long long claims = 0;
     auto claim = [&]() -> long long {
-        if (ASYNC) return (long long)atomicAdd(&p.state->work, 1ull);
+        if (ASYNC && !p.static_claims) return (long long)atomicAdd(&p.state->work, 1ull);
         return (long long)blockIdx.x + (claims++) * G;
     };
     auto issue = [&](long long l, int st, int64_t E0, int64_t E1) {
@@ -1582,6 +1583,12 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const char kind = kv ? kv[0] : 't';
     p.wlmax = L.max_wl;
     p.wmax = L.max_w;
+    // async subdomain order of the per-launch kernels: static round robin (block c sweeps c,
+    // c + G, ...) by default. Measured on B200 (round 1): the device work queue's atomic claims
+    // cost 0.6 ms/iteration on some boxes (C5 k=5: 3.57 vs 2.91 ms) and converged no faster
+    // (59 vs 57 global iterations). BAR_ASYNC_STATIC=0 selects the queue.
+    const char *sc = getenv("BAR_ASYNC_STATIC");
+    p.static_claims = !(sc && sc[0] == '0');
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
