@@ -65,7 +65,11 @@ struct Layout {
     int32_t *col = nullptr;     // [entries]
     int64_t *sptr = nullptr;    // [nslices+1] entry offset of each slice
     int32_t *sw = nullptr;      // [nslices]   wl | (wo << 16)
+    // [q][kGhostRanges] (first column, count) of x ranges holding most of subdomain l's
+    // off-block columns (count 0 = unused): bulk L2 prefetch targets for the a3 gathers
+    int32_t *gr = nullptr;
 };
+constexpr int kGhostRanges = 4;
 
 struct Workspace {
     double *xbuf = nullptr;     // n: second iterate buffer (sync modes)

@@ -138,6 +138,67 @@ __global__ void k_fill(int64_t nslices, int64_t n, int32_t R, int32_t spb, const
     }
 }
 
+// Per subdomain (one block): the off-block columns of a row i are grouped by their offset
+// d = c - i; the (at most kGhostRanges) most frequent offsets, each used by at least a quarter of
+// the subdomain's rows, give the x ranges [TS + d, TE + d) (clipped to the column range and to
+// outside the subdomain itself) that the sweep kernels prefetch into L2 two subdomains ahead of
+// the gathers that read them (a3): on stencils that is every off-block column; irregular
+// matrices simply get fewer or no ranges. A locality hint only — no result depends on it.
+constexpr int kOffSlots = 64;
+__global__ void k_ghost_ranges(int64_t n, int32_t R, int64_t col_lo, int64_t col_hi,
+                               const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                               int32_t *__restrict__ gr) {
+    __shared__ unsigned long long key[kOffSlots];
+    __shared__ int cnt[kOffSlots];
+    const unsigned long long kEmpty = ~0ull;
+    for (int t = threadIdx.x; t < kOffSlots; t += blockDim.x) {
+        key[t] = kEmpty;
+        cnt[t] = 0;
+    }
+    __syncthreads();
+    const int64_t l = blockIdx.x;
+    const int64_t TS = l * (int64_t)R, TE = min(TS + (int64_t)R, n);
+    for (int64_t i = TS + threadIdx.x; i < TE; i += blockDim.x) {
+        for (int32_t p = rowptr[i]; p < rowptr[i + 1]; ++p) {
+            const int64_t c = col[p];
+            if (c >= TS && c < TE) continue;
+            const unsigned long long k = (unsigned long long)(c - i);
+            int h = (int)((k * 0x9E3779B97F4A7C15ull) >> 58);  // 6 bits
+            for (int probe = 0; probe < kOffSlots; ++probe, h = (h + 1) & (kOffSlots - 1)) {
+                unsigned long long old = atomicCAS(&key[h], kEmpty, k);
+                if (old == kEmpty || old == k) {
+                    atomicAdd(&cnt[h], 1);
+                    break;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x != 0) return;
+    const int nrows = (int)(TE - TS);
+    int out = 0;
+    bool used[kOffSlots];
+    for (int t = 0; t < kOffSlots; ++t) used[t] = false;
+    for (; out < kGhostRanges; ++out) {
+        int best = -1;
+        for (int t = 0; t < kOffSlots; ++t)
+            if (!used[t] && key[t] != kEmpty && (best < 0 || cnt[t] > cnt[best])) best = t;
+        if (best < 0 || 4 * cnt[best] < nrows) break;
+        used[best] = true;
+        const int64_t d = (int64_t)key[best];
+        int64_t lo = max(TS + d, col_lo), hi = min(TE + d, col_hi);
+        if (lo < TS && hi > TS) hi = TS;  // the subdomain's own x_J is staged anyway
+        if (lo < TE && hi > TE) lo = TE;
+        if (hi <= lo) { --out; continue; }
+        gr[2 * (l * kGhostRanges + out)] = (int32_t)lo;
+        gr[2 * (l * kGhostRanges + out) + 1] = (int32_t)(hi - lo);
+    }
+    for (; out < kGhostRanges; ++out) {
+        gr[2 * (l * kGhostRanges + out)] = 0;
+        gr[2 * (l * kGhostRanges + out) + 1] = 0;
+    }
+}
+
 template <class T>
 cudaError_t dmalloc(T **p, size_t count) {
     return cudaMalloc((void **)p, sizeof(T) * (count ? count : 1));
@@ -154,6 +215,8 @@ void free_layout(Layout &L) {
     L.col = nullptr;
     L.sptr = nullptr;
     L.sw = nullptr;
+    cudaFree(L.gr);
+    L.gr = nullptr;
 }
 
 static bar_status alloc_fail(cudaError_t e, const char *what) {
@@ -279,6 +342,9 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     BAR_CK(cudaMemsetAsync(L.col + L.entries, 0, 4 * sizeof(int32_t), st));
     k_fill<<<(unsigned)((nsl * kSlice + TB - 1) / TB), TB, 0, st>>>(nsl, n, R, L.spb, d_rowptr, d_col, d_val, L.sptr,
                                                                    L.sw, L.val, L.col);
+    BAR_CK(cudaGetLastError());
+    BAR_ALLOC(dmalloc(&L.gr, (size_t)L.q * kGhostRanges * 2));
+    k_ghost_ranges<<<(unsigned)L.q, 256, 0, st>>>(n, R, col_lo, col_hi, d_rowptr, d_col, L.gr);
     BAR_CK(cudaGetLastError());
     BAR_CK(cudaStreamSynchronize(st));
 

@@ -49,7 +49,19 @@ struct KP {
     const uint8_t *frozen;  // N1 failure injection: rows that keep their value (nullable)
     double tau;             // N3: every update scaled, x + tau (v - x)
     int static_claims;      // async: round-robin subdomain order instead of the work queue
+    const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
 };
+
+// Thread 0: start copying subdomain l's ghost-range entry (kGhostRanges pairs, 32 B) into
+// shared memory with cp.async (completion: cp.async.wait_all before reading it).
+__device__ __forceinline__ void fetch_ghost_entry(const KP &p, long long l, int64_t q, int32_t *dst) {
+    static_assert(kGhostRanges * 2 * sizeof(int32_t) == 32, "two 16-byte cp.async");
+    if (l >= q || !p.gr) return;
+    const int32_t *src = p.gr + 2 * (int64_t)l * kGhostRanges;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst + 4)), "l"(src + 4) : "memory");
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
 
 // N1/N3 update rule (R17/R18): x_old -> v unless the row is frozen; tau-scaled.
 __device__ __forceinline__ double ext_update(double xold, double v, bool frozen, double tau) {
@@ -738,71 +750,100 @@ __host__ __device__ __forceinline__ PipeGeom pipe_geom(int R, int spb, int wmax)
     return g;
 }
 
+// Issue path. Subdomains are claimed statically (block c sweeps l_j = c + j G, G = grid), so
+// every thread knows l_j without communication. Issuing a stage was a ~300-instruction dependent
+// chain on one thread (64-bit address arithmetic and uniform-register moves around six bulk
+// copies) that every other warp waited for at the next sweep barrier — about a fifth of the
+// launch (ncu source-level stall sampling, profiles/). It is now split over four warps, each
+// issuing its share right after the barrier that frees the slab buffer:
+//   warp 0  mbarrier arrive.expect_tx (before that barrier, off the critical path) + values
+//   warp 1  columns + L2 prefetch of the subdomain's ghost x ranges (its a3 gathers)
+//   warp 2  b_J and x_J
+//   warp 3  slice metadata + cp.async of the bounds/ghost ranges of l_{i+4} into a 4-slot ring
+// The arrive.expect_tx of l_{i+2} is posted before the barrier that precedes every copy of
+// l_{i+2}, so no copy completes bytes before its phase expects them.
 template <bool ASYNC, int WLR, bool EXT = false>
 __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[3];
-    __shared__ long long slot_l[3];
+    __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
+    __shared__ __align__(16) int32_t gsm[4][2 * kGhostRanges];  // [j % 4]: ghost ranges of l_j
     const int R = p.R, spb = p.spb;
     const PipeGeom g = pipe_geom(R, spb, p.wmax);
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-
-    // ---- thread 0: claims (four deep) and stage issue. Only two claims stay in registers
-    // across iterations; the next stage's range bounds arrive in shared memory by cp.async, so
-    // no register holds an in-flight load (register pressure = spills on this 64-reg kernel).
-    __shared__ __align__(16) int64_t bnd[2];
-    auto claim = [&](long long j) -> long long {
-        if (ASYNC && !p.static_claims) return (long long)atomicAdd(&p.state->work, 1ull);
-        return (long long)blockIdx.x + j * (long long)gridDim.x;
-    };
+    const long long G = gridDim.x;
+    auto lof = [&](long long j) { return (long long)blockIdx.x + j * G; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
-    auto fetch_bounds = [&](long long l) {  // async: E0, E1 of subdomain l -> bnd[]
-        if (l >= q) return;
-        const unsigned s0 = smem_u32(&bnd[0]), s1 = smem_u32(&bnd[1]);
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s0), "l"(p.sptr + l * spb) : "memory");
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s1), "l"(p.sptr + l * spb + nsl_of(l))
-                     : "memory");
-        asm volatile("cp.async.commit_group;" ::: "memory");
+    auto stage_bytes = [&](long long l, int64_t E0, int64_t E1) -> uint32_t {
+        const int nrows = (int)min((int64_t)R, p.n - (int64_t)l * R);
+        const uint32_t nsl = (uint32_t)((nrows + kSlice - 1) / kSlice);
+        return (uint32_t)(E1 - E0) * 12 + ((uint32_t)nrows & ~1u) * 16 + ((nsl * 8 + 15) & ~15u) +
+               ((nsl * 4 + 15) & ~15u);
     };
-    // subdomain of iteration j: slab buffer j % 2, row slot and barrier j % 3
-    auto issue = [&](long long l, int j, int64_t E0, int64_t E1) {
-        const int vs = j & 1, bs = j % 3;
-        slot_l[bs] = l;
+    // part w (0..3) of the stage of l_j (see above); one lane per warp
+    auto issue_part = [&](int w, long long j, const int64_t *bd, const int32_t *gr) {
+        const long long l = lof(j);
         if (l >= q) return;
+        const int vs = (int)(j & 1), bs = (int)(j % 3);
         const int64_t TS = l * (int64_t)R;
-        const int nrows = (int)min((int64_t)R, p.n - TS);
-        const int nsl = (nrows + kSlice - 1) / kSlice;
-        const uint32_t trows = (uint32_t)nrows & ~1u;
-        const uint32_t nb_sptr = ((uint32_t)nsl * 8 + 15) & ~15u, nb_sw = ((uint32_t)nsl * 4 + 15) & ~15u;
-        const uint32_t ne = (uint32_t)(E1 - E0);
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
         fence_proxy_async_smem();
-        mbar_arrive_expect_tx(&bars[bs], ne * 12 + trows * 16 + nb_sptr + nb_sw);
-        bulk_g2s(V, p.val + E0, ne * 8, &bars[bs]);
-        bulk_g2s(V + (size_t)g.vcap * 8, p.col + E0, ne * 4, &bars[bs]);
-        if (trows) {
-            bulk_g2s(B, p.b + TS, trows * 8, &bars[bs]);
-            bulk_g2s(B + g.o_x, p.x_in + TS, trows * 8, &bars[bs]);
+        if (w == 0) {
+            bulk_g2s(V, p.val + bd[0], (uint32_t)(bd[1] - bd[0]) * 8, &bars[bs]);
+        } else if (w == 1) {
+            bulk_g2s(V + (size_t)g.vcap * 8, p.col + bd[0], (uint32_t)(bd[1] - bd[0]) * 4, &bars[bs]);
+            if (gr) prefetch_ghost_x(p.x_in, gr, kGhostRanges);
+        } else if (w == 2) {
+            const uint32_t trows = (uint32_t)min((int64_t)R, p.n - TS) & ~1u;
+            if (trows) {
+                bulk_g2s(B, p.b + TS, trows * 8, &bars[bs]);
+                bulk_g2s(B + g.o_x, p.x_in + TS, trows * 8, &bars[bs]);
+            }
+        } else {
+            const uint32_t nsl = (uint32_t)nsl_of(l);
+            bulk_g2s(B + g.o_sptr, p.sptr + l * spb, (nsl * 8 + 15) & ~15u, &bars[bs]);
+            bulk_g2s(B + g.o_sw, p.sw + l * spb, (nsl * 4 + 15) & ~15u, &bars[bs]);
         }
-        bulk_g2s(B + g.o_sptr, p.sptr + l * spb, nb_sptr, &bars[bs]);
-        bulk_g2s(B + g.o_sw, p.sw + l * spb, nb_sw, &bars[bs]);
     };
-    long long l2 = 0, l3 = 0;  // claims: next to issue (bounds in flight to bnd[]), the one after
-    if (threadIdx.x == 0) {
+    // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
+    auto fetch_ring = [&](long long j) {
+        const long long l = lof(j);
+        if (l >= q) return;
+        const int r = (int)(j & 3);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
+                     : "memory");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][1])),
+                     "l"(p.sptr + l * spb + nsl_of(l))
+                     : "memory");
+        if (p.gr) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&gsm[r][0])),
+                         "l"(p.gr + 2 * l * kGhostRanges)
+                         : "memory");
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&gsm[r][4])),
+                         "l"(p.gr + 2 * l * kGhostRanges + 4)
+                         : "memory");
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    if (threadIdx.x == 0) {  // prologue: stages of l_0 and l_1, ring slots of l_2 and l_3
         for (int j = 0; j < 3; ++j) mbar_init(&bars[j], 1);
         fence_mbar_init();
-        const long long l0 = claim(0);
-        if (l0 < q) issue(l0, 0, p.sptr[l0 * spb], p.sptr[l0 * spb + nsl_of(l0)]);
-        else slot_l[0] = q;
-        const long long l1 = l0 < q ? claim(1) : q;
-        if (l1 < q) issue(l1, 1, p.sptr[l1 * spb], p.sptr[l1 * spb + nsl_of(l1)]);
-        else slot_l[1] = q;
-        l2 = l1 < q ? claim(2) : q;
-        fetch_bounds(l2);
-        l3 = l2 < q ? claim(3) : q;
+        for (int j = 0; j < 4; ++j) {
+            const long long l = lof(j);
+            if (l >= q) break;
+            bnd[j][0] = p.sptr[l * spb];
+            bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
+            for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
+        }
+        for (int j = 0; j < 2; ++j) {
+            const long long l = lof(j);
+            if (l >= q) break;
+            mbar_arrive_expect_tx(&bars[j], stage_bytes(l, bnd[j][0], bnd[j][1]));
+            for (int w = 0; w < 4; ++w) issue_part(w, j, bnd[j], j == 1 && p.gr ? gsm[j] : nullptr);
+        }
     }
     __syncthreads();
 
@@ -810,7 +851,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     double rr = 0.0, bb = 0.0;
     for (int i = 0;; ++i) {
         const int vs = i & 1, bs = i % 3;
-        const long long l = slot_l[bs];
+        const long long l = lof(i);
         if (l >= q) break;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
@@ -871,14 +912,17 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
             if (EXT) y1[loc] = ext_update(y0[loc], y0[loc] + lv[0] * acc, fz, p.tau);
             else y1[loc] = y0[loc] + lv[0] * acc;
         }
+        // post the byte count of l_{i+2}'s stage before the barrier that frees its buffers, so
+        // that no copy of it can complete bytes before its phase expects them
+        if (threadIdx.x == 0 && lof(i + 2) < q) {
+            const int r = (i + 2) & 3;
+            mbar_arrive_expect_tx(&bars[(i + 2) % 3], stage_bytes(lof(i + 2), bnd[r][0], bnd[r][1]));
+        }
         __syncthreads();
-        if (threadIdx.x == 0) {  // the slab buffer is free: stream subdomain l_{i+2} into it
-            asm volatile("cp.async.wait_all;" ::: "memory");
-            if (l2 < q) issue(l2, i + 2, bnd[0], bnd[1]);
-            else slot_l[(i + 2) % 3] = q;
-            l2 = l3;
-            fetch_bounds(l2);
-            l3 = l2 < q ? claim(i + 4) : q;
+        if (warp < 4 && lane == 0) {  // the slab buffer is free: stream l_{i+2} into it
+            const int r = (i + 2) & 3;
+            issue_part(warp, i + 2, bnd[r], p.gr ? gsm[r] : nullptr);
+            if (warp == 3) fetch_ring(i + 4);  // into slot i % 4 (l_i's, no longer read)
         }
         // a4: sweeps 2..k, direct form, off-block part frozen
         for (int t = 1; t < p.k; ++t) {
@@ -893,11 +937,15 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
             }
             __syncthreads();
         }
+        // ring slot of l_{i+3} complete before the barrier below publishes it (the newest group,
+        // l_{i+4}, may stay in flight)
+        if (warp == 3 && lane == 0) asm volatile("cp.async.wait_group 1;" ::: "memory");
         // a6: write back
         const double *yk = (p.k & 1) ? y1 : y0;
         for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
         __syncthreads();
     }
+    if (warp == 3 && lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
@@ -952,6 +1000,9 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
     // loads are waited on in the iteration that issues them: at iteration i it issues the stage
     // of l_next (bounds loaded during i-1), loads the bounds of l_next2 (claimed during i-1) and
     // claims a new subdomain.
+    // Ghost-range entries travel to shared memory by cp.async one iteration before their x
+    // ranges are prefetched into L2, two subdomains ahead of the gathers (a3) that read them.
+    __shared__ __align__(16) int32_t gsm[2 * kGhostRanges];
     long long l_next = 0, l_next2 = 0;
     int64_t e0n = 0, e1n = 0;
     if (threadIdx.x == 0) {
@@ -964,7 +1015,9 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
         issue(l0, 0, e0, e1);
         l_next = claim();
         bounds(l_next, e0n, e1n);
+        if (p.gr && l_next < q) prefetch_ghost_x(p.x_in, p.gr + 2 * l_next * kGhostRanges, kGhostRanges);
         l_next2 = claim();
+        fetch_ghost_entry(p, l_next2, q, gsm);
     }
     __syncthreads();
 
@@ -976,9 +1029,14 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
         if (l >= q) break;
         if (threadIdx.x == 0) {  // stream the next subdomain into the other stage
             issue(l_next, st ^ 1, e0n, e1n);
+            if (p.gr && l_next2 < q) {
+                asm volatile("cp.async.wait_all;" ::: "memory");
+                prefetch_ghost_x(p.x_in, gsm, kGhostRanges);
+            }
             l_next = l_next2;
             bounds(l_next, e0n, e1n);
             l_next2 = l_next < q ? claim() : q;
+            fetch_ghost_entry(p, l_next2, q, gsm);
         }
         unsigned char *S = smraw + (size_t)st * g.bytes;
         const int64_t TS = l * (int64_t)R;
@@ -1423,6 +1481,10 @@ KP make_kp(const Layout &L) {
     p.nslices = L.nslices;
     p.tau = 1.0;
     p.frozen = nullptr;
+    // measured on B200 (round 1, tools/kernel_ab.py): the L2 prefetch of the gather ranges pays
+    // for large subdomains (C5, R = 1024: 2.78 vs 2.87 ms per sync-block-(5) launch) and costs
+    // for small ones (C4, R = 128: 0.45 vs 0.41 ms), whose ranges are 1 KB
+    p.gr = (getenv("BAR_NO_GHOST_PREFETCH") || L.R < 512) ? nullptr : L.gr;
     return p;
 }
 
@@ -1598,11 +1660,13 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
                          ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
     const PipeGeom pg = pipe_geom(L.R, L.spb, L.max_w);
     const size_t pipe_smem = 2 * (size_t)pg.vc_bytes + 3 * (size_t)pg.bx_bytes;
-    // measured on B200 (round 1, tools/local_iters.py, sweep_R.py): the two-ahead pipeline wins
-    // for sync-block (C5: 2.96 vs 3.52 ms/iteration) and loses for async (3.40 vs 3.05), whose
-    // issue path (work-queue claim) sits on the critical warp; BAR_PIPE=0/1 overrides
+    // measured on B200 (round 1, tools/local_iters.py, kernel_ab.py): the two-ahead pipeline wins
+    // for sync-block (C5: 2.96 vs 3.52 ms/iteration) and, since async claims are static (no
+    // work-queue atomic on the issuing thread), for large-subdomain async and Jacobi too (C5:
+    // 2.88 vs 3.00 and 2.55 vs 2.67 ms); with R = 128 (C4) it is even. BAR_PIPE=0/1 overrides
     const char *pe = getenv("BAR_PIPE");
-    const bool pipe_on = pe ? pe[0] == '1' : (!ASYNC && p.k >= 3);
+    const bool pipe_on = (pe ? pe[0] == '1' : ((!ASYNC && p.k >= 3) || L.R >= 512)) &&
+                         (!ASYNC || p.static_claims);  // the pipeline claims statically
     if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
         if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);
         if (L.max_wl <= 6) return launch_pipe_t<ASYNC, 6>(p, L, pipe_smem, st);

@@ -61,4 +61,22 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         : "memory");
 }
 
+// Bulk L2 prefetch (no shared-memory destination, no completion): a hint that brings
+// [src, src + bytes) into L2 ahead of the loads that will read it. 16-byte aligned and sized.
+__device__ __forceinline__ void bulk_prefetch_l2(const void *src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
+// Prefetch the x ranges of one subdomain's ghost table entry (Layout::gr, kGhostRanges pairs of
+// (first column, count) already in shared memory) into L2.
+__device__ __forceinline__ void prefetch_ghost_x(const double *x, const int32_t *g, int nranges) {
+    for (int r = 0; r < nranges; ++r) {
+        const int32_t cnt = g[2 * r + 1];
+        if (cnt <= 0) continue;
+        const uintptr_t a0 = reinterpret_cast<uintptr_t>(x + g[2 * r]) & ~(uintptr_t)15;
+        const uintptr_t a1 = (reinterpret_cast<uintptr_t>(x + g[2 * r] + cnt) + 15) & ~(uintptr_t)15;
+        bulk_prefetch_l2(reinterpret_cast<const void *>(a0), (uint32_t)(a1 - a0));
+    }
+}
+
 }  // namespace bar

@@ -263,8 +263,10 @@ def test_siam_constant_async(bar, golden):
 # ------------------------------------------------------------------ every kernel generation
 @pytest.mark.parametrize("env", [{"BAR_KERNEL": "s"}, {"BAR_KERNEL": "r"}, {"BAR_KERNEL": "n"}, {"BAR_KERNEL": "p"},
                                  {"BAR_PIPE": "1"}, {"BAR_PIPE": "0"}, {"BAR_JACOBI_ROWWISE": "1"},
-                                 {"BAR_ASYNC_MULTI": "1"}, {"BAR_ASYNC_MULTI": "0"}])
-@pytest.mark.parametrize("name,R", [("fv1", 128), ("s7_m12", 288), ("tref2000", 128)])
+                                 {"BAR_ASYNC_MULTI": "1"}, {"BAR_ASYNC_MULTI": "0"}, {"BAR_NO_GHOST_PREFETCH": "1"},
+                                 {"BAR_ASYNC_STATIC": "0"}])
+@pytest.mark.parametrize("name,R", [("fv1", 128), ("s7_m12", 288), ("tref2000", 128), ("s7_m12", 512),
+                                    ("rand", 1024)])
 def test_forced_kernel_paths(bar, monkeypatch, env, name, R):
     """Each kernel the dispatcher can choose (fallbacks included) gives the oracle's iterates in
     the sync modes and converges in async (the environment variables only steer dispatch)."""

@@ -1,0 +1,95 @@
+"""A/B timing of kernel variants selected by environment switches (tuning aid, not a bench value).
+
+For one matrix, each variant (a set of BAR_* environment variables, read by libbar.so at every
+launch) is timed two ways with CUDA events on the launching stream:
+  * per launch: slope of 8 vs 40 back-to-back bar_sweep launches (cancels fixed overheads);
+  * whole solve: bar_solve to tol, median of --reps solves, with its global-iteration count.
+
+    python tools/kernel_ab.py --workload c5 --modes async,sync-block \
+        --variants 'base:;nopf:BAR_NO_GHOST_PREFETCH=1;pipe:BAR_PIPE=1'
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def parse_variants(spec):
+    out = []
+    for item in spec.split(";"):
+        if not item.strip():
+            continue
+        name, _, envs = item.partition(":")
+        env = {}
+        for kv in envs.split(","):
+            if kv.strip():
+                k, _, v = kv.partition("=")
+                env[k.strip()] = v.strip()
+        out.append((name.strip(), env))
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="c5")
+    ap.add_argument("--R", type=int, default=None)
+    ap.add_argument("--modes", default="async")
+    ap.add_argument("--k", type=int, default=5)
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--variants", default="base:")
+    a = ap.parse_args()
+    import torch
+
+    import bench
+    from paper_conf_ipps_anzttdh12_b200 import bar
+
+    R = a.R or bench.WORKLOADS[a.workload][2]
+    A = bench.make_matrix(a.workload)
+    M = bar.Matrix.from_csr(A, rows_per_block=R)
+    info = M.info()
+    del A
+    n = M.n
+    b = torch.ones(n, dtype=torch.float64, device="cuda")
+    x = torch.zeros(n, dtype=torch.float64, device="cuda")
+    st = torch.cuda.current_stream()
+
+    def ev_time(fn):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(st)
+        out = fn()
+        e1.record(st)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1), out
+
+    base_env = {k: os.environ.get(k) for k in ("BAR_PIPE", "BAR_NO_GHOST_PREFETCH", "BAR_KERNEL", "BAR_ASYNC_STATIC")}
+    for mode in a.modes.split(","):
+        for name, env in parse_variants(a.variants):
+            for k_, v in base_env.items():
+                if v is None:
+                    os.environ.pop(k_, None)
+                else:
+                    os.environ[k_] = v
+            os.environ.update(env)
+            M.sweep(b, x, k=a.k, nsweeps=4, mode=mode)
+            lo, hi = 8, 40
+            t_lo = min(ev_time(lambda: M.sweep(b, x, k=a.k, nsweeps=lo, mode=mode))[0] for _ in range(3))
+            t_hi = min(ev_time(lambda: M.sweep(b, x, k=a.k, nsweeps=hi, mode=mode))[0] for _ in range(3))
+            per_launch = (t_hi - t_lo) / (hi - lo)
+            M.solve(b, None, x, k=a.k, mode=mode)
+            solves = [ev_time(lambda: M.solve(b, None, x, k=a.k, mode=mode)) for _ in range(a.reps)]
+            ms = statistics.median(s[0] for s in solves)
+            iters = [s[1][1]["iters"] for s in solves]
+            print(json.dumps({"workload": a.workload, "R": R, "k": a.k, "mode": mode, "variant": name, "env": env,
+                              "launch_ms": round(per_launch, 4),
+                              "contract_GBs": round(info["model_bytes_per_iter"] / per_launch / 1e6, 1),
+                              "solve_ms": round(ms, 3), "iters": iters}), flush=True)
+    M.close()
+
+
+if __name__ == "__main__":
+    main()
