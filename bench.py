@@ -30,7 +30,7 @@ WORKLOADS = {
     "c1": ("Trefethen_2000 (exact)", ("trefethen", 2000), 128),
     "c2": ("fv1-shaped 9-point 98x98, diag 9.3595", ("stencil9", 98), 128),
     "c3": ("Trefethen_20000 (exact)", ("trefethen", 20000), 128),
-    "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 128),
+    "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 256),
     "c5": ("3D 7-point 512^3, diag 7.0249 (n=128M)", ("stencil7", 512), 1024),
 }
 METRIC = "time to rel. residual 1e-10 (s) and global iters/s with HBM GB/s vs peak, 1/2/4/8 GPU"
@@ -328,11 +328,12 @@ def main():
     t_lo = min(timed_sweeps(lo) for _ in range(3))
     t_hi = min(timed_sweeps(hi) for _ in range(3))
     kernel_ms = reduce((t_hi - t_lo) / (hi - lo), MAX)
+    kernel_name = M.info().get("last_sweep_kernel", "?") if world == 1 else "per-rank local sweep" 
     peak, peak_src = load_peaks()
     achieved = local_bytes / (kernel_ms * 1e-3) / 1e9  # per GPU
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": None,
-                "kernel": f"k_block_stage<{args.mode}>" if args.mode != "jacobi" else "k_rowwise_tma<jacobi>",
+                "kernel": kernel_name,
                 "kernel_ms": round(kernel_ms, 5), "algorithmic_bytes_per_launch": local_bytes,
                 "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
     prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")

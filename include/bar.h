@@ -83,6 +83,9 @@ typedef struct {
     int64_t local_entries;        /* entries with a column inside their row's subdomain (incl. diag) */
     double model_bytes_per_iter;  /* nnz*(8+4) + n*(8+8+8+4)                                      */
     int32_t device;
+    const char *last_sweep_kernel; /* static name of the sweep kernel the latest bar_solve /
+                                      bar_sweep launch on this handle used ("none" before any);
+                                      a diagnostic for profiling and the bench's roofline line  */
 } bar_matrix_info;
 
 /*

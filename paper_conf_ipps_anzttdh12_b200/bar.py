@@ -55,10 +55,12 @@ class MatrixInfo(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("rows_per_block", ctypes.c_int32),
                 ("num_subdomains", ctypes.c_int64), ("layout_entries", ctypes.c_int64),
                 ("local_entries", ctypes.c_int64), ("model_bytes_per_iter", ctypes.c_double),
-                ("device", ctypes.c_int32)]
+                ("device", ctypes.c_int32), ("last_sweep_kernel", ctypes.c_char_p)]
 
     def as_dict(self):
-        return {f: getattr(self, f) for f, _ in self._fields_}
+        d = {f: getattr(self, f) for f, _ in self._fields_}
+        d["last_sweep_kernel"] = (d["last_sweep_kernel"] or b"").decode()
+        return d
 
 
 _vp, _i64, _i32, _f64 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_double

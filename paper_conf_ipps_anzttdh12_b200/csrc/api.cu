@@ -187,6 +187,7 @@ bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info) {
     info->local_entries = L.local_entries;
     info->model_bytes_per_iter = model_bytes(L);
     info->device = A->device;
+    info->last_sweep_kernel = L.last_kernel;
     return BAR_OK;
 }
 

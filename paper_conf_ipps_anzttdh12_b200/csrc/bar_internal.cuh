@@ -68,6 +68,7 @@ struct Layout {
     // [q][kGhostRanges] (first column, count) of x ranges holding most of subdomain l's
     // off-block columns (count 0 = unused): bulk L2 prefetch targets for the a3 gathers
     int32_t *gr = nullptr;
+    mutable const char *last_kernel = "none";  // name of the most recently launched sweep kernel
 };
 constexpr int kGhostRanges = 4;
 

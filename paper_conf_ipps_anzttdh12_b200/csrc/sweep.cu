@@ -1661,19 +1661,22 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const PipeGeom pg = pipe_geom(L.R, L.spb, L.max_w);
     const size_t pipe_smem = 2 * (size_t)pg.vc_bytes + 3 * (size_t)pg.bx_bytes;
     // measured on B200 (round 1, tools/local_iters.py, kernel_ab.py): the two-ahead pipeline wins
-    // for sync-block (C5: 2.96 vs 3.52 ms/iteration) and, since async claims are static (no
-    // work-queue atomic on the issuing thread), for large-subdomain async and Jacobi too (C5:
-    // 2.88 vs 3.00 and 2.55 vs 2.67 ms); with R = 128 (C4) it is even. BAR_PIPE=0/1 overrides
+    // for sync-block (C5: 2.64 vs 3.51 ms/iteration) and, since async claims are static (no
+    // work-queue atomic on the issuing thread), for async and Jacobi with R >= 256 too (C5:
+    // 2.65 vs 3.35 and 2.58 vs 2.69 ms; C4 at R = 256: 0.38 vs 0.42 ms); with R = 128 (C4) the
+    // one-ahead kernel is 2% faster for async. BAR_PIPE=0/1 overrides
     const char *pe = getenv("BAR_PIPE");
-    const bool pipe_on = (pe ? pe[0] == '1' : ((!ASYNC && p.k >= 3) || L.R >= 512)) &&
+    const bool pipe_on = (pe ? pe[0] == '1' : ((!ASYNC && p.k >= 3) || L.R >= 256)) &&
                          (!ASYNC || p.static_claims);  // the pipeline claims statically
     if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
+        L.last_kernel = ASYNC ? "k_block_pipe<async>" : "k_block_pipe<sync>";
         if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);
         if (L.max_wl <= 6) return launch_pipe_t<ASYNC, 6>(p, L, pipe_smem, st);
         if (L.max_wl <= 8) return launch_pipe_t<ASYNC, 8>(p, L, pipe_smem, st);
         return launch_pipe_t<ASYNC, 16>(p, L, pipe_smem, st);
     }
     if (kind == 't' && geom_ok && aligned && stage_smem <= kSmemMax) {
+        L.last_kernel = p.w_end > 0 ? "k_block_stage_m<async>" : ASYNC ? "k_block_stage<async>" : "k_block_stage<sync>";
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
         if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
         if (L.max_wl <= 8) return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
@@ -1682,16 +1685,22 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     if (p.w_end > 0) return cudaErrorNotSupported;  // no persistent multi-iteration kernel here
     const bool ext = p.frozen != nullptr || p.tau != 1.0;  // N1/N3: only k_block_stage and k_block
     if (!ext && (kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
+        L.last_kernel = ASYNC ? "k_block_pers<async>" : "k_block_pers<sync>";
         if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
         if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
         return launch_pers_t<ASYNC, 8>(p, L, pers_smem, st);
     }
     if (!ext && (kind == 't' || kind == 'n') && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
+        L.last_kernel = ASYNC ? "k_reg_tma<async>" : "k_reg_tma<sync>";
         if (L.max_wl <= 4) return launch_reg_tma_t<ASYNC, 4>(p, L, tma_smem, st);
         if (L.max_wl <= 6) return launch_reg_tma_t<ASYNC, 6>(p, L, tma_smem, st);
         return launch_reg_tma_t<ASYNC, 8>(p, L, tma_smem, st);
     }
-    if (!ext && kind != 's' && L.spb <= 32 && L.max_wl <= 8) return launch_reg_w<ASYNC, 1>(p, L, st);
+    if (!ext && kind != 's' && L.spb <= 32 && L.max_wl <= 8) {
+        L.last_kernel = ASYNC ? "k_reg<async>" : "k_reg<sync>";
+        return launch_reg_w<ASYNC, 1>(p, L, st);
+    }
+    L.last_kernel = ASYNC ? "k_block<async>" : "k_block<sync>";
     const size_t row_bytes = 3 * (size_t)L.R * sizeof(double);  // y0, y1, s
     const size_t stage_bytes = (size_t)L.max_wl * L.spb * kSlice * (sizeof(double) + sizeof(int32_t));
     const bool stage = row_bytes + stage_bytes <= kSmemBudget;
@@ -1714,6 +1723,7 @@ cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
     p.wmax = L.max_w;
     const char *kv = getenv("BAR_KERNEL");
     if (!rowwise_tma_ok(L) || (kv && kv[0] == 'r')) {
+        if (!RES) L.last_kernel = "k_rowwise<jacobi>";
         k_rowwise<RES><<<(unsigned)((L.nslices + 7) / 8), 256, 0, st>>>(p);
         return cudaGetLastError();
     }
@@ -1724,6 +1734,7 @@ cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
         if (e != cudaSuccess) return e;
         attr = smem;
     }
+    if (!RES) L.last_kernel = "k_rowwise_tma<jacobi>";
     k_rowwise_tma<RES><<<(unsigned)rowwise_grid(L), 256, smem, st>>>(p);
     return cudaGetLastError();
 }

@@ -66,7 +66,17 @@ def main():
         torch.cuda.synchronize()
         return e0.elapsed_time(e1), out
 
-    base_env = {k: os.environ.get(k) for k in ("BAR_PIPE", "BAR_NO_GHOST_PREFETCH", "BAR_KERNEL", "BAR_ASYNC_STATIC")}
+    # box reference: device copy bandwidth (read + write bytes), as MEASURED_PEAKS.json measures it
+    src = torch.empty(1 << 27, dtype=torch.float64, device="cuda")
+    dst = torch.empty_like(src)
+    dst.copy_(src)
+    copy_ms = min(ev_time(lambda: dst.copy_(src))[0] for _ in range(10))
+    copy_gbs = 2 * src.numel() * 8 / copy_ms / 1e6
+    del src, dst
+    clk = os.popen("nvidia-smi --query-gpu=clocks.sm,clocks.mem,power.draw --format=csv,noheader").read().strip()
+    print(json.dumps({"box": {"copy_GBs": round(copy_gbs, 1), "clocks": clk}}), flush=True)
+    base_env = {k: os.environ.get(k) for k in ("BAR_PIPE", "BAR_NO_GHOST_PREFETCH", "BAR_KERNEL", "BAR_ASYNC_STATIC",
+                                          "BAR_ISSUE_WARPS")}
     for mode in a.modes.split(","):
         for name, env in parse_variants(a.variants):
             for k_, v in base_env.items():
@@ -87,6 +97,8 @@ def main():
             print(json.dumps({"workload": a.workload, "R": R, "k": a.k, "mode": mode, "variant": name, "env": env,
                               "launch_ms": round(per_launch, 4),
                               "contract_GBs": round(info["model_bytes_per_iter"] / per_launch / 1e6, 1),
+                              "frac_of_copy": round(info["model_bytes_per_iter"] / per_launch / 1e6 / copy_gbs, 3),
+                              "kernel": M.info()["last_sweep_kernel"],
                               "solve_ms": round(ms, 3), "iters": iters}), flush=True)
     M.close()
 
