@@ -949,6 +949,223 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+// ---------------------------------------------------------------------------------------------
+// k_block_duo: the pipelined sweep for large subdomains with TWO resident blocks per SM. With one
+// 1024-thread block per SM (k_block_pipe at R = 1024), every block-wide barrier of a subdomain
+// (after its gathers, after each local sweep) idles the SM's memory pipeline until the slowest
+// warp arrives (ncu: barrier stalls were the top reason). Here a block of R/2 threads sweeps a
+// subdomain with two rows per thread (slices w and w + R/64 of warp w), and its shared memory
+// holds ONE matrix slab (values, columns, slice metadata) plus the y double buffer, so two
+// blocks fit per SM and one block's barriers are covered by the other's work. b_J and x_J are
+// read with coalesced loads (their ranges are bulk-prefetched into L2 one subdomain ahead), so
+// y^0 = x_J is written to shared memory by each thread and the first sweep follows the barrier
+// that also frees the slab. The slab of the next subdomain is issued right after that barrier,
+// split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
+// Subdomains are claimed statically: block c sweeps l_j = c + j G.
+struct DuoGeom {
+    uint32_t vcap, o_col, o_sptr, o_sw, o_ya, o_yb, bytes;
+};
+
+__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax) {
+    DuoGeom g;
+    g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
+    g.o_col = g.vcap * 8;
+    g.o_sptr = (g.o_col + g.vcap * 4 + 15) & ~15u;
+    g.o_sw = g.o_sptr + (((uint32_t)spb * 8 + 15) & ~15u);
+    g.o_ya = (g.o_sw + (((uint32_t)spb * 4 + 15) & ~15u) + 127) & ~127u;
+    g.o_yb = g.o_ya + (uint32_t)R * 8;
+    g.bytes = g.o_yb + (uint32_t)R * 8;
+    return g;
+}
+
+template <bool ASYNC, int WLR, bool EXT = false>
+__global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
+    if (*(volatile int *)&p.state->stop) return;
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ __align__(8) uint64_t bar;
+    __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
+    __shared__ __align__(16) int32_t gsm[4][2 * kGhostRanges];  // [j % 4]: ghost ranges of l_j
+    const int R = p.R, spb = p.spb;
+    const DuoGeom g = duo_geom(R, spb, p.wmax);
+    const int64_t q = (p.n + R - 1) / R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nw = blockDim.x >> 5;  // = spb / 2
+    const long long G = gridDim.x;
+    double *ya = reinterpret_cast<double *>(smraw + g.o_ya);
+    double *yb = reinterpret_cast<double *>(smraw + g.o_yb);
+    auto lof = [&](long long j) { return (long long)blockIdx.x + j * G; };
+    auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
+    auto slab_bytes = [&](long long l, const int64_t *bd) -> uint32_t {
+        const uint32_t nsl = (uint32_t)nsl_of(l);
+        return (uint32_t)(bd[1] - bd[0]) * 12 + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u);
+    };
+    // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
+    auto issue_part = [&](int w, long long j) {
+        const long long l = lof(j);
+        if (l >= q) return;
+        const int64_t *bd = bnd[j & 3];
+        if (w == 3) {  // what l_j's first phase reads directly: b_J, x_J and its ghost x ranges
+            const int64_t TS = l * (int64_t)R;
+            const uint32_t nrows = (uint32_t)min((int64_t)R, p.n - TS);
+            const uintptr_t b0 = reinterpret_cast<uintptr_t>(p.b + TS) & ~(uintptr_t)15;
+            const uintptr_t b1 = (reinterpret_cast<uintptr_t>(p.b + TS + nrows) + 15) & ~(uintptr_t)15;
+            bulk_prefetch_l2(reinterpret_cast<const void *>(b0), (uint32_t)(b1 - b0));
+            const uintptr_t x0 = reinterpret_cast<uintptr_t>(p.x_in + TS) & ~(uintptr_t)15;
+            const uintptr_t x1 = (reinterpret_cast<uintptr_t>(p.x_in + TS + nrows) + 15) & ~(uintptr_t)15;
+            bulk_prefetch_l2(reinterpret_cast<const void *>(x0), (uint32_t)(x1 - x0));
+            if (p.gr) prefetch_ghost_x(p.x_in, gsm[j & 3], kGhostRanges);
+            return;
+        }
+        fence_proxy_async_smem();
+        const uint32_t ne = (uint32_t)(bd[1] - bd[0]);
+        if (w == 0) {
+            bulk_g2s(smraw, p.val + bd[0], ne * 8, &bar);
+        } else if (w == 1) {
+            bulk_g2s(smraw + g.o_col, p.col + bd[0], ne * 4, &bar);
+        } else {
+            const uint32_t nsl = (uint32_t)nsl_of(l);
+            bulk_g2s(smraw + g.o_sptr, p.sptr + l * spb, (nsl * 8 + 15) & ~15u, &bar);
+            bulk_g2s(smraw + g.o_sw, p.sw + l * spb, (nsl * 4 + 15) & ~15u, &bar);
+        }
+    };
+    // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
+    auto fetch_ring = [&](long long j) {
+        const long long l = lof(j);
+        if (l >= q) return;
+        const int r = (int)(j & 3);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
+                     : "memory");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][1])),
+                     "l"(p.sptr + l * spb + nsl_of(l))
+                     : "memory");
+        if (p.gr) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&gsm[r][0])),
+                         "l"(p.gr + 2 * l * kGhostRanges)
+                         : "memory");
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&gsm[r][4])),
+                         "l"(p.gr + 2 * l * kGhostRanges + 4)
+                         : "memory");
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    if (threadIdx.x == 0) {  // prologue: ring slots of l_0 .. l_2, the slab of l_0
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+        for (int j = 0; j < 3; ++j) {
+            const long long l = lof(j);
+            if (l >= q) break;
+            bnd[j][0] = p.sptr[l * spb];
+            bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
+            for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
+        }
+        mbar_arrive_expect_tx(&bar, slab_bytes(lof(0), bnd[0]));
+        for (int w = 0; w < 4; ++w) issue_part(w, 0);
+    }
+    __syncthreads();
+
+    constexpr int NP = WLR / 2;
+    double rr = 0.0, bb = 0.0;
+    for (int i = 0;; ++i) {
+        const long long l = lof(i);
+        if (l >= q) break;
+        const int64_t TS = l * (int64_t)R;
+        const int nrows = (int)min((int64_t)R, p.n - TS);
+        const int nsl = (nrows + kSlice - 1) / kSlice;
+        mbar_wait(&bar, i & 1);
+        double lv[2][WLR];
+        uint32_t lc[2][NP];
+        double s[2] = {0.0, 0.0};
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) lv[h][e] = 0.0;
+#pragma unroll
+            for (int e = 0; e < NP; ++e) lc[h][e] = 0;
+        }
+        auto row_of = [&](int h) { return (warp + h * nw) * kSlice + lane; };  // local row of slice h
+        // a2/a3: b_i and x_i (direct, L2-prefetched; x_i -> y^0), the off-block part with x as
+        // it stands, the local entries into registers
+        const int64_t *ssp = reinterpret_cast<const int64_t *>(smraw + g.o_sptr);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int sl = warp + h * nw, loc = row_of(h);
+            if (sl >= nsl || loc >= nrows) continue;
+            const int sw = reinterpret_cast<const int32_t *>(smraw + g.o_sw)[sl];
+            const int wl = sw & 0xffff, wo = sw >> 16;
+            const int64_t off = ssp[sl] - ssp[0] + lane;
+            const double *sv = reinterpret_cast<const double *>(smraw) + off;
+            const int32_t *sc = reinterpret_cast<const int32_t *>(smraw + g.o_col) + off;
+            const double bi = p.b[TS + loc];
+            ya[loc] = ldx<ASYNC>(p.x_in + TS + loc);
+            double acc = bi;
+            for (int e0 = 0; e0 < wo; e0 += U) {
+                double xv[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+            }
+            s[h] = acc;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) {
+                if (e < wl) {
+                    lv[h][e] = sv[(wo + e) * kSlice];
+                    lc[h][e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                }
+            }
+            bb += bi * bi;
+        }
+        // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
+        if (threadIdx.x == 0 && lof(i + 1) < q) mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3]));
+        __syncthreads();
+        if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
+            issue_part(warp, i + 1);
+            if (warp == 3) fetch_ring(i + 3);  // into slot (i + 3) % 4 (l_{i-1}'s, no longer read)
+        }
+        // first local sweep in the correction form; its numerator is the residual (a5)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int loc = row_of(h);
+            if (warp + h * nw >= nsl || loc >= nrows) continue;
+            double acc = s[h];
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[h][e] * ya[(lc[h][e >> 1] >> (16 * (e & 1))) & 0xffff];
+            lv[h][0] = 1.0 / lv[h][0];
+            rr += acc * acc;
+            const double xo = ya[loc];
+            if (EXT) yb[loc] = ext_update(xo, xo + lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
+            else yb[loc] = xo + lv[h][0] * acc;
+        }
+        __syncthreads();
+        // a4: sweeps 2..k, direct form, off-block part frozen
+        for (int t = 1; t < p.k; ++t) {
+            const double *yi = (t & 1) ? yb : ya;
+            double *yo = (t & 1) ? ya : yb;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int loc = row_of(h);
+                if (warp + h * nw >= nsl || loc >= nrows) continue;
+                double acc = s[h];
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[h][e] * yi[(lc[h][e >> 1] >> (16 * (e & 1))) & 0xffff];
+                if (EXT) yo[loc] = ext_update(yi[loc], lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
+                else yo[loc] = lv[h][0] * acc;
+            }
+            __syncthreads();
+        }
+        // ring slot of l_{i+2} complete before the barrier below publishes it
+        if (warp == 3 && lane == 0) asm volatile("cp.async.wait_group 1;" ::: "memory");
+        // a6: write back
+        const double *yk = (p.k & 1) ? yb : ya;
+        for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
+        __syncthreads();
+    }
+    if (warp == 3 && lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
+    reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
+}
+
 // Per-launch staged sweep (one global iteration per launch).
 template <bool ASYNC, int WLR, bool EXT = false>
 __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
@@ -1617,6 +1834,32 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
 }
 
 template <bool ASYNC, int WLR>
+cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    const bool ext = p.frozen != nullptr || p.tau != 1.0;
+    auto kfn = ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>;
+    static size_t attr[2] = {0, 0};
+    static size_t c_smem[2] = {0, 0};
+    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
+    const int v = ext ? 1 : 0;
+    const int threads = L.spb / 2 * kSlice;
+    if (smem > attr[v]) {
+        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        attr[v] = smem;
+    }
+    if (c_smem[v] != smem || c_threads[v] != threads) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, threads, smem) != cudaSuccess || occ[v] < 1)
+            occ[v] = 1;
+        c_smem[v] = smem;
+        c_threads[v] = threads;
+    }
+    int64_t g = (int64_t)occ[v] * L.sms;
+    if (g > L.q) g = L.q;
+    kfn<<<(unsigned)g, threads, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <bool ASYNC, int WLR>
 cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     if (ASYNC && p.w_end > 0) return launch_stage_m<true, WLR, true>(p, L, smem, st);
     return launch_stage_m<ASYNC, WLR, false>(p, L, smem, st);
@@ -1668,6 +1911,22 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const char *pe = getenv("BAR_PIPE");
     const bool pipe_on = (pe ? pe[0] == '1' : ((!ASYNC && p.k >= 3) || L.R >= 256)) &&
                          (!ASYNC || p.static_claims);  // the pipeline claims statically
+    // two-blocks-per-SM variant (k_block_duo) where the pipelined kernel holds a whole SM (C5
+    // sync modes, B200 round 1, tools/kernel_ab.py: Jacobi 2.45 vs 2.58 ms, sync-block-(5) 2.56-2.67
+    // vs 2.67 ms per launch); BAR_DUO=0/1 overrides
+    const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w).bytes;
+    const char *de = getenv("BAR_DUO");
+    const bool duo_fits = L.spb % 2 == 0 && L.spb >= 8 && L.max_wl <= 4 && 2 * (duo_smem + 2048) <= 228 * 1024;
+    // Async keeps one block per SM by default: with 2 x 148 subdomains in flight the window of
+    // concurrently swept rows (303K on C5) exceeds the plane coupling distance (262K), the
+    // block Gauss-Seidel effect of the monotone order (R15) is lost and async-(5) needs 65
+    // instead of 58 global iterations (faster launches, slower solve)
+    const bool duo_on = (de ? de[0] == '1' : (!ASYNC && pipe_smem > 113 * 1024)) && duo_fits &&
+                        (!ASYNC || p.static_claims);
+    if (kind == 't' && duo_on && p.w_end == 0 && geom_ok && aligned) {
+        L.last_kernel = ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>";
+        return launch_duo_t<ASYNC, 4>(p, L, duo_smem, st);  // two rows per thread: <= 4 local entries
+    }
     if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
         L.last_kernel = ASYNC ? "k_block_pipe<async>" : "k_block_pipe<sync>";
         if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);

@@ -283,3 +283,26 @@ def test_forced_kernel_paths(bar, monkeypatch, env, name, R):
         _close(x, ref)
     x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10)
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+# ------------------------------------------------------------------ pipelined / two-blocks-per-SM
+@pytest.mark.parametrize("env", [{"BAR_DUO": "1"}, {"BAR_DUO": "0"}, {"BAR_DUO": "0", "BAR_PIPE": "0"}])
+def test_large_subdomain_kernels(bar, monkeypatch, env):
+    """C5's shape at a testable size: 3D 7-point, m = 128, R = 256 = two grid lines (so a row has
+    at most 4 local entries, as at 512^3 with R = 1024). The two-blocks-per-SM kernel
+    (k_block_duo), the pipelined kernel (k_block_pipe) and the one-ahead kernel (k_block_stage)
+    give the oracle's sync-block-(5) and Jacobi iterates and converge in async."""
+    for k_, v in env.items():
+        monkeypatch.setenv(k_, v)
+    A = W.stencil7_3d(128)
+    R = 256
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(5).uniform(-1, 1, A.n)
+    for mode, k in (("sync-block", 5), ("jacobi", 1)):
+        ref = x0
+        for _ in range(2):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x, _ = _solve(bar, A, b, R, k, mode, 2, 0.0, x0)
+        _close(x, ref)
+    x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10)
+    assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
