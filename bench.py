@@ -161,6 +161,56 @@ def oracle_sample(workload: str, k: int, R: int, mode: str, budget_rows: int):
     return dt * scale, desc
 
 
+# Smaller grid of the same stencil (same diagonal, rho(B) within 0.3%) whose oracle solves give
+# the Jacobi / Gauss-Seidel iteration counts for the configs too large to iterate on the host.
+PROXY = {"c4": ("stencil9", 400), "c5": ("stencil7", 64)}
+
+
+def oracle_jacobi_gs(workload: str, budget_rows: int):
+    """The oracle's Jacobi (O1) and forward Gauss-Seidel (O3) time to rel_res 1e-10 on one host
+    core (north star: "the oracle's Jacobi and Gauss-Seidel time on the box's host cores").
+
+    C1-C3: full oracle solves. C4/C5: seconds per iteration from ONE sweep over the leading
+    principal submatrix of the first `budget_rows` rows (x rows/n to the full matrix), times the
+    iteration count of the oracle's solve on PROXY's smaller grid of the same stencil."""
+    import oracle as O
+    import workloads as W
+
+    n, _ = matrix_dims(workload)
+    out = {}
+    if workload not in PROXY:
+        A = make_matrix(workload)
+        b = np.ones(n)
+        for name, method in (("jacobi", O.JACOBI), ("gauss_seidel", O.GAUSS_SEIDEL)):
+            t0 = time.perf_counter()
+            r = O.solve(A, b, method=method, max_iters=20000, tol=1e-10)
+            dt = time.perf_counter() - t0
+            out[name] = {"value": dt, "unit": "s", "iters": r.iters, "converged": r.converged,
+                         "sample": "full oracle solve to rel_res 1e-10 (b = 1, x0 = 0)"}
+        return out
+    rows = min(n, budget_rows)
+    A = make_matrix(workload, 0, rows)
+    keep = A.col < rows  # leading principal submatrix: a square system the sweeps can run on
+    cnt = np.add.reduceat(keep.astype(np.int64), A.rowptr[:-1]) if rows else np.zeros(0, np.int64)
+    rp = np.zeros(rows + 1, dtype=np.int32)
+    np.cumsum(cnt, out=rp[1:])
+    S = W.CSR(rows, rp, np.ascontiguousarray(A.col[keep]), np.ascontiguousarray(A.val[keep]))
+    del A
+    kind, m = PROXY[workload]
+    P = W.stencil9_2d(m, W.FV1_DIAG, -1.0) if kind == "stencil9" else W.stencil7_3d(m, W.S7_DIAG, -1.0)
+    bs, xs = np.ones(rows), np.full(rows, 0.5)
+    for name, method, sweep in (("jacobi", O.JACOBI, lambda: O.jacobi_step(S, bs, xs)),
+                                ("gauss_seidel", O.GAUSS_SEIDEL, lambda: O.gauss_seidel_step(S, bs, xs))):
+        t0 = time.perf_counter()
+        sweep()
+        s_iter = (time.perf_counter() - t0) * n / rows
+        r = O.solve(P, np.ones(P.n), method=method, max_iters=20000, tol=1e-10)
+        out[name] = {"value": s_iter * r.iters, "unit": "s", "iters": r.iters, "s_per_iter": s_iter,
+                     "sample": f"1 oracle sweep over the leading {rows}x{rows} block, x{n / rows:.2f} to n; "
+                               f"iterations of the oracle's own solve on the {kind} m={m} grid (same diagonal)"}
+    return out
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle as it stands, on this box's host cores (rank 0 only)."""
     rank = int(os.environ.get("RANK", "0"))
@@ -307,9 +357,14 @@ def main():
     assert all(i["converged"] for i in infos), infos
     mean_iters = sum(iters) / len(iters)
 
-    # dominant kernel: per-launch duration of the block-sweep kernel, from the slope of
-    # back-to-back launch batches timed with CUDA events on the launching stream (cancels fixed
-    # overheads); multi-GPU: the local kernel of each rank (no exchange), max over ranks
+    # dominant kernel, live: libbar records CUDA events on the launching stream around every
+    # block-sweep launch of the timed solves (bar_solve_info.sweep_kernel_ms / _iters; launches
+    # queued after a stop request excluded) -> device ms per global iteration, max over ranks
+    sk_ms = sum(i["sweep_kernel_ms"] for i in infos)
+    sk_it = sum(i["sweep_kernel_iters"] for i in infos)
+    kernel_ms = reduce(sk_ms / sk_it if sk_it > 0 else float("nan"), MAX)
+    # cross-check: per-launch duration from the slope of back-to-back launch batches outside the
+    # solve (cancels fixed overheads); multi-GPU: the local kernel of each rank, max over ranks
     xs = torch.zeros(n_loc, dtype=torch.float64, device=dev)
 
     def timed_sweeps(nsw):
@@ -327,7 +382,7 @@ def main():
     lo, hi = 8, 40
     t_lo = min(timed_sweeps(lo) for _ in range(3))
     t_hi = min(timed_sweeps(hi) for _ in range(3))
-    kernel_ms = reduce((t_hi - t_lo) / (hi - lo), MAX)
+    kernel_ms_isolated = reduce((t_hi - t_lo) / (hi - lo), MAX)
     kernel_name = M.info().get("last_sweep_kernel", "?") if world == 1 else "per-rank local sweep" 
     peak, peak_src = load_peaks()
     achieved = local_bytes / (kernel_ms * 1e-3) / 1e9  # per GPU
@@ -335,6 +390,10 @@ def main():
                 "frac": round(achieved / peak, 4), "traffic": None,
                 "kernel": kernel_name,
                 "kernel_ms": round(kernel_ms, 5), "algorithmic_bytes_per_launch": local_bytes,
+                "timing": f"CUDA events around each sweep launch inside the {args.steps} timed solves "
+                          f"({sk_it:g} global iterations, {sk_ms:.3f} ms of sweep kernels on rank 0)",
+                "kernel_ms_isolated": round(kernel_ms_isolated, 5),
+                "frac_isolated": round(local_bytes / (kernel_ms_isolated * 1e-3) / 1e9 / peak, 4),
                 "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
     prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")
     if world == 1 and os.path.exists(prof):
@@ -372,6 +431,7 @@ def main():
         cpu = {"value": s_iter * mean_iters, "unit": "s", "cores": 1, "kind": "oracle",
                "sample": desc + f" ({mean_iters:g})", "cpu": model, "host_cores": cores,
                "s_per_global_iter": s_iter}
+        cpu.update(oracle_jacobi_gs(args.workload, 4_000_000))
 
     value = ms_per_step / 1e3
     line = {

@@ -73,6 +73,12 @@ typedef struct {
     int64_t cta_iters_max;  /*   counts (= iters otherwise)                                       */
     double model_bytes_per_iter; /* nnz*(8+4) + n*(8+8+8+4): the contract bytes of one iteration */
     int64_t kernel_launches;     /* kernels this call launched (all of them libbar's own)         */
+    double sweep_kernel_ms;      /* device time of the block-sweep launches that did work, from CUDA
+                                    events recorded on cuda_stream around each launch (excludes
+                                    residual/setup kernels and launches queued after a stop)     */
+    double sweep_kernel_iters;   /* global iterations those launches performed (one per launch; the
+                                    single-launch async kernel: subdomain sweeps claimed / q), so
+                                    sweep_kernel_ms / sweep_kernel_iters = device ms per iteration */
 } bar_solve_info;
 
 typedef struct {

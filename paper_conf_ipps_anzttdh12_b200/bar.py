@@ -39,7 +39,8 @@ EXPORTS = ("bar_create_csr", "bar_solve", "bar_solve_ex", "bar_sweep", "bar_resi
 class SolveInfo(ctypes.Structure):
     _fields_ = [("iters", ctypes.c_int64), ("rel_res", ctypes.c_double), ("converged", ctypes.c_int32),
                 ("cta_iters_min", ctypes.c_int64), ("cta_iters_max", ctypes.c_int64),
-                ("model_bytes_per_iter", ctypes.c_double), ("kernel_launches", ctypes.c_int64)]
+                ("model_bytes_per_iter", ctypes.c_double), ("kernel_launches", ctypes.c_int64),
+                ("sweep_kernel_ms", ctypes.c_double), ("sweep_kernel_iters", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -78,6 +78,47 @@ bar_status read_state(bar_matrix A, cudaStream_t st) {
     return BAR_OK;
 }
 
+void timer_reset(KernelTimer &T) {
+    T.used = 0;
+    T.ms = 0.0;
+    T.iters = 0.0;
+}
+
+bar_status timer_begin(KernelTimer &T, int64_t m, cudaStream_t st) {
+    if (T.used >= KernelTimer::kMax) return BAR_OK;  // not recorded (never reached: chunks <= kMax)
+    cudaEvent_t &e0 = T.ev[2 * T.used], &e1 = T.ev[2 * T.used + 1];
+    if (!e0) BAR_CUDA(cudaEventCreate(&e0));
+    if (!e1) BAR_CUDA(cudaEventCreate(&e1));
+    T.m[T.used] = m;
+    BAR_CUDA(cudaEventRecord(e0, st));
+    return BAR_OK;
+}
+
+bar_status timer_end(KernelTimer &T, cudaStream_t st) {
+    if (T.used >= KernelTimer::kMax) return BAR_OK;
+    BAR_CUDA(cudaEventRecord(T.ev[2 * T.used + 1], st));
+    ++T.used;
+    return BAR_OK;
+}
+
+bar_status timer_collect(KernelTimer &T, int64_t bound, double iters_each) {
+    for (int i = 0; i < T.used; ++i) {
+        if (T.m[i] > bound) continue;
+        float ms = 0.f;
+        BAR_CUDA(cudaEventElapsedTime(&ms, T.ev[2 * i], T.ev[2 * i + 1]));
+        T.ms += ms;
+        T.iters += iters_each;
+    }
+    T.used = 0;
+    return BAR_OK;
+}
+
+void timer_free(KernelTimer &T) {
+    for (auto &e : T.ev)
+        if (e) cudaEventDestroy(e), e = nullptr;
+    T.used = 0;
+}
+
 }  // namespace bar
 
 using namespace bar;
@@ -163,6 +204,7 @@ void bar_destroy(bar_matrix A) {
     DeviceGuard g(A->device);
     free_layout(A->L);
     Workspace &W = A->W;
+    timer_free(W.timer);
     cudaFree(W.xbuf);
     cudaFree(W.stage_b);
     cudaFree(W.stage_x);
@@ -296,6 +338,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
     const size_t bytes = sizeof(double) * (size_t)n;
     bar_status r = ensure_workspace(A);
     if (r != BAR_OK) return r;
+    KernelTimer &T = W.timer;
+    timer_reset(T);
     int64_t launches = 0;
     // N1 failure mask (device copy) and the per-launch window; residual history buffer
     const uint8_t *d_mask = nullptr;
@@ -360,12 +404,16 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 SweepArgs a{&L, db, (m & 1) ? buf0 : buf1, (m & 1) ? buf1 : buf0, k, W.state, W.partials, d_hist};
                 a.frozen = mask_at(m);
                 a.tau = tau;
+                if ((r = timer_begin(T, m, st)) != BAR_OK) return r;
                 BAR_CUDA(launch_sweep(a, mode, st));
+                if ((r = timer_end(T, st)) != BAR_OK) return r;
             }
             launches += c;
             issued += c;
             if ((r = read_state(A, st)) != BAR_OK) return r;
             stopped = H.stop != 0;
+            // H.iter counts the launches that ran (those queued after the stop returned at once)
+            if ((r = timer_collect(T, (int64_t)H.iter, 1.0)) != BAR_OK) return r;
             chunk = std::min<int64_t>(chunk * 2, 256);
         }
         if (stopped) {
@@ -405,18 +453,28 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         if (ext_opts) multi = false;
         bool used_multi = false;
         const long long w_end = (long long)max_global_iters * (long long)L.q;
+        unsigned long long claimed_before = 0;
         while (multi && !converged && !bzero && !diverged && max_global_iters > 0) {
             SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+            if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
             cudaError_t e = launch_async_multi(a, w_end, st);
             if (e == cudaErrorNotSupported) {
                 cudaGetLastError();
+                T.used = 0;
                 multi = false;
                 break;
             }
             BAR_CUDA(e);
+            if ((r = timer_end(T, st)) != BAR_OK) return r;
             used_multi = true;
             ++launches;
             if ((r = read_state(A, st)) != BAR_OK) return r;
+            {  // this launch swept (claimed now - claimed before) subdomains = that / q global iterations
+                const unsigned long long claimed_now = H.stop ? H.work_resume : H.work;
+                const double its = (double)(claimed_now - claimed_before) / (double)L.q;
+                claimed_before = claimed_now;
+                if ((r = timer_collect(T, 1, its)) != BAR_OK) return r;
+            }
             if (H.diverged == 1) {
                 diverged = true;
                 break;
@@ -446,10 +504,13 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, d_hist};
                 a.frozen = mask_at(m);
                 a.tau = tau;
+                if ((r = timer_begin(T, m, st)) != BAR_OK) return r;
                 BAR_CUDA(launch_sweep(a, mode, st));
+                if ((r = timer_end(T, st)) != BAR_OK) return r;
             }
             launches += c;
             if ((r = read_state(A, st)) != BAR_OK) return r;
+            if ((r = timer_collect(T, (int64_t)H.iter, 1.0)) != BAR_OK) return r;  // H.iter: launches that ran
             chunk = std::min<int64_t>(chunk * 2, 256);
             if (H.diverged == 1) {
                 diverged = true;
@@ -492,6 +553,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         info->cta_iters_max = cta_max >= iters ? cta_max : iters;
         info->model_bytes_per_iter = model_bytes(L);
         info->kernel_launches = launches;
+        info->sweep_kernel_ms = T.ms;
+        info->sweep_kernel_iters = T.iters;
     }
     if (nonfinite) {
         set_error("non-finite b or x0");

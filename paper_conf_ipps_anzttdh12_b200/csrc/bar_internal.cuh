@@ -72,7 +72,19 @@ struct Layout {
 };
 constexpr int kGhostRanges = 4;
 
+// Device time of the sweep-kernel launches of one solve, taken with CUDA events on the
+// launching stream around each launch (the bench's live per-launch duration inside its timed
+// region). Launches queued after a stop request return at once and are not counted.
+struct KernelTimer {
+    static constexpr int kMax = 256;  // >= the largest chunk of launches between host reads
+    cudaEvent_t ev[2 * kMax] = {};
+    int64_t m[kMax] = {};             // global iteration index of recorded launch i
+    int used = 0;
+    double ms = 0.0, iters = 0.0;     // accumulated over the current solve
+};
+
 struct Workspace {
+    KernelTimer timer;
     double *xbuf = nullptr;     // n: second iterate buffer (sync modes)
     double *stage_b = nullptr;  // n: device staging of host b (end-to-end path)
     double *stage_x = nullptr;  // n: device staging of host x0/x
@@ -117,6 +129,13 @@ bar_status ensure_buf(double **p, int64_t n);
 double model_bytes(const Layout &L);
 bool use_async_multi(const Layout &L);
 bar_status read_state(bar_matrix A, cudaStream_t st);
+// KernelTimer: bracket one sweep launch of global iteration m; after the stream has synchronised,
+// add the launches with m <= bound (each worth `iters_each` global iterations) and reset.
+void timer_reset(KernelTimer &T);
+bar_status timer_begin(KernelTimer &T, int64_t m, cudaStream_t st);
+bar_status timer_end(KernelTimer &T, cudaStream_t st);
+bar_status timer_collect(KernelTimer &T, int64_t bound, double iters_each);
+void timer_free(KernelTimer &T);
 
 #define BAR_CUDA(call)                                              \
     do {                                                            \

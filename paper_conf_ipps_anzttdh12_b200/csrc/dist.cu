@@ -173,7 +173,7 @@ __global__ void k_publish(const double *__restrict__ part, double *const *__rest
     asm volatile("st.relaxed.sys.global.f64 [%0], %1;" ::"l"(dst + 1), "d"(part[1]) : "memory");
 }
 
-bar_status p2p_iteration(bar_dist D, const SweepArgs &a, bar_mode mode, cudaStream_t st) {
+bar_status p2p_iteration(bar_dist D, const SweepArgs &a, bar_mode mode, cudaStream_t st, KernelTimer *T, int64_t m) {
     const int64_t ng = D->n_glo + D->n_ghi;
     if (ng > 0) {
         int64_t blocks = (ng + 255) / 256;
@@ -182,7 +182,10 @@ bar_status p2p_iteration(bar_dist D, const SweepArgs &a, bar_mode mode, cudaStre
                                                          D->d_peer_own);
         BAR_CUDA(cudaGetLastError());
     }
+    bar_status r;
+    if (T && (r = timer_begin(*T, m, st)) != BAR_OK) return r;
     BAR_CUDA(launch_sweep(a, mode, st));
+    if (T && (r = timer_end(*T, st)) != BAR_OK) return r;
     k_publish<<<1, 32 * ((D->nranks + 31) / 32), 0, st>>>(D->part, D->d_peer_board, D->rank, D->nranks);
     BAR_CUDA(cudaGetLastError());
     // the board holds every rank's latest partial (others' possibly a few launches old)
@@ -254,6 +257,9 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
 #endif
         }
     }
+    // device time of the local sweeps of this process's first rank (bar_solve_info.sweep_kernel_*)
+    KernelTimer &T = D0->A->W.timer;
+    timer_reset(T);
     int64_t issued = 0, chunk = 8;
     int64_t iters = 0;
     double rel = 0.0;
@@ -275,7 +281,7 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                         bar_dist D = ranks[i];
                         SweepArgs a{&D->A->L, D->bbuf, own(D, D->xa), own(D, D->xa), k, D->A->W.state,
                                     D->A->W.partials, nullptr, D->part};
-                        if ((r = p2p_iteration(D, a, mode, st)) != BAR_OK) return r;
+                        if ((r = p2p_iteration(D, a, mode, st, i == 0 ? &T : nullptr, m)) != BAR_OK) return r;
                     }
                     launches += 4 * nr;
                     continue;
@@ -285,7 +291,9 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                     bar_dist D = ranks[i];
                     SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state,
                                 D->A->W.partials, nullptr, D->part};
+                    if (i == 0 && (r = timer_begin(T, m, st)) != BAR_OK) return r;
                     BAR_CUDA(launch_sweep(a, mode, st));
+                    if (i == 0 && (r = timer_end(T, st)) != BAR_OK) return r;
                 }
                 if ((r = reduce_decide(ranks, nr, false, st)) != BAR_OK) return r;
                 launches += 2 * nr;
@@ -297,6 +305,7 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                 if ((r = read_state(D0->A, st)) != BAR_OK) return r;
                 stopped = H.stop != 0;
             }
+            if ((r = timer_collect(T, (int64_t)H.iter, 1.0)) != BAR_OK) return r;
             chunk = std::min<int64_t>(chunk * 2, 256);
         }
         if (stopped && mode != BAR_MODE_ASYNC) {
@@ -352,6 +361,8 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
         for (int i = 0; i < nr; ++i) mb += model_bytes(ranks[i]->A->L);
         info->model_bytes_per_iter = mb;
         info->kernel_launches = launches;
+        info->sweep_kernel_ms = T.ms;
+        info->sweep_kernel_iters = T.iters;
     }
     if (diverged) {
         set_error("relative residual became non-finite or exceeded 1e30");
