@@ -30,7 +30,7 @@ WORKLOADS = {
     "c1": ("Trefethen_2000 (exact)", ("trefethen", 2000), 128),
     "c2": ("fv1-shaped 9-point 98x98, diag 9.3595", ("stencil9", 98), 128),
     "c3": ("Trefethen_20000 (exact)", ("trefethen", 20000), 128),
-    "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 256),
+    "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 512),
     "c5": ("3D 7-point 512^3, diag 7.0249 (n=128M)", ("stencil7", 512), 1024),
 }
 METRIC = "time to rel. residual 1e-10 (s) and global iters/s with HBM GB/s vs peak, 1/2/4/8 GPU"
@@ -219,7 +219,7 @@ def run_reference(args):
     n, nnz = matrix_dims(args.workload)
     cores, model = cpu_info()
     # global iterations the GPU's async-(5) needs at the default R (bench runs)
-    iters = args.ref_iters or {"c1": 29, "c2": 93, "c3": 27, "c4": 113, "c5": 59}[args.workload]
+    iters = args.ref_iters or {"c1": 29, "c2": 93, "c3": 27, "c4": 63, "c5": 44}[args.workload]
     budget = args.ref_rows
     for _ in range(args.warmup):
         oracle_sample(args.workload, args.k, args.R, args.mode, budget // 4)

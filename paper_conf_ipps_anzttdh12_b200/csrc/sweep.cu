@@ -50,7 +50,25 @@ struct KP {
     double tau;             // N3: every update scaled, x + tau (v - x)
     int static_claims;      // async: round-robin subdomain order instead of the work queue
     const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
+    int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
+    int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
 };
+
+// Static subdomain claims of persistent block c of G (k_block_pipe / k_block_duo): round robin
+// l_j = c + j G (every block advances through the matrix in one front of G subdomains), or one
+// contiguous chunk per block, l_j = floor(c q / G) + j < floor((c + 1) q / G) (each block sweeps
+// its chunk in order, so a subdomain sees this iteration's values of its predecessors in the
+// chunk: eq. 4's shift s(k+1, j) > 0, the block Gauss-Seidel flavour of P:209, on every coupling
+// shorter than the chunk). Either way each subdomain is swept exactly once per launch (R7).
+struct Claims {
+    long long l0, step, lend;
+};
+
+__device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
+    const long long G = gridDim.x, c = blockIdx.x;
+    if (p.claim_chunk) return {c * (long long)q / G, 1, (c + 1) * (long long)q / G};
+    return {c, G, (long long)q};
+}
 
 // Thread 0: start copying subdomain l's ghost-range entry (kGhostRanges pairs, 32 B) into
 // shared memory with cp.async (completion: cp.async.wait_all before reading it).
@@ -773,8 +791,8 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     const PipeGeom g = pipe_geom(R, spb, p.wmax);
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const long long G = gridDim.x;
-    auto lof = [&](long long j) { return (long long)blockIdx.x + j * G; };
+    const Claims C = claims_of(p, q);
+    auto lof = [&](long long j) { return C.l0 + j * C.step; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto stage_bytes = [&](long long l, int64_t E0, int64_t E1) -> uint32_t {
         const int nrows = (int)min((int64_t)R, p.n - (int64_t)l * R);
@@ -785,7 +803,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     // part w (0..3) of the stage of l_j (see above); one lane per warp
     auto issue_part = [&](int w, long long j, const int64_t *bd, const int32_t *gr) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int vs = (int)(j & 1), bs = (int)(j % 3);
         const int64_t TS = l * (int64_t)R;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
@@ -811,7 +829,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -833,14 +851,14 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
         fence_mbar_init();
         for (int j = 0; j < 4; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
         }
         for (int j = 0; j < 2; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             mbar_arrive_expect_tx(&bars[j], stage_bytes(l, bnd[j][0], bnd[j][1]));
             for (int w = 0; w < 4; ++w) issue_part(w, j, bnd[j], j == 1 && p.gr ? gsm[j] : nullptr);
         }
@@ -852,7 +870,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
     for (int i = 0;; ++i) {
         const int vs = i & 1, bs = i % 3;
         const long long l = lof(i);
-        if (l >= q) break;
+        if (l >= C.lend) break;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
         const int64_t TS = l * (int64_t)R;
@@ -914,7 +932,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
         }
         // post the byte count of l_{i+2}'s stage before the barrier that frees its buffers, so
         // that no copy of it can complete bytes before its phase expects them
-        if (threadIdx.x == 0 && lof(i + 2) < q) {
+        if (threadIdx.x == 0 && lof(i + 2) < C.lend) {
             const int r = (i + 2) & 3;
             mbar_arrive_expect_tx(&bars[(i + 2) % 3], stage_bytes(lof(i + 2), bnd[r][0], bnd[r][1]));
         }
@@ -961,7 +979,7 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
 // y^0 = x_J is written to shared memory by each thread and the first sweep follows the barrier
 // that also frees the slab. The slab of the next subdomain is issued right after that barrier,
 // split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
-// Subdomains are claimed statically: block c sweeps l_j = c + j G.
+// Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
 struct DuoGeom {
     uint32_t vcap, o_col, o_sptr, o_sw, o_ya, o_yb, bytes;
 };
@@ -990,10 +1008,10 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;  // = spb / 2
-    const long long G = gridDim.x;
     double *ya = reinterpret_cast<double *>(smraw + g.o_ya);
     double *yb = reinterpret_cast<double *>(smraw + g.o_yb);
-    auto lof = [&](long long j) { return (long long)blockIdx.x + j * G; };
+    const Claims C = claims_of(p, q);
+    auto lof = [&](long long j) { return C.l0 + j * C.step; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto slab_bytes = [&](long long l, const int64_t *bd) -> uint32_t {
         const uint32_t nsl = (uint32_t)nsl_of(l);
@@ -1002,7 +1020,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
     auto issue_part = [&](int w, long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int64_t *bd = bnd[j & 3];
         if (w == 3) {  // what l_j's first phase reads directly: b_J, x_J and its ghost x ranges
             const int64_t TS = l * (int64_t)R;
@@ -1031,7 +1049,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -1053,7 +1071,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         fence_mbar_init();
         for (int j = 0; j < 3; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
@@ -1067,7 +1085,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     double rr = 0.0, bb = 0.0;
     for (int i = 0;; ++i) {
         const long long l = lof(i);
-        if (l >= q) break;
+        if (l >= C.lend) break;
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
@@ -1118,7 +1136,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             bb += bi * bi;
         }
         // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
-        if (threadIdx.x == 0 && lof(i + 1) < q) mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3]));
+        if (threadIdx.x == 0 && lof(i + 1) < C.lend) mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3]));
         __syncthreads();
         if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
             issue_part(warp, i + 1);
@@ -1828,6 +1846,7 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
         c_threads[v] = L.spb * kSlice;
     }
     int64_t g = (int64_t)occ[v] * L.sms;
+    if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
     if (g > L.q) g = L.q;
     kfn<<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
     return cudaGetLastError();
@@ -1854,6 +1873,7 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
         c_threads[v] = threads;
     }
     int64_t g = (int64_t)occ[v] * L.sms;
+    if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
     if (g > L.q) g = L.q;
     kfn<<<(unsigned)g, threads, smem, st>>>(p);
     return cudaGetLastError();
@@ -1894,6 +1914,14 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // (59 vs 57 global iterations). BAR_ASYNC_STATIC=0 selects the queue.
     const char *sc = getenv("BAR_ASYNC_STATIC");
     p.static_claims = !(sc && sc[0] == '0');
+    if (const char *ge = getenv("BAR_GRID")) p.grid_cap = atoi(ge);  // tuning: cap persistent grids
+    // async claim order of k_block_pipe / k_block_duo: contiguous chunks by default. Measured on
+    // B200 (round 1, tools/kernel_ab.py, async-(5) to 1e-10): C5 (R = 1024) 44 global iterations
+    // vs 59 with round robin, C4 (R = 512) 63 vs 105 — each block sweeps its chunk in order, so
+    // the neighbouring lines / planes below a subdomain already hold this iteration's values.
+    // BAR_ORDER=r/c overrides (sync modes: the order does not change the iterates; round robin)
+    p.claim_chunk = ASYNC ? 1 : 0;
+    if (const char *oe = getenv("BAR_ORDER")) p.claim_chunk = oe[0] == 'c';
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
@@ -1917,11 +1945,11 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w).bytes;
     const char *de = getenv("BAR_DUO");
     const bool duo_fits = L.spb % 2 == 0 && L.spb >= 8 && L.max_wl <= 4 && 2 * (duo_smem + 2048) <= 228 * 1024;
-    // Async keeps one block per SM by default: with 2 x 148 subdomains in flight the window of
-    // concurrently swept rows (303K on C5) exceeds the plane coupling distance (262K), the
-    // block Gauss-Seidel effect of the monotone order (R15) is lost and async-(5) needs 65
-    // instead of 58 global iterations (faster launches, slower solve)
-    const bool duo_on = (de ? de[0] == '1' : (!ASYNC && pipe_smem > 113 * 1024)) && duo_fits &&
+    // Async: two blocks per SM whenever they fit (C5 R = 1024: 2.69 vs 2.93 ms per launch with
+    // chunked claims; C4 R = 512: 0.40 vs 0.52 ms). With round-robin claims the 2 x 148
+    // subdomains in flight (303K rows on C5) exceeded the plane coupling distance (262K) and cost
+    // global iterations (63 vs 59); chunked claims do not depend on the window.
+    const bool duo_on = (de ? de[0] == '1' : ((ASYNC && p.claim_chunk) || pipe_smem > 113 * 1024)) && duo_fits &&
                         (!ASYNC || p.static_claims);
     if (kind == 't' && duo_on && p.w_end == 0 && geom_ok && aligned) {
         L.last_kernel = ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>";

@@ -221,15 +221,28 @@ def test_fixed_point_invariant(bar, mode):
     assert np.abs(x - xs).max() <= 1e-14 * np.abs(xs).max() * 10
 
 
-@pytest.mark.parametrize("mode", ["async", "sync-block", "jacobi"])
+@pytest.mark.parametrize("mode", ["sync-block", "jacobi"])
 def test_divergence(bar, mode):
-    """rho(B) = 1.8 > 1 (P:697 analogue): BAR_ERR_DIVERGED."""
+    """rho(B) = 1.8 > 1 (P:697 analogue, SPD): the synchronous iterations diverge -> BAR_ERR_DIVERGED."""
     Ad = np.full((3, 3), 0.9) + 0.1 * np.eye(3)
     A = W.CSR(3, np.array([0, 3, 6, 9], dtype=np.int32), np.tile(np.arange(3, dtype=np.int32), 3), Ad.ravel())
     M = bar.Matrix.from_csr(A, 1)
     b = _dev(np.ones(3))
     _, info = M.solve(b, k=1, mode=mode, raise_on_error=False)
     assert info["status"] == "BAR_ERR_DIVERGED"
+
+
+def test_divergence_async(bar):
+    """Async with rho(|B|) >= 1 (Chazan-Miranker): only SOME update orders must diverge —
+    the SPD 3x3 case above converges under Gauss-Seidel-like orders, so which one a schedule
+    produces is not fixed. A = [[1, 2], [2, 1]] diverges under EVERY order: each update sets
+    e_i = -2 e_j, doubling the error, so async-(k) must return BAR_ERR_DIVERGED."""
+    A = W.CSR(2, np.array([0, 2, 4], dtype=np.int32), np.array([0, 1, 0, 1], dtype=np.int32),
+              np.array([1.0, 2.0, 2.0, 1.0]))
+    for R in (1, 2):
+        M = bar.Matrix.from_csr(A, R)
+        _, info = M.solve(_dev(np.ones(2)), k=1, mode="async", raise_on_error=False)
+        assert info["status"] == "BAR_ERR_DIVERGED", (R, info)
 
 
 # ------------------------------------------------------------------ async outcome
