@@ -383,7 +383,9 @@ def main():
     t_lo = min(timed_sweeps(lo) for _ in range(3))
     t_hi = min(timed_sweeps(hi) for _ in range(3))
     kernel_ms_isolated = reduce((t_hi - t_lo) / (hi - lo), MAX)
-    kernel_name = M.info().get("last_sweep_kernel", "?") if world == 1 else "per-rank local sweep" 
+    kernel_name = M.info().get("last_sweep_kernel", "?") if world == 1 else "per-rank local sweep"
+    if world == 1:
+        minfo = M.info()
     peak, peak_src = load_peaks()
     achieved = local_bytes / (kernel_ms * 1e-3) / 1e9  # per GPU
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",

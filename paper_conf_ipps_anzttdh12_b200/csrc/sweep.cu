@@ -54,12 +54,12 @@ struct KP {
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
 };
 
-// Static subdomain claims of persistent block c of G (k_block_pipe / k_block_duo): round robin
-// l_j = c + j G (every block advances through the matrix in one front of G subdomains), or one
-// contiguous chunk per block, l_j = floor(c q / G) + j < floor((c + 1) q / G) (each block sweeps
-// its chunk in order, so a subdomain sees this iteration's values of its predecessors in the
-// chunk: eq. 4's shift s(k+1, j) > 0, the block Gauss-Seidel flavour of P:209, on every coupling
-// shorter than the chunk). Either way each subdomain is swept exactly once per launch (R7).
+// Static subdomain claims of persistent block c of G (k_block_pipe / k_block_duo), R15: round
+// robin l_j = c + j G (every block advances through the matrix in one front of G subdomains), or
+// one contiguous chunk per block, l_j = floor(c q / G) + j < floor((c + 1) q / G) (each block
+// sweeps its chunk in order, so a subdomain sees this iteration's values of its predecessors in
+// the chunk: eq. 4's shift s(k+1, j) > 0, the block Gauss-Seidel flavour of P:209, on every
+// coupling shorter than the chunk). Either way each subdomain is swept exactly once per launch (R7).
 struct Claims {
     long long l0, step, lend;
 };
@@ -810,14 +810,15 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
         fence_proxy_async_smem();
         if (w == 0) {
-            bulk_g2s(V, p.val + bd[0], (uint32_t)(bd[1] - bd[0]) * 8, &bars[bs]);
+            bulk_g2s_hint(V, p.val + bd[0], (uint32_t)(bd[1] - bd[0]) * 8, &bars[bs], policy_evict_first());
         } else if (w == 1) {
-            bulk_g2s(V + (size_t)g.vcap * 8, p.col + bd[0], (uint32_t)(bd[1] - bd[0]) * 4, &bars[bs]);
+            bulk_g2s_hint(V + (size_t)g.vcap * 8, p.col + bd[0], (uint32_t)(bd[1] - bd[0]) * 4, &bars[bs],
+                          policy_evict_first());
             if (gr) prefetch_ghost_x(p.x_in, gr, kGhostRanges);
         } else if (w == 2) {
             const uint32_t trows = (uint32_t)min((int64_t)R, p.n - TS) & ~1u;
             if (trows) {
-                bulk_g2s(B, p.b + TS, trows * 8, &bars[bs]);
+                bulk_g2s_hint(B, p.b + TS, trows * 8, &bars[bs], policy_evict_first());
                 bulk_g2s(B + g.o_x, p.x_in + TS, trows * 8, &bars[bs]);
             }
         } else {
@@ -1027,7 +1028,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             const uint32_t nrows = (uint32_t)min((int64_t)R, p.n - TS);
             const uintptr_t b0 = reinterpret_cast<uintptr_t>(p.b + TS) & ~(uintptr_t)15;
             const uintptr_t b1 = (reinterpret_cast<uintptr_t>(p.b + TS + nrows) + 15) & ~(uintptr_t)15;
-            bulk_prefetch_l2(reinterpret_cast<const void *>(b0), (uint32_t)(b1 - b0));
+            bulk_prefetch_l2_hint(reinterpret_cast<const void *>(b0), (uint32_t)(b1 - b0), policy_evict_first());
             const uintptr_t x0 = reinterpret_cast<uintptr_t>(p.x_in + TS) & ~(uintptr_t)15;
             const uintptr_t x1 = (reinterpret_cast<uintptr_t>(p.x_in + TS + nrows) + 15) & ~(uintptr_t)15;
             bulk_prefetch_l2(reinterpret_cast<const void *>(x0), (uint32_t)(x1 - x0));
@@ -1037,9 +1038,9 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         fence_proxy_async_smem();
         const uint32_t ne = (uint32_t)(bd[1] - bd[0]);
         if (w == 0) {
-            bulk_g2s(smraw, p.val + bd[0], ne * 8, &bar);
+            bulk_g2s_hint(smraw, p.val + bd[0], ne * 8, &bar, policy_evict_first());
         } else if (w == 1) {
-            bulk_g2s(smraw + g.o_col, p.col + bd[0], ne * 4, &bar);
+            bulk_g2s_hint(smraw + g.o_col, p.col + bd[0], ne * 4, &bar, policy_evict_first());
         } else {
             const uint32_t nsl = (uint32_t)nsl_of(l);
             bulk_g2s(smraw + g.o_sptr, p.sptr + l * spb, (nsl * 8 + 15) & ~15u, &bar);

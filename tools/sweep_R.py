@@ -30,14 +30,19 @@ def main():
         for k in [int(v) for v in a.k.split(",")]:
             for mode in a.modes.split(","):
                 M.solve(b, None, x, k=k, mode=mode)  # warm-up
-                torch.cuda.synchronize()
-                t0 = time.perf_counter()
-                _, info = M.solve(b, None, x, k=k, mode=mode)
-                torch.cuda.synchronize()
-                dt = time.perf_counter() - t0
+                ts, its = [], []
+                for _ in range(5):
+                    torch.cuda.synchronize()
+                    t0 = time.perf_counter()
+                    _, info = M.solve(b, None, x, k=k, mode=mode)
+                    torch.cuda.synchronize()
+                    ts.append(time.perf_counter() - t0)
+                    its.append(info["iters"])
+                dt = sorted(ts)[2]
                 print(json.dumps({"workload": a.workload, "R": R, "k": k, "mode": mode, "iters": info["iters"],
                                   "s": round(dt, 5), "ms_per_iter": round(dt / max(1, info["iters"]) * 1e3, 4),
-                                  "rel_res": info["rel_res"]}), flush=True)
+                                  "rel_res": info["rel_res"], "iters_all": its,
+                                  "kernel": M.info()["last_sweep_kernel"]}), flush=True)
         M.close()
 
 
