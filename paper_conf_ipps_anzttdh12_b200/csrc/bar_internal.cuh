@@ -68,9 +68,18 @@ struct Layout {
     // [q][kGhostRanges] (first column, count) of x ranges holding most of subdomain l's
     // off-block columns (count 0 = unused): bulk L2 prefetch targets for the a3 gathers
     int32_t *gr = nullptr;
+    // Coded columns (built when every subdomain has <= kDictMax distinct column offsets d = col - row,
+    // as stencil / FE matrices do; else NULL): codes[e] indexes the dictionary of entry e's
+    // subdomain, dict[dptr[l] .. dptr[l+1]) (16-byte padded), so a column costs 1 byte of HBM
+    // traffic instead of 4 in the kernels that read them (k_block_duo).
+    uint8_t *codes = nullptr;   // [entries]
+    int32_t *dict = nullptr;    // [dptr[q]]
+    int32_t *dptr = nullptr;    // [q + 1]
+    int64_t dict_entries = 0;
     mutable const char *last_kernel = "none";  // name of the most recently launched sweep kernel
 };
 constexpr int kGhostRanges = 4;
+constexpr int kDictMax = 256;
 
 // Device time of the sweep-kernel launches of one solve, taken with CUDA events on the
 // launching stream around each launch (the bench's live per-launch duration inside its timed

@@ -5,6 +5,9 @@
 // every timed region ("initialisation ... subtracted").
 #include <cub/cub.cuh>
 
+#include <climits>
+#include <cstdlib>
+
 #include "bar_internal.cuh"
 
 namespace bar {
@@ -199,6 +202,88 @@ __global__ void k_ghost_ranges(int64_t n, int32_t R, int64_t col_lo, int64_t col
     }
 }
 
+// Per subdomain (one block): the dictionary of its column offsets d = col - row (off-block
+// entries store global columns, local ones col - TS; padding has d = 0) and each entry's 1-byte
+// code. dcount[l] = dictionary size, or -1 if it exceeds kDictMax (then no coded layout).
+// Entries of the rows past n in the last subdomain are never read: code 0.
+constexpr int kDictSlots = 2 * kDictMax;
+__global__ void k_codes(int64_t n, int32_t R, int32_t spb, const int64_t *__restrict__ sptr,
+                        const int32_t *__restrict__ sw, const int32_t *__restrict__ col, uint8_t *__restrict__ codes,
+                        int32_t *__restrict__ dtmp, int32_t *__restrict__ dcount) {
+    __shared__ int32_t key[kDictSlots];
+    __shared__ int32_t code[kDictSlots];
+    __shared__ int overflow;
+    const int32_t kEmpty = INT32_MIN;
+    for (int t = threadIdx.x; t < kDictSlots; t += blockDim.x) key[t] = kEmpty;
+    if (threadIdx.x == 0) overflow = 0;
+    __syncthreads();
+    const int64_t l = blockIdx.x, TS = l * (int64_t)R;
+    const int nrows = (int)min((int64_t)R, n - TS);
+    const int nsl = (nrows + kSlice - 1) / kSlice;
+    auto slot_of = [&](int32_t d, bool insert) -> int {
+        int h = (int)(((uint32_t)d * 2654435761u) >> 23) & (kDictSlots - 1);  // 9 bits
+        for (int probe = 0; probe < kDictSlots; ++probe, h = (h + 1) & (kDictSlots - 1)) {
+            const int32_t k = key[h];
+            if (k == d) return h;
+            if (k == kEmpty) {
+                if (!insert) return -1;
+                const int32_t old = atomicCAS(&key[h], kEmpty, d);
+                if (old == kEmpty || old == d) return h;
+            }
+        }
+        return -1;
+    };
+    for (int pass = 0; pass < 2; ++pass) {
+        for (int j = 0; j < nsl; ++j) {
+            const int64_t s = l * spb + j, E = sptr[s];
+            const int wl = sw[s] & 0xffff, wo = sw[s] >> 16;
+            for (int t = threadIdx.x; t < kSlice * (wl + wo); t += blockDim.x) {
+                const int lane = t & (kSlice - 1), e = t / kSlice, loc = j * kSlice + lane;
+                if (loc >= nrows) {
+                    if (pass == 1) codes[E + t] = 0;
+                    continue;
+                }
+                const int32_t c = col[E + t];
+                const int32_t d = e < wo ? (int32_t)(c - (TS + loc)) : c - loc;
+                const int h = slot_of(d, pass == 0);
+                if (h < 0) {
+                    overflow = 1;
+                    continue;
+                }
+                if (pass == 1) codes[E + t] = (uint8_t)code[h];
+            }
+        }
+        __syncthreads();
+        if (pass == 0 && threadIdx.x == 0) {
+            int cnt = 0;
+            for (int h = 0; h < kDictSlots; ++h) {
+                if (key[h] == kEmpty) continue;
+                if (cnt < kDictMax) dtmp[l * kDictMax + cnt] = key[h];
+                code[h] = cnt++;
+            }
+            if (cnt == 0) dtmp[l * kDictMax + cnt++] = 0;
+            if (cnt > kDictMax) overflow = 1;
+            dcount[l] = overflow ? -1 : cnt;
+        }
+        __syncthreads();
+        if (overflow) return;
+    }
+}
+
+// Padded dictionary sizes (multiples of 4 int32 = 16 bytes, the bulk-copy granule).
+__global__ void k_dict_pad(int64_t q, const int32_t *__restrict__ dcount, int32_t *__restrict__ dsize) {
+    const int64_t l = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (l < q) dsize[l] = (dcount[l] + 3) & ~3;
+    if (l == q) dsize[l] = 0;
+}
+
+__global__ void k_dict_compact(int64_t q, const int32_t *__restrict__ dtmp, const int32_t *__restrict__ dcount,
+                               const int32_t *__restrict__ dptr, int32_t *__restrict__ dict) {
+    const int64_t l = blockIdx.x;
+    const int cnt = dcount[l], sz = dptr[l + 1] - dptr[l];
+    for (int c = threadIdx.x; c < sz; c += blockDim.x) dict[dptr[l] + c] = c < cnt ? dtmp[l * kDictMax + c] : 0;
+}
+
 template <class T>
 cudaError_t dmalloc(T **p, size_t count) {
     return cudaMalloc((void **)p, sizeof(T) * (count ? count : 1));
@@ -217,6 +302,70 @@ void free_layout(Layout &L) {
     L.sw = nullptr;
     cudaFree(L.gr);
     L.gr = nullptr;
+    cudaFree(L.codes);
+    cudaFree(L.dict);
+    cudaFree(L.dptr);
+    L.codes = nullptr;
+    L.dict = nullptr;
+    L.dptr = nullptr;
+    L.dict_entries = 0;
+}
+
+// Coded columns (Layout::codes); leaves them NULL when a subdomain has more than kDictMax
+// distinct offsets or memory is short (the kernels then read the int32 columns).
+static void build_codes(Layout &L, cudaStream_t st) {
+    const int64_t q = L.q;
+    int32_t *dtmp = nullptr, *dcount = nullptr, *dsize = nullptr;
+    void *tmp = nullptr;
+    size_t tb = 0;
+    int32_t mn = 0, total = 0;
+    bool ok = false;
+    if (cudaMalloc(&L.codes, (size_t)L.entries + 16) != cudaSuccess ||
+        cudaMalloc(&dtmp, sizeof(int32_t) * (size_t)q * kDictMax) != cudaSuccess ||
+        cudaMalloc(&dcount, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess ||
+        cudaMalloc(&dsize, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess ||
+        cudaMalloc(&L.dptr, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess)
+        goto out;
+    k_codes<<<(unsigned)q, 256, 0, st>>>(L.n, L.R, L.spb, L.sptr, L.sw, L.col, L.codes, dtmp, dcount);
+    if (cub::DeviceReduce::Min(nullptr, tb, dcount, dsize + q, q, st) != cudaSuccess) goto out;
+    {
+        size_t tb2 = 0;
+        if (cub::DeviceScan::ExclusiveSum(nullptr, tb2, dsize, L.dptr, q + 1, st) != cudaSuccess) goto out;
+        if (tb2 > tb) tb = tb2;
+    }
+    if (cudaMalloc(&tmp, tb) != cudaSuccess) goto out;
+    {
+        size_t t = tb;
+        if (cub::DeviceReduce::Min(tmp, t, dcount, dsize + q, q, st) != cudaSuccess) goto out;
+        if (cudaMemcpyAsync(&mn, dsize + q, sizeof(int32_t), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+            cudaStreamSynchronize(st) != cudaSuccess || mn < 1)
+            goto out;
+        k_dict_pad<<<(unsigned)((q + 1 + 255) / 256), 256, 0, st>>>(q, dcount, dsize);
+        t = tb;
+        if (cub::DeviceScan::ExclusiveSum(tmp, t, dsize, L.dptr, q + 1, st) != cudaSuccess) goto out;
+        if (cudaMemcpyAsync(&total, L.dptr + q, sizeof(int32_t), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+            cudaStreamSynchronize(st) != cudaSuccess)
+            goto out;
+    }
+    if (cudaMalloc(&L.dict, sizeof(int32_t) * (size_t)(total + 4)) != cudaSuccess) goto out;
+    k_dict_compact<<<(unsigned)q, 64, 0, st>>>(q, dtmp, dcount, L.dptr, L.dict);
+    ok = cudaStreamSynchronize(st) == cudaSuccess && cudaGetLastError() == cudaSuccess;
+    L.dict_entries = total;
+out:
+    cudaGetLastError();
+    cudaFree(dtmp);
+    cudaFree(dcount);
+    cudaFree(dsize);
+    cudaFree(tmp);
+    if (!ok) {
+        cudaFree(L.codes);
+        cudaFree(L.dict);
+        cudaFree(L.dptr);
+        L.codes = nullptr;
+        L.dict = nullptr;
+        L.dptr = nullptr;
+        L.dict_entries = 0;
+    }
 }
 
 static bar_status alloc_fail(cudaError_t e, const char *what) {
@@ -347,6 +496,7 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     k_ghost_ranges<<<(unsigned)L.q, 256, 0, st>>>(n, R, col_lo, col_hi, d_rowptr, d_col, L.gr);
     BAR_CK(cudaGetLastError());
     BAR_CK(cudaStreamSynchronize(st));
+    if (!getenv("BAR_NO_CODES")) build_codes(L, st);
 
 done:
     cudaFree(nloc);

@@ -52,6 +52,9 @@ struct KP {
     const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
     int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
+    const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
+    const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
+    const int32_t *dptr;
 };
 
 // Static subdomain claims of persistent block c of G (k_block_pipe / k_block_duo), R15: round
@@ -982,14 +985,17 @@ __global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
 // split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
 // Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
 struct DuoGeom {
-    uint32_t vcap, o_col, o_sptr, o_sw, o_ya, o_yb, bytes;
+    uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, bytes;
 };
 
-__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax) {
+// CODED: the column block holds 1-byte codes and is followed by the subdomain's dictionary
+// (<= kDictMax int32 offsets); otherwise int32 columns.
+__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, bool coded = false) {
     DuoGeom g;
     g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
     g.o_col = g.vcap * 8;
-    g.o_sptr = (g.o_col + g.vcap * 4 + 15) & ~15u;
+    g.o_dict = (g.o_col + g.vcap * (coded ? 1 : 4) + 15) & ~15u;
+    g.o_sptr = (g.o_dict + (coded ? kDictMax * 4 : 0) + 15) & ~15u;
     g.o_sw = g.o_sptr + (((uint32_t)spb * 8 + 15) & ~15u);
     g.o_ya = (g.o_sw + (((uint32_t)spb * 4 + 15) & ~15u) + 127) & ~127u;
     g.o_yb = g.o_ya + (uint32_t)R * 8;
@@ -997,15 +1003,16 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax) {
     return g;
 }
 
-template <bool ASYNC, int WLR, bool EXT = false>
+template <bool ASYNC, int WLR, bool EXT = false, bool CODED = false>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bar;
     __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
     __shared__ __align__(16) int32_t gsm[4][2 * kGhostRanges];  // [j % 4]: ghost ranges of l_j
+    __shared__ __align__(16) int32_t dbd[4][2];                 // [j % 4]: dictionary D0, D1 (CODED)
     const int R = p.R, spb = p.spb;
-    const DuoGeom g = duo_geom(R, spb, p.wmax);
+    const DuoGeom g = duo_geom(R, spb, p.wmax, CODED);
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;  // = spb / 2
@@ -1014,9 +1021,11 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     const Claims C = claims_of(p, q);
     auto lof = [&](long long j) { return C.l0 + j * C.step; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
-    auto slab_bytes = [&](long long l, const int64_t *bd) -> uint32_t {
+    auto slab_bytes = [&](long long l, const int64_t *bd, const int32_t *db) -> uint32_t {
         const uint32_t nsl = (uint32_t)nsl_of(l);
-        return (uint32_t)(bd[1] - bd[0]) * 12 + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u);
+        const uint32_t colb = CODED ? (uint32_t)(bd[1] - bd[0]) + (uint32_t)(db[1] - db[0]) * 4
+                                    : (uint32_t)(bd[1] - bd[0]) * 4;
+        return (uint32_t)(bd[1] - bd[0]) * 8 + colb + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u);
     };
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
     auto issue_part = [&](int w, long long j) {
@@ -1040,7 +1049,13 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         if (w == 0) {
             bulk_g2s_hint(smraw, p.val + bd[0], ne * 8, &bar, policy_evict_first());
         } else if (w == 1) {
-            bulk_g2s_hint(smraw + g.o_col, p.col + bd[0], ne * 4, &bar, policy_evict_first());
+            if (CODED) {
+                const int32_t *db = dbd[j & 3];
+                bulk_g2s_hint(smraw + g.o_col, p.codes + bd[0], ne, &bar, policy_evict_first());
+                bulk_g2s(smraw + g.o_dict, p.dict + db[0], (uint32_t)(db[1] - db[0]) * 4, &bar);
+            } else {
+                bulk_g2s_hint(smraw + g.o_col, p.col + bd[0], ne * 4, &bar, policy_evict_first());
+            }
         } else {
             const uint32_t nsl = (uint32_t)nsl_of(l);
             bulk_g2s(smraw + g.o_sptr, p.sptr + l * spb, (nsl * 8 + 15) & ~15u, &bar);
@@ -1065,6 +1080,12 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                          "l"(p.gr + 2 * l * kGhostRanges + 4)
                          : "memory");
         }
+        if (CODED) {
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(&dbd[r][0])), "l"(p.dptr + l)
+                         : "memory");
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(&dbd[r][1])), "l"(p.dptr + l + 1)
+                         : "memory");
+        }
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
     if (threadIdx.x == 0) {  // prologue: ring slots of l_0 .. l_2, the slab of l_0
@@ -1076,8 +1097,12 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
+            if (CODED) {
+                dbd[j][0] = p.dptr[l];
+                dbd[j][1] = p.dptr[l + 1];
+            }
         }
-        mbar_arrive_expect_tx(&bar, slab_bytes(lof(0), bnd[0]));
+        mbar_arrive_expect_tx(&bar, slab_bytes(lof(0), bnd[0], dbd[0]));
         for (int w = 0; w < 4; ++w) issue_part(w, 0);
     }
     __syncthreads();
@@ -1114,6 +1139,11 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             const int64_t off = ssp[sl] - ssp[0] + lane;
             const double *sv = reinterpret_cast<const double *>(smraw) + off;
             const int32_t *sc = reinterpret_cast<const int32_t *>(smraw + g.o_col) + off;
+            const uint8_t *s8 = reinterpret_cast<const uint8_t *>(smraw + g.o_col) + off;
+            const int32_t *dic = reinterpret_cast<const int32_t *>(smraw + g.o_dict);
+            // column of stored entry e: global for off-block entries, local index for local ones
+            auto gcol = [&](int e) -> int64_t { return CODED ? TS + loc + dic[s8[e * kSlice]] : sc[e * kSlice]; };
+            auto lcol = [&](int e) -> uint32_t { return CODED ? (uint32_t)(loc + dic[s8[e * kSlice]]) : (uint32_t)sc[e * kSlice]; };
             const double bi = p.b[TS + loc];
             ya[loc] = ldx<ASYNC>(p.x_in + TS + loc);
             double acc = bi;
@@ -1121,7 +1151,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 double xv[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + sc[(e0 + u) * kSlice]);
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + gcol(e0 + u));
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
@@ -1131,13 +1161,14 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             for (int e = 0; e < WLR; ++e) {
                 if (e < wl) {
                     lv[h][e] = sv[(wo + e) * kSlice];
-                    lc[h][e >> 1] |= (uint32_t)sc[(wo + e) * kSlice] << (16 * (e & 1));
+                    lc[h][e >> 1] |= lcol(wo + e) << (16 * (e & 1));
                 }
             }
             bb += bi * bi;
         }
         // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
-        if (threadIdx.x == 0 && lof(i + 1) < C.lend) mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3]));
+        if (threadIdx.x == 0 && lof(i + 1) < C.lend)
+            mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3], dbd[(i + 1) & 3]));
         __syncthreads();
         if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
             issue_part(warp, i + 1);
@@ -1856,11 +1887,13 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
 template <bool ASYNC, int WLR>
 cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
-    auto kfn = ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>;
-    static size_t attr[2] = {0, 0};
-    static size_t c_smem[2] = {0, 0};
-    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
-    const int v = ext ? 1 : 0;
+    const bool coded = p.codes != nullptr;
+    auto kfn = coded ? (ext ? k_block_duo<ASYNC, WLR, true, true> : k_block_duo<ASYNC, WLR, false, true>)
+                     : (ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>);
+    static size_t attr[4] = {0, 0, 0, 0};
+    static size_t c_smem[4] = {0, 0, 0, 0};
+    static int c_threads[4] = {0, 0, 0, 0}, occ[4] = {0, 0, 0, 0};
+    const int v = (ext ? 1 : 0) + (coded ? 2 : 0);
     const int threads = L.spb / 2 * kSlice;
     if (smem > attr[v]) {
         cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1943,7 +1976,11 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // two-blocks-per-SM variant (k_block_duo) where the pipelined kernel holds a whole SM (C5
     // sync modes, B200 round 1, tools/kernel_ab.py: Jacobi 2.45 vs 2.58 ms, sync-block-(5) 2.56-2.67
     // vs 2.67 ms per launch); BAR_DUO=0/1 overrides
-    const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w).bytes;
+    // coded columns (Layout::codes, 1 byte per entry instead of 4) for the duo kernel when the
+    // layout has them; BAR_CODED=0 reads the int32 columns instead
+    const char *ce = getenv("BAR_CODED");
+    const bool coded = L.codes != nullptr && !(ce && ce[0] == '0');
+    const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w, coded).bytes;
     const char *de = getenv("BAR_DUO");
     const bool duo_fits = L.spb % 2 == 0 && L.spb >= 8 && L.max_wl <= 4 && 2 * (duo_smem + 2048) <= 228 * 1024;
     // Async: two blocks per SM whenever they fit (C5 R = 1024: 2.69 vs 2.93 ms per launch with
@@ -1953,8 +1990,15 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const bool duo_on = (de ? de[0] == '1' : ((ASYNC && p.claim_chunk) || pipe_smem > 113 * 1024)) && duo_fits &&
                         (!ASYNC || p.static_claims);
     if (kind == 't' && duo_on && p.w_end == 0 && geom_ok && aligned) {
-        L.last_kernel = ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>";
-        return launch_duo_t<ASYNC, 4>(p, L, duo_smem, st);  // two rows per thread: <= 4 local entries
+        L.last_kernel = coded ? (ASYNC ? "k_block_duo<async,coded>" : "k_block_duo<sync,coded>")
+                              : (ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>");
+        KP pc = p;
+        if (coded) {
+            pc.codes = L.codes;
+            pc.dict = L.dict;
+            pc.dptr = L.dptr;
+        }
+        return launch_duo_t<ASYNC, 4>(pc, L, duo_smem, st);  // two rows per thread: <= 4 local entries
     }
     if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
         L.last_kernel = ASYNC ? "k_block_pipe<async>" : "k_block_pipe<sync>";
