@@ -1130,20 +1130,20 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         // a2/a3: b_i and x_i (direct, L2-prefetched; x_i -> y^0), the off-block part with x as
         // it stands, the local entries into registers
         const int64_t *ssp = reinterpret_cast<const int64_t *>(smraw + g.o_sptr);
+        const uint32_t sb = smem_u32(smraw);
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
             const int sl = warp + h * nw, loc = row_of(h);
             if (sl >= nsl || loc >= nrows) continue;
-            const int sw = reinterpret_cast<const int32_t *>(smraw + g.o_sw)[sl];
+            const int sw = lds_s32(sb + g.o_sw + 4 * sl);
             const int wl = sw & 0xffff, wo = sw >> 16;
-            const int64_t off = ssp[sl] - ssp[0] + lane;
-            const double *sv = reinterpret_cast<const double *>(smraw) + off;
-            const int32_t *sc = reinterpret_cast<const int32_t *>(smraw + g.o_col) + off;
-            const uint8_t *s8 = reinterpret_cast<const uint8_t *>(smraw + g.o_col) + off;
-            const int32_t *dic = reinterpret_cast<const int32_t *>(smraw + g.o_dict);
-            // column of stored entry e: global for off-block entries, local index for local ones
-            auto gcol = [&](int e) -> int64_t { return CODED ? TS + loc + dic[s8[e * kSlice]] : sc[e * kSlice]; };
-            auto lcol = [&](int e) -> uint32_t { return CODED ? (uint32_t)(loc + dic[s8[e * kSlice]]) : (uint32_t)sc[e * kSlice]; };
+            const uint32_t off = (uint32_t)(ssp[sl] - ssp[0]) + lane;
+            const uint32_t av = sb + off * 8, ac = sb + g.o_col + off * (CODED ? 1 : 4), ad = sb + g.o_dict;
+            // stored column of entry e: global for off-block entries, local index for local ones
+            // (CODED: the offset d = col - row from the subdomain's dictionary)
+            auto dcol = [&](int e) -> int32_t {
+                return CODED ? lds_s32(ad + 4 * lds_u8(ac + e * kSlice)) : lds_s32(ac + e * kSlice * 4);
+            };
             const double bi = p.b[TS + loc];
             ya[loc] = ldx<ASYNC>(p.x_in + TS + loc);
             double acc = bi;
@@ -1151,17 +1151,17 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 double xv[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + gcol(e0 + u));
+                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + (CODED ? TS + loc : 0) + dcol(e0 + u));
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (e0 + u < wo) acc -= sv[(e0 + u) * kSlice] * xv[u];
+                    if (e0 + u < wo) acc -= lds_f64(av + (e0 + u) * kSlice * 8) * xv[u];
             }
             s[h] = acc;
 #pragma unroll
             for (int e = 0; e < WLR; ++e) {
                 if (e < wl) {
-                    lv[h][e] = sv[(wo + e) * kSlice];
-                    lc[h][e >> 1] |= lcol(wo + e) << (16 * (e & 1));
+                    lv[h][e] = lds_f64(av + (wo + e) * kSlice * 8);
+                    lc[h][e >> 1] |= (uint32_t)((CODED ? loc : 0) + dcol(wo + e)) << (16 * (e & 1));
                 }
             }
             bb += bi * bi;

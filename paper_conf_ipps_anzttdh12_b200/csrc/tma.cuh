@@ -61,6 +61,24 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         : "memory");
 }
 
+// Shared-memory loads by 32-bit shared-window address (hoisted base + offsets: no generic-to-shared
+// conversion per access inside branchy per-entry code).
+__device__ __forceinline__ double lds_f64(uint32_t a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ int32_t lds_s32(uint32_t a) {
+    int32_t v;
+    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
+    uint16_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=h"(v) : "r"(a));
+    return v;
+}
+
 // L2 eviction policies for the streaming kernels (createpolicy; used as .L2::cache_hint operands).
 // The matrix slab and b are read once per global iteration and never again within it: evict them
 // first, so that L2 keeps the iterate x between the reads of one subdomain's values as its own
