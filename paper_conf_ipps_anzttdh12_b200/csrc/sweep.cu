@@ -1157,12 +1157,15 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                     if (e0 + u < wo) acc -= lds_f64(av + (e0 + u) * kSlice * 8) * xv[u];
             }
             s[h] = acc;
+            // local entries, branch-free: slots past wl read in-bounds shared memory (the regions
+            // after the slab) and are zeroed (value 0, column 0)
 #pragma unroll
             for (int e = 0; e < WLR; ++e) {
-                if (e < wl) {
-                    lv[h][e] = lds_f64(av + (wo + e) * kSlice * 8);
-                    lc[h][e >> 1] |= (uint32_t)((CODED ? loc : 0) + dcol(wo + e)) << (16 * (e & 1));
-                }
+                const bool ok = e < wl;
+                const double v = lds_f64(av + (wo + e) * kSlice * 8);
+                const uint32_t c = (uint32_t)((CODED ? loc : 0) + dcol(wo + e)) & 0xffffu;
+                lv[h][e] = ok ? v : 0.0;
+                lc[h][e >> 1] |= (ok ? c : 0u) << (16 * (e & 1));
             }
             bb += bi * bi;
         }
