@@ -397,10 +397,19 @@ def main():
                 "kernel_ms_isolated": round(kernel_ms_isolated, 5),
                 "frac_isolated": round(local_bytes / (kernel_ms_isolated * 1e-3) / 1e9 / peak, 4),
                 "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
+    # the layout's own compulsory bytes (coded columns move 1 B per entry instead of the contract's
+    # 4) and, from the committed ncu capture of the same kernel, the DRAM bytes one launch moved
+    if world == 1:
+        lb = M.info()["layout_bytes_per_iter"]
+        roofline["layout_bytes_per_launch"] = lb
+        roofline["frac_layout"] = round(lb / (kernel_ms * 1e-3) / 1e9 / peak, 4)
     prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")
     if world == 1 and os.path.exists(prof):
         try:
-            roofline["traffic"] = json.load(open(prof))["dram_bytes_per_launch"]
+            tj = json.load(open(prof))
+            if tj.get("kernel", kernel_name) == kernel_name:
+                roofline["traffic"] = tj["dram_bytes_per_launch"]
+                roofline["frac_dram"] = round(tj["dram_bytes_per_launch"] / (kernel_ms * 1e-3) / 1e9 / peak, 4)
         except Exception:
             pass
 

@@ -92,6 +92,12 @@ typedef struct {
     const char *last_sweep_kernel; /* static name of the sweep kernel the latest bar_solve /
                                       bar_sweep launch on this handle used ("none" before any);
                                       a diagnostic for profiling and the bench's roofline line  */
+    int32_t coded;                /* 1: the layout also holds 1-byte column codes + per-subdomain
+                                     offset dictionaries (read by the two-blocks-per-SM sweep)   */
+    double layout_bytes_per_iter; /* compulsory HBM bytes of one sweep of THIS layout: values (8 B),
+                                     columns (1 B coded / 4 B) per stored entry incl. padding,
+                                     b + x read + x write (24 B) per row, slice metadata and
+                                     dictionaries (excludes re-reads of off-block x)            */
 } bar_matrix_info;
 
 /*

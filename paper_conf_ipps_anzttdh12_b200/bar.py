@@ -56,7 +56,8 @@ class MatrixInfo(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("rows_per_block", ctypes.c_int32),
                 ("num_subdomains", ctypes.c_int64), ("layout_entries", ctypes.c_int64),
                 ("local_entries", ctypes.c_int64), ("model_bytes_per_iter", ctypes.c_double),
-                ("device", ctypes.c_int32), ("last_sweep_kernel", ctypes.c_char_p)]
+                ("device", ctypes.c_int32), ("last_sweep_kernel", ctypes.c_char_p), ("coded", ctypes.c_int32),
+                ("layout_bytes_per_iter", ctypes.c_double)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}

@@ -230,6 +230,9 @@ bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info) {
     info->model_bytes_per_iter = model_bytes(L);
     info->device = A->device;
     info->last_sweep_kernel = L.last_kernel;
+    info->coded = L.codes != nullptr;
+    info->layout_bytes_per_iter = (double)L.entries * (8 + (L.codes ? 1 : 4)) + (double)L.n * 24 +
+                                  (double)L.nslices * 12 + (L.codes ? (double)L.dict_entries * 4 + (double)L.q * 4 : 0.0);
     return BAR_OK;
 }
 

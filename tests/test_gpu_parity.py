@@ -299,7 +299,8 @@ def test_forced_kernel_paths(bar, monkeypatch, env, name, R):
 
 
 # ------------------------------------------------------------------ pipelined / two-blocks-per-SM
-@pytest.mark.parametrize("env", [{"BAR_DUO": "1"}, {"BAR_DUO": "0"}, {"BAR_DUO": "0", "BAR_PIPE": "0"}])
+@pytest.mark.parametrize("env", [{"BAR_DUO": "1"}, {"BAR_DUO": "0"}, {"BAR_DUO": "0", "BAR_PIPE": "0"},
+                                 {"BAR_DUO": "1", "BAR_CODED": "0"}, {"BAR_ORDER": "r"}, {"BAR_ORDER": "c"}])
 def test_large_subdomain_kernels(bar, monkeypatch, env):
     """C5's shape at a testable size: 3D 7-point, m = 128, R = 256 = two grid lines (so a row has
     at most 4 local entries, as at 512^3 with R = 1024). The two-blocks-per-SM kernel
@@ -319,3 +320,28 @@ def test_large_subdomain_kernels(bar, monkeypatch, env):
         _close(x, ref)
     x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10)
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+def test_coded_columns(bar, monkeypatch):
+    """Coded columns (1-byte codes into per-subdomain offset dictionaries) are built for stencils
+    and give bitwise the int32-column iterates; matrices with more than 256 distinct column offsets
+    in a subdomain keep the int32 columns only (and still match the oracle)."""
+    A = W.stencil7_3d(128)  # R = two grid lines: <= 4 local entries per row, the duo kernel applies
+    R = 256
+    M = bar.Matrix.from_csr(A, R)
+    assert M.info()["coded"] == 1
+    assert M.info()["layout_bytes_per_iter"] < M.info()["model_bytes_per_iter"]
+    b = _dev(np.ones(A.n))
+    x0 = _dev(np.random.default_rng(9).uniform(-1, 1, A.n))
+    out = {}
+    for coded in ("1", "0"):
+        monkeypatch.setenv("BAR_CODED", coded)
+        for mode, k in (("sync-block", 5), ("jacobi", 1)):
+            x, info = M.solve(b, x0, k=k, max_global_iters=4, tol=0.0, mode=mode)
+            out[coded, mode] = x.cpu().numpy()
+            assert ("coded" in M.info()["last_sweep_kernel"]) == (coded == "1")
+    for mode in ("sync-block", "jacobi"):
+        assert np.array_equal(out["1", mode], out["0", mode])
+    R = W.random_dd(4096, nnz_per_row=7, seed=3)
+    MR = bar.Matrix.from_csr(R, 1024)
+    assert MR.info()["coded"] == 0
