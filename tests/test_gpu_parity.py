@@ -334,6 +334,7 @@ def test_coded_columns(bar, monkeypatch):
     b = _dev(np.ones(A.n))
     x0 = _dev(np.random.default_rng(9).uniform(-1, 1, A.n))
     out = {}
+    monkeypatch.setenv("BAR_DUO", "1")  # the sync modes pick the duo kernel only for larger slabs
     for coded in ("1", "0"):
         monkeypatch.setenv("BAR_CODED", coded)
         for mode, k in (("sync-block", 5), ("jacobi", 1)):
