@@ -28,7 +28,7 @@ sys.path.insert(0, ROOT)
 WORKLOADS = {
     # name: (description, generator kwargs, default R)
     "c1": ("Trefethen_2000 (exact)", ("trefethen", 2000), 128),
-    "c2": ("fv1-shaped 9-point 98x98, diag 9.3595", ("stencil9", 98), 128),
+    "c2": ("fv1-shaped 9-point 98x98, diag 9.3595", ("stencil9", 98), 384),
     "c3": ("Trefethen_20000 (exact)", ("trefethen", 20000), 128),
     "c4": ("2D 9-point 4000x4000, diag 9.3595 (n=16M)", ("stencil9", 4000), 512),
     "c5": ("3D 7-point 512^3, diag 7.0249 (n=128M)", ("stencil7", 512), 1024),

@@ -784,7 +784,7 @@ __host__ __device__ __forceinline__ PipeGeom pipe_geom(int R, int spb, int wmax)
 // The arrive.expect_tx of l_{i+2} is posted before the barrier that precedes every copy of
 // l_{i+2}, so no copy completes bytes before its phase expects them.
 template <bool ASYNC, int WLR, bool EXT = false>
-__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_pipe(KP p) {
+__global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_pipe(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[3];
@@ -1221,7 +1221,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
 
 // Per-launch staged sweep (one global iteration per launch).
 template <bool ASYNC, int WLR, bool EXT = false>
-__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage(KP p) {
+__global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_stage(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[2];
@@ -1411,7 +1411,7 @@ struct T0State {
 };
 
 template <bool ASYNC, int WLR, bool MULTI>
-__global__ void __launch_bounds__(WLR > 8 ? 256 : 1024, 1) k_block_stage_m(KP p) {
+__global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_stage_m(KP p) {
     if (!MULTI && *(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[2];
@@ -1926,7 +1926,7 @@ cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream
 bool staged_ok(const KP &p, const Layout &L) {
     const bool aligned = ((uintptr_t)p.b % 16 == 0) && ((uintptr_t)p.x_in % 16 == 0);
     const bool geom_ok = L.spb % 4 == 0 && L.R % 2 == 0 &&
-                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
+                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 16 && L.max_wl <= 12) || (L.spb <= 8 && L.max_wl <= 16));
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
     return aligned && geom_ok && stage_smem <= kSmemMax;
 }
@@ -1965,7 +1965,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const bool aligned = ((uintptr_t)p.b % 16 == 0) && ((uintptr_t)p.x_in % 16 == 0);
     // bulk-copy sources must be 16-byte aligned: b/x at l*R rows (R even), ptr/sw at l*spb
     const bool geom_ok = L.spb % 4 == 0 && L.R % 2 == 0 &&
-                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 8 && L.max_wl <= 16));
+                         ((L.spb <= 32 && L.max_wl <= 8) || (L.spb <= 16 && L.max_wl <= 12) || (L.spb <= 8 && L.max_wl <= 16));
     const PipeGeom pg = pipe_geom(L.R, L.spb, L.max_w);
     const size_t pipe_smem = 2 * (size_t)pg.vc_bytes + 3 * (size_t)pg.bx_bytes;
     // measured on B200 (round 1, tools/local_iters.py, kernel_ab.py): the two-ahead pipeline wins
@@ -2008,6 +2008,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);
         if (L.max_wl <= 6) return launch_pipe_t<ASYNC, 6>(p, L, pipe_smem, st);
         if (L.max_wl <= 8) return launch_pipe_t<ASYNC, 8>(p, L, pipe_smem, st);
+        if (L.max_wl <= 12) return launch_pipe_t<ASYNC, 12>(p, L, pipe_smem, st);  // <= 512 threads
         return launch_pipe_t<ASYNC, 16>(p, L, pipe_smem, st);
     }
     if (kind == 't' && geom_ok && aligned && stage_smem <= kSmemMax) {
@@ -2015,6 +2016,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
         if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
         if (L.max_wl <= 8) return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
+        if (L.max_wl <= 12) return launch_stage_t<ASYNC, 12>(p, L, stage_smem, st);  // <= 512 threads
         return launch_stage_t<ASYNC, 16>(p, L, stage_smem, st);  // <= 256 threads per block
     }
     if (p.w_end > 0) return cudaErrorNotSupported;  // no persistent multi-iteration kernel here
