@@ -457,8 +457,10 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         bool used_multi = false;
         const long long w_end = (long long)max_global_iters * (long long)L.q;
         unsigned long long claimed_before = 0;
+        long long m0 = 0;  // k_block_resident: restart iteration after a resume
         while (multi && !converged && !bzero && !diverged && max_global_iters > 0) {
             SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+            a.m0 = m0;
             if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
             cudaError_t e = launch_async_multi(a, w_end, st);
             if (e == cudaErrorNotSupported) {
@@ -489,7 +491,11 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             if (!std::isfinite(rel) || rel > 1e30) diverged = true;
             else if (rel <= tol) converged = 1;
             else if (!H.stop || (long long)H.work_resume >= w_end) break;  // max_global_iters reached
-            else BAR_CUDA(launch_resume_queue(W.state, st));
+            else {
+                const bool resident = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0;
+                m0 = H.iters_done;
+                BAR_CUDA(launch_resume_queue(W.state, st, resident));
+            }
         }
         if (used_multi) {
             // global iterations needed: the iteration whose fused estimate met tol (the returned

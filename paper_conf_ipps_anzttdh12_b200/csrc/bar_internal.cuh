@@ -171,6 +171,7 @@ struct SweepArgs {
     double *dist_out = nullptr;  // multi-GPU: receives this rank's [sum r^2, sum b^2]
     const uint8_t *frozen = nullptr;  // N1: rows that do not update in this launch (nullable)
     double tau = 1.0;                 // N3: relaxation weight, B = I - tau D^-1 A
+    long long m0 = 0;                 // single-launch async: global iteration of the first sweep
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);
@@ -188,6 +189,8 @@ cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nran
 cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
-cudaError_t launch_resume_queue(DevState *state, cudaStream_t st);  // reopen a closed async queue
+// reopen a closed async queue; clear_slots: also zero the per-iteration residual slots
+// (k_block_resident restarts every block at the last completed iteration)
+cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slots = false);
 
 }  // namespace bar

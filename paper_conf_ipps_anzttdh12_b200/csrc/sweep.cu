@@ -44,6 +44,7 @@ struct KP {
     int wlmax;
     int wmax;  // widest slice (local + off-block entries)
     long long w_end;  // async persistent: claims [0, w_end) = global iterations [0, w_end / q)
+    long long m0;     // k_block_resident: global iteration index of this launch's first sweep
     int fresh_xj;     // async persistent with q < 4 * grid: read x_J when a subdomain starts
     double *dist_out; // multi-GPU: [sum r^2, sum b^2] of this rank (no stopping decision here)
     const uint8_t *frozen;  // N1 failure injection: rows that keep their value (nullable)
@@ -1614,6 +1615,142 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     if (!MULTI) reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+// k_block_resident: the fully asynchronous solve for systems whose subdomains all fit on the
+// device at once (q <= co-resident blocks; C1-C3). Block c OWNS subdomain c for the whole launch,
+// the paper's picture taken literally: one thread block per subdomain, iterating with no
+// synchronisation with the other blocks (Alg. 1, eq. 3). Everything that does not change between
+// iterations is loaded ONCE: the block's local entries and 1/a_ii in registers, its off-block
+// entries in shared memory, b_i in a register, and x_J stays in shared memory (only this block
+// ever writes it). A global iteration is then: gather the off-block x as it stands (relaxed
+// loads), k local sweeps, relaxed write-back of x_J, residual publication for iteration m
+// (iteration_publish: the block completing iteration m evaluates rel_res_m and stops the solve).
+// Blocks stop on the stop flag or after max_global_iters sweeps; state->work counts the sweeps
+// (one per block and iteration) so the host's stop / resume / iteration accounting is the work
+// queue's. A block may run at most 48 iterations ahead of the
+// last completed one (the 64 residual slots; P:109's bounded delay), spinning otherwise.
+template <int WLR>
+__global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_resident(KP p) {
+    extern __shared__ __align__(128) unsigned char smraw[];
+    __shared__ double sred[2][32];
+    __shared__ int go;
+    const int R = p.R, spb = p.spb;
+    const int64_t q = (p.n + R - 1) / R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t l = blockIdx.x, TS = l * (int64_t)R;
+    const int nrows = (int)min((int64_t)R, p.n - TS);
+    const int nsl = (nrows + kSlice - 1) / kSlice;
+    const int loc = warp * kSlice + lane;
+    const bool ok = warp < nsl && loc < nrows;
+    double *const ybase = reinterpret_cast<double *>(smraw);  // y buffer c at ybase + c R
+    auto ybuf = [&](int c) { return ybase + (c ? R : 0); };
+    // off-block entries of the subdomain: values then columns, slice-major as in the layout
+    double *ov = reinterpret_cast<double *>(smraw) + 2 * R;
+    const int64_t E0 = p.sptr[l * spb];
+    const int ocap = p.wmax * spb * kSlice;
+    int32_t *oc = reinterpret_cast<int32_t *>(ov + ocap);
+    constexpr int NP = WLR / 2;
+    double lv[WLR];
+    uint32_t lc[NP];
+    double bi = 0.0;
+    int wo = 0;
+    uint32_t ooff = 0;
+#pragma unroll
+    for (int e = 0; e < WLR; ++e) lv[e] = 0.0;
+#pragma unroll
+    for (int e = 0; e < NP; ++e) lc[e] = 0;
+    if (ok) {  // once per launch: matrix rows into registers / shared memory, x_J and b_i
+        const int64_t so = p.sptr[l * spb + warp];
+        const int sw = p.sw[l * spb + warp];
+        const int wl = sw & 0xffff;
+        wo = sw >> 16;
+        ooff = (uint32_t)(so - E0) + lane;
+        for (int e = 0; e < wo; ++e) {
+            ov[ooff + e * kSlice] = p.val[so + e * kSlice + lane];
+            oc[ooff + e * kSlice] = p.col[so + e * kSlice + lane];
+        }
+#pragma unroll
+        for (int e = 0; e < WLR; ++e) {
+            if (e < wl) {
+                lv[e] = p.val[so + (int64_t)(wo + e) * kSlice + lane];
+                lc[e >> 1] |= (uint32_t)p.col[so + (int64_t)(wo + e) * kSlice + lane] << (16 * (e & 1));
+            }
+        }
+        bi = p.b[TS + loc];
+        ybase[loc] = ldx<true>(p.x_in + TS + loc);
+    }
+    const double dinv = ok ? 1.0 / lv[0] : 0.0;  // lv[0] = a_ii stays for the correction form
+    // sum of b_i^2 of the block (the same every iteration)
+    double bsum;
+    {
+        const double wb = warp_sum(bi * bi);
+        if (lane == 0) sred[1][warp] = wb;
+        __syncthreads();
+        const int W = blockDim.x >> 5;
+        bsum = 0.0;
+        for (int w = 0; w < W; ++w) bsum += sred[1][w];
+    }
+    int cur = 0;
+    for (long long m = p.m0;; ++m) {
+        if (threadIdx.x == 0) {
+            // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops;
+            // state->work counts the sweeps (the queue kernel's claim count, for the host)
+            int g = m < p.w_end / q && !*(volatile int *)&p.state->stop;
+            if (g) atomicAdd(&p.state->work, 1ull);
+            // bounded lead over the last completed iteration (residual slots are reused mod 64)
+            while (g && m - *(volatile long long *)&p.state->iters_done > 48) {
+                if (*(volatile int *)&p.state->stop) g = 0;
+            }
+            go = g;
+        }
+        __syncthreads();
+        if (!go) break;
+        const double *y0 = ybuf(cur);
+        double *y1 = ybuf(cur ^ 1);
+        double s = bi, rr = 0.0;
+        if (ok) {
+            // a3: off-block part, x as it stands
+            for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                double xv[2 * U];
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) xv[u] = ldx<true>(p.x_in + oc[ooff + (e0 + u) * kSlice]);
+#pragma unroll
+                for (int u = 0; u < 2 * U; ++u)
+                    if (e0 + u < wo) s -= ov[ooff + (e0 + u) * kSlice] * xv[u];
+            }
+            // first local sweep in the correction form: its numerator is r_i (a5)
+            double acc = s;
+#pragma unroll
+            for (int e = 0; e < WLR; ++e) acc -= lv[e] * y0[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+            rr = acc * acc;
+            y1[loc] = y0[loc] + dinv * acc;
+        }
+        __syncthreads();
+        for (int t = 1; t < p.k; ++t) {  // a4: sweeps 2..k, direct form, off-block part frozen
+            const double *yi = ybuf(cur ^ (t & 1));
+            double *yo = ybuf(cur ^ ((t + 1) & 1));
+            if (ok) {
+                double acc = s;
+#pragma unroll
+                for (int e = 1; e < WLR; ++e) acc -= lv[e] * yi[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                yo[loc] = dinv * acc;
+            }
+            __syncthreads();
+        }
+        cur ^= p.k & 1;
+        if (ok) stx<true>(p.x_out + TS + loc, ybuf(cur)[loc]);  // a6
+        const double wr = warp_sum(rr);
+        if (lane == 0) sred[0][warp] = wr;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            const int W = blockDim.x >> 5;
+            double a0 = 0.0;
+            for (int w = 0; w < W; ++w) a0 += sred[0][w];
+            iteration_publish(p, m, 1u, a0, bsum, q);
+        }
+    }
+}
+
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
 // g, g + G, g + 2G, ... (G = warps in the grid) and keeps the next slice's bulk copy in flight
 // (two slice buffers per warp) while computing the current one.
@@ -1916,9 +2053,47 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     return cudaGetLastError();
 }
 
+// k_block_resident for a single-launch async solve when all q subdomains fit on the device at
+// once (grid = q blocks co-resident); BAR_RESIDENT=0 keeps the work-queue kernel.
+template <int WLR>
+bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_t &err) {
+    const char *re = getenv("BAR_RESIDENT");
+    if (re && re[0] == '0') return false;
+    const int threads = L.spb * kSlice;
+    const size_t smem = 2 * (size_t)L.R * sizeof(double) + (size_t)L.max_w * threads * 12;
+    if (smem > kSmemMax) return false;
+    static size_t attr = 0;
+    static size_t c_smem = 0;
+    static int c_threads = 0, occ = 0;
+    if (smem > attr) {
+        if (cudaFuncSetAttribute(k_block_resident<WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            return false;
+        }
+        attr = smem;
+    }
+    if (c_smem != smem || c_threads != threads) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_block_resident<WLR>, threads, smem) != cudaSuccess)
+            occ = 0;
+        cudaGetLastError();
+        c_smem = smem;
+        c_threads = threads;
+    }
+    if ((int64_t)occ * L.sms < L.q) return false;  // every subdomain's block must be co-resident
+    L.last_kernel = "k_block_resident<async>";
+    k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(p);
+    err = cudaGetLastError();
+    return true;
+}
+
 template <bool ASYNC, int WLR>
 cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
-    if (ASYNC && p.w_end > 0) return launch_stage_m<true, WLR, true>(p, L, smem, st);
+    if (ASYNC && p.w_end > 0) {
+        cudaError_t e = cudaSuccess;
+        if (launch_resident_t<WLR>(p, L, st, e)) return e;
+        return launch_stage_m<true, WLR, true>(p, L, smem, st);
+    }
     return launch_stage_m<ASYNC, WLR, false>(p, L, smem, st);
 }
 
@@ -2144,6 +2319,7 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
     p.frozen = a.frozen;
     p.tau = a.tau;
     p.w_end = w_end > 0 ? w_end : 1;
+    p.m0 = a.m0;
     return launch_block<true>(p, *a.L, st);
 }
 
@@ -2190,13 +2366,20 @@ cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nran
     return cudaGetLastError();
 }
 
-__global__ void k_resume_queue(DevState *S) {
-    S->stop = 0;
-    S->work = S->work_resume;
+__global__ void k_resume_queue(DevState *S, int clear_slots) {
+    if (clear_slots) {
+        S->done[threadIdx.x] = 0u;
+        S->ss[threadIdx.x] = 0.0;
+        S->bs[threadIdx.x] = 0.0;
+    }
+    if (threadIdx.x == 0) {
+        S->stop = 0;
+        S->work = S->work_resume;
+    }
 }
 
-cudaError_t launch_resume_queue(DevState *state, cudaStream_t st) {
-    k_resume_queue<<<1, 1, 0, st>>>(state);
+cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slots) {
+    k_resume_queue<<<1, kSlots, 0, st>>>(state, clear_slots ? 1 : 0);
     return cudaGetLastError();
 }
 
