@@ -442,23 +442,36 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         }
     } else {
         // async-(k): in place on buf0. Check x^(0) first (exact), then iterate.
-        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
-        ++launches;
-        if ((r = read_state(A, st)) != BAR_OK) return r;
-        rel = H.exact_rel;
-        if (H.bnorm == 0.0) bzero = true;
-        else if (!std::isfinite(rel)) diverged = true;
-        else if (rel <= tol) converged = 1;
-        // Fully asynchronous persistent solve (one launch for all global iterations); a stop
-        // request raised by the fused estimate is confirmed by an exact residual, else resumed.
         bool multi = use_async_multi(L);
         if (opts && opts->async_single_launch >= 0) multi = opts->async_single_launch == 1;
         if (ext_opts) multi = false;
+        multi = multi && max_global_iters > 0;
+        // the single-launch path decides the x^(0) check on the device (k_init_check), so the
+        // x^(0) residual, the solve and the confirming residual need ONE host round trip
+        bool init_pending = false;
+        auto apply_init = [&](double r0) {
+            rel = r0;
+            if (H.bnorm == 0.0) bzero = true;
+            else if (!std::isfinite(r0)) diverged = true;
+            else if (r0 <= tol) converged = 1;
+        };
+        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+        ++launches;
+        if (multi) {
+            BAR_CUDA(launch_init_check(W.state, st));
+            ++launches;
+            init_pending = true;
+        } else {
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            apply_init(H.exact_rel);
+        }
+        // Fully asynchronous persistent solve (one launch for all global iterations); a stop
+        // request raised by the fused estimate is confirmed by an exact residual, else resumed.
         bool used_multi = false;
         const long long w_end = (long long)max_global_iters * (long long)L.q;
         unsigned long long claimed_before = 0;
         long long m0 = 0;  // k_block_resident: restart iteration after a resume
-        while (multi && !converged && !bzero && !diverged && max_global_iters > 0) {
+        while (multi && !converged && !bzero && !diverged) {
             SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
             a.m0 = m0;
             if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
@@ -467,15 +480,31 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 cudaGetLastError();
                 T.used = 0;
                 multi = false;
+                if (init_pending) {  // fall back to the per-launch kernels with the host-side check
+                    if ((r = read_state(A, st)) != BAR_OK) return r;
+                    apply_init(H.init_rel);
+                    init_pending = false;
+                }
                 break;
             }
             BAR_CUDA(e);
             if ((r = timer_end(T, st)) != BAR_OK) return r;
-            used_multi = true;
+            ++launches;
+            BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
             ++launches;
             if ((r = read_state(A, st)) != BAR_OK) return r;
+            if (init_pending) {
+                init_pending = false;
+                apply_init(H.init_rel);
+                if (converged || bzero || diverged) {  // the kernel returned without sweeping
+                    T.used = 0;
+                    break;
+                }
+            }
+            used_multi = true;
+            const bool resident = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0;
             {  // this launch swept (claimed now - claimed before) subdomains = that / q global iterations
-                const unsigned long long claimed_now = H.stop ? H.work_resume : H.work;
+                const unsigned long long claimed_now = resident ? H.res_sweeps : (H.stop ? H.work_resume : H.work);
                 const double its = (double)(claimed_now - claimed_before) / (double)L.q;
                 claimed_before = claimed_now;
                 if ((r = timer_collect(T, 1, its)) != BAR_OK) return r;
@@ -484,15 +513,11 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 diverged = true;
                 break;
             }
-            BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
-            ++launches;
-            if ((r = read_state(A, st)) != BAR_OK) return r;
             rel = H.exact_rel;
             if (!std::isfinite(rel) || rel > 1e30) diverged = true;
             else if (rel <= tol) converged = 1;
-            else if (!H.stop || (long long)H.work_resume >= w_end) break;  // max_global_iters reached
+            else if (!H.stop || (!resident && (long long)H.work_resume >= w_end)) break;  // max_global_iters reached
             else {
-                const bool resident = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0;
                 m0 = H.iters_done;
                 BAR_CUDA(launch_resume_queue(W.state, st, resident));
             }
@@ -502,7 +527,9 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             // x has that many complete global iterations plus the sweeps still in flight when
             // the queue closed, counted in cta_iters_max)
             iters = (converged && H.stop_iter > 0) ? H.stop_iter : H.iters_done;
-            const unsigned long long claimed = H.stop ? H.work_resume : H.work;
+            const unsigned long long claimed = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0
+                                                   ? H.res_sweeps
+                                                   : (H.stop ? H.work_resume : H.work);
             cta_max = (int64_t)((claimed + L.q - 1) / L.q);
         }
         while (!multi && !converged && !bzero && !diverged && H.iter < max_global_iters) {

@@ -46,6 +46,8 @@ struct DevState {
     unsigned int done[64];  // subdomains of iteration m finished (slot m % 64)
     double ss[64];          // sum of r_i^2 of those subdomains (x as it stood)
     double bs[64];          // sum of b_i^2
+    double init_rel;        // single-launch async: exact rel_res of x^(0) (k_init_check)
+    unsigned long long res_sweeps;  // k_block_resident: subdomain sweeps done (all launches)
 };
 constexpr int kSlots = 64;
 
@@ -76,6 +78,7 @@ struct Layout {
     int32_t *dict = nullptr;    // [dptr[q]]
     int32_t *dptr = nullptr;    // [q + 1]
     int64_t dict_entries = 0;
+    mutable int64_t rw_grid = -1;  // cached rowwise_grid (occupancy queries cost API round trips)
     mutable const char *last_kernel = "none";  // name of the most recently launched sweep kernel
 };
 constexpr int kGhostRanges = 4;
@@ -189,6 +192,10 @@ cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nran
 cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
+// after the exact residual of x^(0): init_rel = exact_rel; if x^(0) already meets tol (or b = 0,
+// or it is not finite) raise stop and close the work queue, so a following single-launch async
+// kernel returns at once — the x^(0) check without a host round trip
+cudaError_t launch_init_check(DevState *state, cudaStream_t st);
 // reopen a closed async queue; clear_slots: also zero the per-iteration residual slots
 // (k_block_resident restarts every block at the last completed iteration)
 cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slots = false);

@@ -1624,9 +1624,8 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // ever writes it). A global iteration is then: gather the off-block x as it stands (relaxed
 // loads), k local sweeps, relaxed write-back of x_J, residual publication for iteration m
 // (iteration_publish: the block completing iteration m evaluates rel_res_m and stops the solve).
-// Blocks stop on the stop flag or after max_global_iters sweeps; state->work counts the sweeps
-// (one per block and iteration) so the host's stop / resume / iteration accounting is the work
-// queue's. A block may run at most 48 iterations ahead of the
+// Blocks stop on the stop flag (read one iteration ahead, so its latency is hidden) or after
+// max_global_iters sweeps; state->res_sweeps counts the sweeps for the host's accounting. A block may run at most 48 iterations ahead of the
 // last completed one (the 64 residual slots; P:109's bounded delay), spinning otherwise.
 template <int WLR>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_resident(KP p) {
@@ -1690,20 +1689,28 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         for (int w = 0; w < W; ++w) bsum += sred[1][w];
     }
     int cur = 0;
+    // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
+    // it before the launch: x^(0) already meets tol)
+    int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
+    unsigned long long sweeps = 0;
     for (long long m = p.m0;; ++m) {
         if (threadIdx.x == 0) {
-            // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops;
-            // state->work counts the sweeps (the queue kernel's claim count, for the host)
-            int g = m < p.w_end / q && !*(volatile int *)&p.state->stop;
-            if (g) atomicAdd(&p.state->work, 1ull);
-            // bounded lead over the last completed iteration (residual slots are reused mod 64)
-            while (g && m - *(volatile long long *)&p.state->iters_done > 48) {
-                if (*(volatile int *)&p.state->stop) g = 0;
+            // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
+            int g = m < p.w_end / q && !stop_seen;
+            // bounded lead over the last completed iteration (residual slots are reused mod 64),
+            // checked every 8 iterations
+            if (g && (m & 7) == 0) {
+                while (g && m - *(volatile long long *)&p.state->iters_done > 40) {
+                    if (*(volatile int *)&p.state->stop) g = 0;
+                }
             }
             go = g;
         }
         __syncthreads();
         if (!go) break;
+        ++sweeps;
+        if (threadIdx.x == 0)  // issued now, consumed at the next iteration's start
+            asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(stop_ld) : "l"(&p.state->stop));
         const double *y0 = ybuf(cur);
         double *y1 = ybuf(cur ^ 1);
         double s = bi, rr = 0.0;
@@ -1747,8 +1754,10 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             double a0 = 0.0;
             for (int w = 0; w < W; ++w) a0 += sred[0][w];
             iteration_publish(p, m, 1u, a0, bsum, q);
+            stop_seen = stop_ld;
         }
     }
+    if (threadIdx.x == 0) atomicAdd(&p.state->res_sweeps, sweeps);
 }
 
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
@@ -1869,6 +1878,7 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->iters_done = 0;
     S->stop_iter = -1;
     S->work_resume = 0;
+    S->res_sweeps = 0;
     for (int i = 0; i < kSlots; ++i) {
         S->done[i] = 0;
         S->ss[i] = 0.0;
@@ -2254,8 +2264,9 @@ cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
 }  // namespace
 
 int64_t rowwise_grid(const Layout &L) {
+    if (L.rw_grid >= 0) return L.rw_grid;
     const int64_t groups = (L.nslices + 7) / 8;
-    if (!rowwise_tma_ok(L)) return groups;
+    if (!rowwise_tma_ok(L)) return L.rw_grid = groups;
     const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
     int a = 0, b = 0;
     cudaFuncSetAttribute(k_rowwise_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBudget);
@@ -2268,7 +2279,7 @@ int64_t rowwise_grid(const Layout &L) {
     int64_t per_sm = a < b ? a : b;  // the same grid for both (deterministic reductions)
     if (per_sm < 1) per_sm = 1;
     const int64_t g = per_sm * L.sms;
-    return g < groups ? g : groups;
+    return L.rw_grid = (g < groups ? g : groups);
 }
 
 int64_t num_blocks_for(const Layout &L, bar_mode mode) {
@@ -2380,6 +2391,19 @@ __global__ void k_resume_queue(DevState *S, int clear_slots) {
 
 cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slots) {
     k_resume_queue<<<1, kSlots, 0, st>>>(state, clear_slots ? 1 : 0);
+    return cudaGetLastError();
+}
+
+__global__ void k_init_check(DevState *S) {
+    S->init_rel = S->exact_rel;
+    if (S->bnorm == 0.0 || !isfinite(S->exact_rel) || S->exact_rel <= S->tol) {
+        S->stop = 1;
+        S->work = 0x3fffffffffffffffull;  // closed: every claim is past any w_end
+    }
+}
+
+cudaError_t launch_init_check(DevState *state, cudaStream_t st) {
+    k_init_check<<<1, 1, 0, st>>>(state);
     return cudaGetLastError();
 }
 
