@@ -958,7 +958,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                 if (EXT) yo[loc] = ext_update(yi[loc], lv[0] * acc, fz, p.tau);
                 else yo[loc] = lv[0] * acc;
             }
-            __syncthreads();
+            if (t + 1 < p.k) __syncthreads();  // the write-back reads only the thread's own row
         }
         // ring slot of l_{i+3} complete before the barrier below publishes it (the newest group,
         // l_{i+4}, may stay in flight)
@@ -1192,7 +1192,9 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             if (EXT) yb[loc] = ext_update(xo, xo + lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
             else yb[loc] = xo + lv[h][0] * acc;
         }
-        __syncthreads();
+        // every thread writes back exactly its own two rows, so the last sweep needs no barrier
+        // before the write-back (the barrier after it guards the buffers' reuse)
+        if (p.k > 1) __syncthreads();
         // a4: sweeps 2..k, direct form, off-block part frozen
         for (int t = 1; t < p.k; ++t) {
             const double *yi = (t & 1) ? yb : ya;
@@ -1207,7 +1209,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 if (EXT) yo[loc] = ext_update(yi[loc], lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
                 else yo[loc] = lv[h][0] * acc;
             }
-            __syncthreads();
+            if (t + 1 < p.k) __syncthreads();
         }
         // ring slot of l_{i+2} complete before the barrier below publishes it
         if (warp == 3 && lane == 0) asm volatile("cp.async.wait_group 1;" ::: "memory");
