@@ -1695,15 +1695,24 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // it before the launch: x^(0) already meets tol)
     int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
     unsigned long long sweeps = 0;
+    int unpaced = 0;  // thread 0: gave up waiting for lagging blocks (see below)
     for (long long m = p.m0;; ++m) {
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
             // bounded lead over the last completed iteration (residual slots are reused mod 64),
-            // checked every 8 iterations
-            if (g && (m & 7) == 0) {
+            // checked every 8 iterations. The wait is itself bounded (~2 ms): if other work on the
+            // device keeps some blocks from being resident, this block goes on iterating without
+            // publishing residuals (unpaced) instead of waiting for them forever; the solve then
+            // ends at max_global_iters and the host's exact residual decides convergence.
+            if (g && !unpaced && (m & 7) == 0) {
+                const long long t0c = clock64();
                 while (g && m - *(volatile long long *)&p.state->iters_done > 40) {
                     if (*(volatile int *)&p.state->stop) g = 0;
+                    if (clock64() - t0c > 4000000ll) {
+                        unpaced = 1;
+                        break;
+                    }
                 }
             }
             go = g;
@@ -1755,7 +1764,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             const int W = blockDim.x >> 5;
             double a0 = 0.0;
             for (int w = 0; w < W; ++w) a0 += sred[0][w];
-            iteration_publish(p, m, 1u, a0, bsum, q);
+            if (!unpaced) iteration_publish(p, m, 1u, a0, bsum, q);
             stop_seen = stop_ld;
         }
     }
