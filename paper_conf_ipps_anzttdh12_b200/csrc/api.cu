@@ -455,7 +455,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             else if (!std::isfinite(r0)) diverged = true;
             else if (r0 <= tol) converged = 1;
         };
-        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+        if (x0 == nullptr) BAR_CUDA(launch_zero_start_residual(L, db, W.state, W.partials, st));
+        else BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
         ++launches;
         if (multi) {
             BAR_CUDA(launch_init_check(W.state, st));

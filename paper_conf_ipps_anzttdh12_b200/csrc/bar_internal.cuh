@@ -189,7 +189,10 @@ cudaError_t launch_residual(const Layout &L, const double *b, const double *x, D
 cudaError_t launch_pack(const double *x_own, const int32_t *idx, int64_t cnt, double *out, cudaStream_t st);
 cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nranks, bool residual_only,
                                cudaStream_t st);
-cudaError_t launch_bnorm(const Layout &L, const double *b, DevState *state, double *partials, cudaStream_t st);
+// exact residual of x^(0) = 0 without the SpMV: b - A 0 = b, so ||r||_2 = ||b||_2 and rel_res = 1
+// (0 for b = 0) — a read of b instead of the matrix (x0 == NULL in bar_solve)
+cudaError_t launch_zero_start_residual(const Layout &L, const double *b, DevState *state, double *partials,
+                                       cudaStream_t st);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
 // after the exact residual of x^(0): init_rel = exact_rel; if x^(0) already meets tol (or b = 0,

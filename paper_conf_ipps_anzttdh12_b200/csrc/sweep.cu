@@ -2405,6 +2405,25 @@ cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slo
     return cudaGetLastError();
 }
 
+__global__ void __launch_bounds__(256) k_zero_start(KP p) {
+    double s = 0.0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < p.n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double v = p.b[i];
+        s += v * v;
+    }
+    reduce_finalize<kResidual>(s, s, p);  // exact_ss = ||b||^2, exact_rel = ||b|| / ||b||
+}
+
+cudaError_t launch_zero_start_residual(const Layout &L, const double *b, DevState *state, double *partials,
+                                       cudaStream_t st) {
+    KP p = make_kp(L);
+    p.b = b;
+    p.state = state;
+    p.partials = partials;
+    k_zero_start<<<(unsigned)rowwise_grid(L), 256, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
 __global__ void k_init_check(DevState *S) {
     S->init_rel = S->exact_rel;
     if (S->bnorm == 0.0 || !isfinite(S->exact_rel) || S->exact_rel <= S->tol) {

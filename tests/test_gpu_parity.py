@@ -210,6 +210,18 @@ def test_b_zero_and_converged_start(bar):
         assert info["iters"] == 0 and info["converged"] and np.array_equal(x, xs)
 
 
+def test_zero_start_shortcut(bar):
+    """x0 = NULL (zero start): the exact residual of x^(0) is ||b|| / ||b|| = 1 without an SpMV
+    (b = 0: x = 0 returned at once); the solve is the same as with an explicit zero x0."""
+    A = W.trefethen(500)
+    x, info = _solve(bar, A, np.zeros(500), 128, 5, "async", 100, 1e-10)
+    assert info["iters"] == 0 and info["converged"] and np.all(x == 0)
+    x1, i1 = _solve(bar, A, np.ones(500), 128, 5, "async", 0, 1e-10)
+    assert i1["iters"] == 0 and not i1["converged"] and i1["rel_res"] == 1.0 and np.all(x1 == 0)
+    x2, i2 = _solve(bar, A, np.ones(500), 128, 5, "async", 20000, 1e-10)
+    assert i2["converged"] and O.rel_res(A, np.ones(500), x2) <= 1e-10 * (1 + 1e-6)
+
+
 @pytest.mark.parametrize("mode", ["async", "sync-block", "jacobi"])
 def test_fixed_point_invariant(bar, mode):
     """Starting at x* with tol = 0, every mode (async included) stays at x* (P7)."""
