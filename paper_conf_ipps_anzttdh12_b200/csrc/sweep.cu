@@ -17,6 +17,7 @@
 //
 // Every kernel is HBM-bound (about 0.17 flop/byte): no tensor cores. Matrix entries are read
 // with coalesced warp-wide loads from the sliced layout (bar_internal.cuh).
+#include <algorithm>
 #include <cstdlib>
 
 #include "bar_internal.cuh"
@@ -45,6 +46,7 @@ struct KP {
     int wmax;  // widest slice (local + off-block entries)
     long long w_end;  // async persistent: claims [0, w_end) = global iterations [0, w_end / q)
     long long m0;     // k_block_resident: global iteration index of this launch's first sweep
+    int lead;         // k_block_resident: max sweeps a block may run ahead of the last completed iteration
     int fresh_xj;     // async persistent with q < 4 * grid: read x_J when a subdomain starts
     double *dist_out; // multi-GPU: [sum r^2, sum b^2] of this rank (no stopping decision here)
     const uint8_t *frozen;  // N1 failure injection: rows that keep their value (nullable)
@@ -1694,20 +1696,22 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
     // it before the launch: x^(0) already meets tol)
     int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
+    long long done_ld = p.m0;  // thread 0: iters_done, loaded one iteration ahead of its use
     unsigned long long sweeps = 0;
     int unpaced = 0;  // thread 0: gave up waiting for lagging blocks (see below)
     for (long long m = p.m0;; ++m) {
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
-            // bounded lead over the last completed iteration (residual slots are reused mod 64),
-            // checked every 8 iterations. The wait is itself bounded (~2 ms): if other work on the
-            // device keeps some blocks from being resident, this block goes on iterating without
-            // publishing residuals (unpaced) instead of waiting for them forever; the solve then
-            // ends at max_global_iters and the host's exact residual decides convergence.
-            if (g && !unpaced && (m & 7) == 0) {
+            // bounded lead over the last completed iteration (p.lead sweeps; residual slots are
+            // reused mod 64). The lead is checked against iters_done as loaded one iteration ago
+            // and only re-read (waited on) when exceeded. The wait is itself bounded (~2 ms): if
+            // other work on the device keeps some blocks from being resident, this block goes on
+            // iterating without publishing residuals (unpaced) instead of waiting for them
+            // forever; the solve then ends at max_global_iters and the exact residual decides.
+            if (g && !unpaced && m - done_ld > p.lead) {
                 const long long t0c = clock64();
-                while (g && m - *(volatile long long *)&p.state->iters_done > 40) {
+                while (g && m - *(volatile long long *)&p.state->iters_done > p.lead) {
                     if (*(volatile int *)&p.state->stop) g = 0;
                     if (clock64() - t0c > 4000000ll) {
                         unpaced = 1;
@@ -1720,8 +1724,10 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         __syncthreads();
         if (!go) break;
         ++sweeps;
-        if (threadIdx.x == 0)  // issued now, consumed at the next iteration's start
+        if (threadIdx.x == 0) {  // issued now, consumed at the next iteration's start
             asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(stop_ld) : "l"(&p.state->stop));
+            asm volatile("ld.relaxed.gpu.global.s64 %0, [%1];" : "=l"(done_ld) : "l"(&p.state->iters_done));
+        }
         const double *y0 = ybuf(cur);
         double *y1 = ybuf(cur ^ 1);
         double s = bi, rr = 0.0;
@@ -2103,7 +2109,12 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     }
     if ((int64_t)occ * L.sms < L.q) return false;  // every subdomain's block must be co-resident
     L.last_kernel = "k_block_resident<async>";
-    k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(p);
+    // lead 3 (B200, round 1, tools/kernel_ab.py): C2 51 vs 56-59 global iterations with lead 40
+    // (0.29 vs 0.33 ms), C3 0.205 vs 0.217 ms; blocks racing far ahead sweep on stale ghosts
+    KP pp = p;
+    pp.lead = 3;
+    if (const char *le = getenv("BAR_LEAD")) pp.lead = std::max(1, std::min(48, atoi(le)));
+    k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(pp);
     err = cudaGetLastError();
     return true;
 }

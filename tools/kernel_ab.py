@@ -76,7 +76,7 @@ def main():
     clk = os.popen("nvidia-smi --query-gpu=clocks.sm,clocks.mem,power.draw --format=csv,noheader").read().strip()
     print(json.dumps({"box": {"copy_GBs": round(copy_gbs, 1), "clocks": clk}}), flush=True)
     base_env = {k: os.environ.get(k) for k in ("BAR_PIPE", "BAR_NO_GHOST_PREFETCH", "BAR_KERNEL", "BAR_ASYNC_STATIC",
-                                          "BAR_DUO", "BAR_JACOBI_ROWWISE", "BAR_GRID", "BAR_ORDER", "BAR_CODED", "BAR_RESIDENT")}
+                                          "BAR_DUO", "BAR_JACOBI_ROWWISE", "BAR_GRID", "BAR_ORDER", "BAR_CODED", "BAR_RESIDENT", "BAR_LEAD")}
     for mode in a.modes.split(","):
         for name, env in parse_variants(a.variants):
             for k_, v in base_env.items():
