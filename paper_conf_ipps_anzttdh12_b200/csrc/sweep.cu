@@ -19,6 +19,7 @@
 // with coalesced warp-wide loads from the sliced layout (bar_internal.cuh).
 #include <algorithm>
 #include <cstdlib>
+#include <mutex>
 
 #include "bar_internal.cuh"
 #include "tma.cuh"
@@ -94,6 +95,10 @@ __device__ __forceinline__ double ext_update(double xold, double v, bool frozen,
 }
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
+
+// Guards the per-kernel static caches of the launchers (dynamic-smem attribute, occupancy):
+// different matrices may be used from different host threads at once.
+std::recursive_mutex g_launch_mu;
 
 constexpr size_t kSmemBudget = 200 * 1024;  // dynamic smem per block; leaves room for static scratch
 constexpr size_t kSmemMax = 227 * 1024 - 1024;  // hardware limit per block minus static scratch
@@ -1924,6 +1929,7 @@ KP make_kp(const Layout &L) {
 
 template <bool ASYNC, bool STAGE>
 cudaError_t launch_block_t(const KP &p, int threads, size_t smem, unsigned grid, cudaStream_t st) {
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr = 0;
     if (smem > attr) {
         cudaError_t e =
@@ -1954,6 +1960,7 @@ cudaError_t launch_reg_w(const KP &p, const Layout &L, cudaStream_t st) {
 
 template <bool ASYNC, int WLR>
 cudaError_t launch_reg_tma_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr = 0;
     if (smem > attr) {
         cudaError_t e =
@@ -1968,6 +1975,7 @@ cudaError_t launch_reg_tma_t(const KP &p, const Layout &L, size_t smem, cudaStre
 // Persistent grid of k_block_pers: every block that fits on the device at once.
 template <bool ASYNC, int WLR>
 int64_t pers_grid(const Layout &L, size_t smem) {
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr = 0;
     if (smem > attr) {
         if (cudaFuncSetAttribute(k_block_pers<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
@@ -1997,6 +2005,7 @@ cudaError_t launch_stage_m(const KP &p, const Layout &L, size_t smem, cudaStream
     const bool ext = !MULTI && (p.frozen != nullptr || p.tau != 1.0);  // N1 / N3 requested
     auto kfn = MULTI ? k_block_stage_m<true, WLR, true>
                      : (ext ? k_block_stage<ASYNC, WLR, true> : k_block_stage<ASYNC, WLR, false>);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr[2] = {0, 0};
     static size_t c_smem[2] = {0, 0};
     static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
@@ -2028,6 +2037,7 @@ template <bool ASYNC, int WLR>
 cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
     auto kfn = ext ? k_block_pipe<ASYNC, WLR, true> : k_block_pipe<ASYNC, WLR, false>;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr[2] = {0, 0};
     static size_t c_smem[2] = {0, 0};
     static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
@@ -2057,6 +2067,7 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     const bool coded = p.codes != nullptr;
     auto kfn = coded ? (ext ? k_block_duo<ASYNC, WLR, true, true> : k_block_duo<ASYNC, WLR, false, true>)
                      : (ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr[4] = {0, 0, 0, 0};
     static size_t c_smem[4] = {0, 0, 0, 0};
     static int c_threads[4] = {0, 0, 0, 0}, occ[4] = {0, 0, 0, 0};
@@ -2089,6 +2100,7 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     const int threads = L.spb * kSlice;
     const size_t smem = 2 * (size_t)L.R * sizeof(double) + (size_t)L.max_w * threads * 12;
     if (smem > kSmemMax) return false;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr = 0;
     static size_t c_smem = 0;
     static int c_threads = 0, occ = 0;
@@ -2272,6 +2284,7 @@ cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
         return cudaGetLastError();
     }
     const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
     static size_t attr = 0;
     if (smem > attr) {
         cudaError_t e = cudaFuncSetAttribute(k_rowwise_tma<RES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
