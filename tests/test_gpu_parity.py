@@ -358,3 +358,35 @@ def test_coded_columns(bar, monkeypatch):
     R = W.random_dd(4096, nnz_per_row=7, seed=3)
     MR = bar.Matrix.from_csr(R, 1024)
     assert MR.info()["coded"] == 0
+
+
+def test_concurrent_handles_threads(bar):
+    """Two matrices solved at the same time from two host threads on two streams (the launchers'
+    static caches are shared): both results meet the exact residual."""
+    import threading
+
+    import torch
+
+    mats = [W.trefethen(2000), W.stencil9_2d(98)]
+    out = [None, None]
+
+    def work(t):
+        A = mats[t]
+        st = torch.cuda.Stream()
+        M = bar.Matrix.from_csr(A, 128)
+        b = _dev(np.ones(A.n))
+        for _ in range(20):
+            with torch.cuda.stream(st):
+                x, info = M.solve(b, None, None, k=5, tol=1e-10, mode="async", stream=st)
+        st.synchronize()
+        out[t] = (x.cpu().numpy(), info)
+        M.close()
+
+    ths = [threading.Thread(target=work, args=(t,)) for t in range(2)]
+    for th in ths:
+        th.start()
+    for th in ths:
+        th.join()
+    for t in range(2):
+        x, info = out[t]
+        assert info["converged"] and O.rel_res(mats[t], np.ones(mats[t].n), x) <= 1e-10 * (1 + 1e-6)
