@@ -72,6 +72,10 @@ bool use_async_multi(const Layout &L) {
     return model_bytes(L) < 256e6;
 }
 
+// single-launch kernels with static ownership (k_block_resident): they count their sweeps in
+// res_sweeps and restart at the last completed iteration after a resume
+static bool static_multi(const char *k) { return std::strstr(k, "resident") != nullptr; }
+
 bar_status read_state(bar_matrix A, cudaStream_t st) {
     BAR_CUDA(cudaMemcpyAsync(A->W.h_state, A->W.state, sizeof(DevState), cudaMemcpyDeviceToHost, st));
     BAR_CUDA(cudaStreamSynchronize(st));
@@ -205,6 +209,8 @@ void bar_destroy(bar_matrix A) {
     free_layout(A->L);
     Workspace &W = A->W;
     timer_free(W.timer);
+    if (W.graph.exec) cudaGraphExecDestroy(W.graph.exec);
+    if (W.graph.cap) cudaStreamDestroy(W.graph.cap);
     cudaFree(W.xbuf);
     cudaFree(W.stage_b);
     cudaFree(W.stage_x);
@@ -448,79 +454,136 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         multi = multi && max_global_iters > 0;
         // the single-launch path decides the x^(0) check on the device (k_init_check), so the
         // x^(0) residual, the solve and the confirming residual need ONE host round trip
-        bool init_pending = false;
         auto apply_init = [&](double r0) {
             rel = r0;
             if (H.bnorm == 0.0) bzero = true;
             else if (!std::isfinite(r0)) diverged = true;
             else if (r0 <= tol) converged = 1;
         };
-        if (x0 == nullptr) BAR_CUDA(launch_zero_start_residual(L, db, W.state, W.partials, st));
-        else BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
-        ++launches;
-        if (multi) {
-            BAR_CUDA(launch_init_check(W.state, st));
-            ++launches;
-            init_pending = true;
-        } else {
-            if ((r = read_state(A, st)) != BAR_OK) return r;
-            apply_init(H.exact_rel);
-        }
-        // Fully asynchronous persistent solve (one launch for all global iterations); a stop
-        // request raised by the fused estimate is confirmed by an exact residual, else resumed.
         bool used_multi = false;
         const long long w_end = (long long)max_global_iters * (long long)L.q;
         unsigned long long claimed_before = 0;
-        long long m0 = 0;  // k_block_resident: restart iteration after a resume
-        while (multi && !converged && !bzero && !diverged) {
-            SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
-            a.m0 = m0;
-            if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
-            cudaError_t e = launch_async_multi(a, w_end, st);
-            if (e == cudaErrorNotSupported) {
-                cudaGetLastError();
-                T.used = 0;
-                multi = false;
-                if (init_pending) {  // fall back to the per-launch kernels with the host-side check
-                    if ((r = read_state(A, st)) != BAR_OK) return r;
-                    apply_init(H.init_rel);
-                    init_pending = false;
-                }
-                break;
-            }
-            BAR_CUDA(e);
-            if ((r = timer_end(T, st)) != BAR_OK) return r;
-            ++launches;
-            BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
-            ++launches;
-            if ((r = read_state(A, st)) != BAR_OK) return r;
-            if (init_pending) {
-                init_pending = false;
-                apply_init(H.init_rel);
-                if (converged || bzero || diverged) {  // the kernel returned without sweeping
-                    T.used = 0;
-                    break;
-                }
-            }
+        long long m0 = 0;  // static-ownership single-launch kernels: restart iteration after a resume
+        double graph_ms = -1.0;  // >= 0: device time of a graph-replayed launch (kernel timestamps)
+        // after a single launch (and its confirming residual) completed: iteration accounting and
+        // the decision; returns true when the solve must be resumed
+        auto after_launch = [&](bool &resume) -> bar_status {
+            resume = false;
             used_multi = true;
-            const bool resident = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0;
+            const bool resident = static_multi(L.last_kernel);
             {  // this launch swept (claimed now - claimed before) subdomains = that / q global iterations
                 const unsigned long long claimed_now = resident ? H.res_sweeps : (H.stop ? H.work_resume : H.work);
                 const double its = (double)(claimed_now - claimed_before) / (double)L.q;
                 claimed_before = claimed_now;
-                if ((r = timer_collect(T, 1, its)) != BAR_OK) return r;
+                if (graph_ms >= 0.0) {  // graph replay: the kernel's own timestamps
+                    if (graph_ms > 0.0) {
+                        T.ms += graph_ms;
+                        T.iters += its;
+                    }
+                    T.used = 0;
+                } else {
+                    bar_status rs = timer_collect(T, 1, its);
+                    if (rs != BAR_OK) return rs;
+                }
             }
             if (H.diverged == 1) {
                 diverged = true;
-                break;
+                return BAR_OK;
             }
             rel = H.exact_rel;
             if (!std::isfinite(rel) || rel > 1e30) diverged = true;
             else if (rel <= tol) converged = 1;
-            else if (!H.stop || (!resident && (long long)H.work_resume >= w_end)) break;  // max_global_iters reached
+            else if (!H.stop || (!resident && (long long)H.work_resume >= w_end)) return BAR_OK;  // max iters
             else {
                 m0 = H.iters_done;
                 BAR_CUDA(launch_resume_queue(W.state, st, resident));
+                resume = true;
+            }
+            return BAR_OK;
+        };
+        if (!multi) {
+            if (x0 == nullptr) BAR_CUDA(launch_zero_start_residual(L, db, W.state, W.partials, st));
+            else BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+            ++launches;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            apply_init(H.exact_rel);
+        } else {
+            // first pass: x^(0) residual, device-side x^(0) check (k_init_check: the kernel then
+            // returns at once), the single-launch solve between the timer events, the confirming
+            // residual and the state read-back — ONE host round trip
+            if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;  // creates the events
+            T.used = 0;
+            cudaEvent_t ev0 = T.ev[0], ev1 = T.ev[1];
+            auto enqueue_first = [&](cudaStream_t s) -> cudaError_t {
+                cudaError_t e = x0 == nullptr ? launch_zero_start_residual(L, db, W.state, W.partials, s)
+                                              : launch_residual(L, db, buf0, W.state, W.partials, s);
+                if (e != cudaSuccess) return e;
+                if ((e = launch_init_check(W.state, s)) != cudaSuccess) return e;
+                if ((e = cudaEventRecord(ev0, s)) != cudaSuccess) return e;
+                SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+                if ((e = launch_async_multi(a, w_end, s)) != cudaSuccess) return e;
+                if ((e = cudaEventRecord(ev1, s)) != cudaSuccess) return e;
+                if ((e = launch_residual(L, db, buf0, W.state, W.partials, s)) != cudaSuccess) return e;
+                return cudaMemcpyAsync(W.h_state, W.state, sizeof(DevState), cudaMemcpyDeviceToHost, s);
+            };
+            SolveGraph &Gr = W.graph;
+            const char *ge = getenv("BAR_GRAPH");
+            const bool same = Gr.b == db && Gr.x0 == x0 && Gr.x == buf0 && Gr.k == k &&
+                              Gr.max_iters == max_global_iters && Gr.tol == tol;
+            bool use_graph = !(ge && ge[0] == '0') && !(same && Gr.unsupported);
+            if (use_graph && !(same && Gr.exec)) {  // (re)capture for this call
+                if (Gr.exec) cudaGraphExecDestroy(Gr.exec);
+                Gr.exec = nullptr;
+                Gr.b = db, Gr.x0 = x0, Gr.x = buf0, Gr.k = k, Gr.max_iters = max_global_iters, Gr.tol = tol;
+                Gr.unsupported = false;
+                if (!Gr.cap) BAR_CUDA(cudaStreamCreateWithFlags(&Gr.cap, cudaStreamNonBlocking));
+                cudaGraph_t graph = nullptr;
+                BAR_CUDA(cudaStreamBeginCapture(Gr.cap, cudaStreamCaptureModeRelaxed));
+                const cudaError_t ec = enqueue_first(Gr.cap);
+                const cudaError_t ee = cudaStreamEndCapture(Gr.cap, &graph);
+                cudaGetLastError();
+                if (ec == cudaSuccess && ee == cudaSuccess && graph &&
+                    cudaGraphInstantiate(&Gr.exec, graph, 0) != cudaSuccess)
+                    Gr.exec = nullptr;
+                if (ec == cudaErrorNotSupported) Gr.unsupported = true;
+                if (graph) cudaGraphDestroy(graph);
+                cudaGetLastError();
+                use_graph = Gr.exec != nullptr;
+            }
+            cudaError_t e = use_graph ? cudaGraphLaunch(Gr.exec, st) : enqueue_first(st);
+            launches += 4;
+            if (e == cudaErrorNotSupported) {  // no single-launch kernel: per-launch kernels below
+                cudaGetLastError();
+                multi = false;
+                launches -= 2;
+                if ((r = read_state(A, st)) != BAR_OK) return r;
+                apply_init(H.init_rel);
+            } else {
+                BAR_CUDA(e);
+                BAR_CUDA(cudaStreamSynchronize(st));
+                // kernel time from the events, or (graph replay) from the kernel's own timestamps
+                T.m[0] = 1;
+                T.used = use_graph ? 0 : 1;
+                graph_ms = !use_graph ? -1.0 : H.t_last > H.t_first ? (H.t_last - H.t_first) * 1e-6 : 0.0;
+                apply_init(H.init_rel);
+                if (converged || bzero || diverged) {  // x^(0) met tol: the kernel returned at once
+                    T.used = 0;
+                } else {
+                    bool resume = false;
+                    if ((r = after_launch(resume)) != BAR_OK) return r;
+                    graph_ms = -1.0;  // resumes launch directly and time with events
+                    while (resume && !converged && !diverged) {  // rare: estimate met tol, exact did not
+                        SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+                        a.m0 = m0;
+                        if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
+                        BAR_CUDA(launch_async_multi(a, w_end, st));
+                        if ((r = timer_end(T, st)) != BAR_OK) return r;
+                        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+                        launches += 2;
+                        if ((r = read_state(A, st)) != BAR_OK) return r;
+                        if ((r = after_launch(resume)) != BAR_OK) return r;
+                    }
+                }
             }
         }
         if (used_multi) {
@@ -528,9 +591,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             // x has that many complete global iterations plus the sweeps still in flight when
             // the queue closed, counted in cta_iters_max)
             iters = (converged && H.stop_iter > 0) ? H.stop_iter : H.iters_done;
-            const unsigned long long claimed = std::strcmp(L.last_kernel, "k_block_resident<async>") == 0
-                                                   ? H.res_sweeps
-                                                   : (H.stop ? H.work_resume : H.work);
+            const unsigned long long claimed = static_multi(L.last_kernel) ? H.res_sweeps
+                                                                           : (H.stop ? H.work_resume : H.work);
             cta_max = (int64_t)((claimed + L.q - 1) / L.q);
         }
         while (!multi && !converged && !bzero && !diverged && H.iter < max_global_iters) {

@@ -48,6 +48,9 @@ struct DevState {
     double bs[64];          // sum of b_i^2
     double init_rel;        // single-launch async: exact rel_res of x^(0) (k_init_check)
     unsigned long long res_sweeps;  // k_block_resident: subdomain sweeps done (all launches)
+    unsigned long long t_first, t_last;  // single-launch kernels: %globaltimer (ns) of the first
+                                         // block start and the last block exit (graph replays
+                                         // cannot time their kernel with host-visible events)
 };
 constexpr int kSlots = 64;
 
@@ -95,8 +98,23 @@ struct KernelTimer {
     double ms = 0.0, iters = 0.0;     // accumulated over the current solve
 };
 
+// The first pass of a single-launch async solve (x^(0) residual, device-side x^(0) check, the
+// solve, the confirming residual, the state read-back) captured as a CUDA graph and replayed when
+// the same call repeats: one graph launch instead of five API launches per solve.
+struct SolveGraph {
+    cudaStream_t cap = nullptr;      // capture stream (library-private)
+    cudaGraphExec_t exec = nullptr;
+    bool unsupported = false;        // the key's call has no single-launch kernel: do not capture
+    const double *b = nullptr, *x0 = nullptr;
+    double *x = nullptr;
+    int32_t k = 0;
+    int64_t max_iters = 0;
+    double tol = 0.0;
+};
+
 struct Workspace {
     KernelTimer timer;
+    SolveGraph graph;
     double *xbuf = nullptr;     // n: second iterate buffer (sync modes)
     double *stage_b = nullptr;  // n: device staging of host b (end-to-end path)
     double *stage_x = nullptr;  // n: device staging of host x0/x

@@ -702,6 +702,17 @@ __host__ __device__ __forceinline__ StageGeom stage_geom(int R, int spb, int wma
     return g;
 }
 
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Thread 0: the state reset leaves t_first = ~0, t_last = 0; every block of a single-launch
+// kernel lowers t_first at its start and raises t_last at its exit.
+__device__ __forceinline__ void stamp_first(DevState *S) { atomicMin(&S->t_first, globaltimer_ns()); }
+__device__ __forceinline__ void stamp_last(DevState *S) { atomicMax(&S->t_last, globaltimer_ns()); }
+
 // Thread 0 of a block that finished a subdomain of global iteration m (MULTI): add its
 // residual contribution to iteration m's accumulators; the block finishing the q-th subdomain
 // of iteration m evaluates rel_res_m (an estimate: each subdomain saw x as it stood) and
@@ -1423,6 +1434,7 @@ struct T0State {
 template <bool ASYNC, int WLR, bool MULTI>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_stage_m(KP p) {
     if (!MULTI && *(volatile int *)&p.state->stop) return;
+    if (MULTI && threadIdx.x == 0) stamp_first(p.state);
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[2];
     __shared__ long long stage_w[2];    // claim held by each stage (>= wend: none)
@@ -1621,6 +1633,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         }
     }
     if (MULTI && threadIdx.x == 0 && t0.pub_cnt) iteration_publish(p, t0.pub_m, t0.pub_cnt, t0.pub_ss, t0.pub_bs, q);
+    if (MULTI && threadIdx.x == 0) stamp_last(p.state);
     if (!MULTI) reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
@@ -1641,6 +1654,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ double sred[2][32];
     __shared__ int go;
+    if (threadIdx.x == 0) stamp_first(p.state);
     const int R = p.R, spb = p.spb;
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -1779,7 +1793,10 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             stop_seen = stop_ld;
         }
     }
-    if (threadIdx.x == 0) atomicAdd(&p.state->res_sweeps, sweeps);
+    if (threadIdx.x == 0) {
+        atomicAdd(&p.state->res_sweeps, sweeps);
+        stamp_last(p.state);
+    }
 }
 
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
@@ -1901,6 +1918,8 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->stop_iter = -1;
     S->work_resume = 0;
     S->res_sweeps = 0;
+    S->t_first = ~0ull;
+    S->t_last = 0;
     for (int i = 0; i < kSlots; ++i) {
         S->done[i] = 0;
         S->ss[i] = 0.0;
