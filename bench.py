@@ -392,8 +392,9 @@ def main():
                 "frac": round(achieved / peak, 4), "traffic": None,
                 "kernel": kernel_name,
                 "kernel_ms": round(kernel_ms, 5), "algorithmic_bytes_per_launch": local_bytes,
-                "timing": f"CUDA events around each sweep launch inside the {args.steps} timed solves "
-                          f"({sk_it:g} global iterations, {sk_ms:.3f} ms of sweep kernels on rank 0)",
+                "timing": f"device time of the sweep kernels inside the {args.steps} timed solves ({sk_it:g} global "
+                          f"iterations, {sk_ms:.3f} ms on rank 0): CUDA events on the launching stream around each "
+                          f"launch (graph-replayed single-launch solves: the kernel's %globaltimer stamps)",
                 "kernel_ms_isolated": round(kernel_ms_isolated, 5),
                 "frac_isolated": round(local_bytes / (kernel_ms_isolated * 1e-3) / 1e9 / peak, 4),
                 "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
