@@ -390,3 +390,34 @@ def test_concurrent_handles_threads(bar):
     for t in range(2):
         x, info = out[t]
         assert info["converged"] and O.rel_res(mats[t], np.ones(mats[t].n), x) <= 1e-10 * (1 + 1e-6)
+
+
+def test_graph_replay(bar, monkeypatch):
+    """Repeated single-launch solves replay a captured graph: same pointers (new contents of b are
+    read), new pointers (recaptured), max_global_iters / tol changes, and BAR_GRAPH=0 all give
+    solutions that meet the exact residual; the graph's kernel time is reported."""
+    import torch
+
+    A = W.trefethen(2000)
+    M = bar.Matrix.from_csr(A, 128)
+    b = _dev(np.ones(A.n))
+    x = torch.empty_like(b)
+    infos = []
+    for rep in range(3):
+        _, info = M.solve(b, None, x, k=5, tol=1e-10, mode="async")
+        infos.append(info)
+        assert info["converged"] and O.rel_res(A, np.ones(A.n), x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    assert infos[-1]["sweep_kernel_ms"] > 0 and infos[-1]["sweep_kernel_iters"] > 0
+    b2 = np.random.default_rng(4).uniform(0.5, 1.5, A.n)
+    b.copy_(torch.from_numpy(b2))  # same pointer, new right-hand side
+    _, info = M.solve(b, None, x, k=5, tol=1e-10, mode="async")
+    assert info["converged"] and O.rel_res(A, b2, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    x2 = torch.empty_like(b)  # new output pointer: recaptured
+    _, info = M.solve(b, None, x2, k=5, tol=1e-12, mode="async")
+    assert info["converged"] and O.rel_res(A, b2, x2.cpu().numpy()) <= 1e-12 * (1 + 1e-6)
+    _, info = M.solve(b, None, x2, k=5, max_global_iters=3, tol=0.0, mode="async")
+    assert info["iters"] == 3 and not info["converged"]
+    monkeypatch.setenv("BAR_GRAPH", "0")
+    _, info = M.solve(b, None, x, k=5, tol=1e-10, mode="async")
+    assert info["converged"] and O.rel_res(A, b2, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    M.close()
