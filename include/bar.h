@@ -29,7 +29,8 @@
  * last error on the calling thread is available from bar_last_error(). Not converging within
  * max_global_iters is NOT an error (BAR_OK with info.converged = 0).
  *
- * Threads. A bar_matrix may be used by one thread at a time (its workspace is reused).
+ * Threads. A bar_matrix may be used by one thread at a time (its workspace is reused); different
+ * matrices may be used from different threads at once.
  */
 #ifndef BAR_H
 #define BAR_H
@@ -130,7 +131,12 @@ bar_status bar_create_csr(int64_t n, int64_t nnz, const int32_t *rowptr, const i
  * Stopping rule (reading R6): x^(0) is checked first; the sync modes return the
  * first x^(m) with rel_res <= tol (bitwise the oracle's m up to the order of the residual sum);
  * async returns the first iterate whose fused residual estimate AND exact confirming residual
- * are <= tol. b = 0 returns x = 0, iters = 0, converged.
+ * are <= tol. b = 0 returns x = 0, iters = 0, converged. With x0 == NULL the exact residual of
+ * x^(0) = 0 is ||b|| / ||b|| (one read of b, no SpMV).
+ * Async kernels: large systems run one launch per global iteration; systems whose
+ * subdomains all fit on the device at once run ONE launch for all iterations, and a repeated call
+ * with the same pointers, k, max_global_iters and tol replays that solve from a CUDA graph the
+ * handle captured on the first such call (the contents behind the pointers may change).
  * Errors: BAR_ERR_INVALID_ARG, BAR_ERR_NONFINITE (b or x0), BAR_ERR_DIVERGED, BAR_ERR_CUDA,
  *         BAR_ERR_OOM. On BAR_ERR_DIVERGED x holds the last iterate.
  */
