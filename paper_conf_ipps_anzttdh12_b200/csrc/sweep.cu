@@ -726,10 +726,12 @@ __device__ __forceinline__ void iteration_publish(const KP &p, long long m, unsi
     const int slot = (int)(m % kSlots);
     atomicAdd(&S->ss[slot], t0);
     atomicAdd(&S->bs[slot], t1);
-    __threadfence();
-    const unsigned int c = atomicAdd(&S->done[slot], cnt);
+    // the count is an acq_rel atomic: it releases this block's sums and, for the block that
+    // completes the iteration, acquires every other block's (no separate gpu-scope fences)
+    unsigned int c;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(c) : "l"(&S->done[slot]), "r"(cnt)
+                 : "memory");
     if (c + cnt != (unsigned int)q) return;
-    __threadfence();
     const double ss = __longlong_as_double(
         (long long)atomicExch(reinterpret_cast<unsigned long long *>(&S->ss[slot]), 0ull));
     const double bsq = __longlong_as_double(
