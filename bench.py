@@ -219,7 +219,7 @@ def run_reference(args):
     n, nnz = matrix_dims(args.workload)
     cores, model = cpu_info()
     # global iterations the GPU's async-(5) needs at the default R (bench runs)
-    iters = args.ref_iters or {"c1": 29, "c2": 56, "c3": 27, "c4": 62, "c5": 44}[args.workload]
+    iters = args.ref_iters or {"c1": 29, "c2": 51, "c3": 27, "c4": 62, "c5": 44}[args.workload]
     budget = args.ref_rows
     for _ in range(args.warmup):
         oracle_sample(args.workload, args.k, args.R, args.mode, budget // 4)
