@@ -675,7 +675,7 @@ __global__ void __launch_bounds__(1024, 1) k_block_pers(KP p) {
 }
 
 // ---------------------------------------------------------------------------------------------
-// k_block_stage: the default block sweep. Persistent blocks; everything one subdomain needs —
+// k_block_stage: the staged block sweep (R = 128-class subdomains). Persistent blocks; everything one subdomain needs —
 // its slices' values and columns (one contiguous range of the layout), b_J, x_J (= y^0), and
 // the slices' metadata — arrives in one shared-memory STAGE through six bulk copies (TMA) that
 // complete on one mbarrier. Two stages: while the block sweeps subdomain l out of one stage,
@@ -2171,11 +2171,17 @@ bool staged_ok(const KP &p, const Layout &L) {
     return aligned && geom_ok && stage_smem <= kSmemMax;
 }
 
-// Kernel choice for one block-sweep launch (async / sync-block):
-//   k_block_stage persistent, whole-subdomain TMA stages (default when it fits)
-//   k_block_pers  persistent, double-buffered TMA slice stream (default when it fits)
-//   k_reg_tma  subdomains of <= 1024 rows with <= 8 local entries per row (every stencil
-//              config): TMA-streamed slices, register-resident local entries
+// Kernel choice for one block-sweep launch (async / sync-block / Jacobi), in order:
+//   k_block_duo    two blocks per SM, <= 4 local entries per row, R >= 256 (C4, C5; coded
+//                  columns when the layout has them); async always, sync when the pipelined
+//                  kernel would hold a whole SM
+//   k_block_pipe   persistent, two subdomains of look-ahead (R >= 256 or sync-block k >= 3)
+//   k_block_stage  persistent, whole-subdomain TMA stages; with p.w_end > 0 (single launch for
+//                  all iterations): k_block_resident when every subdomain fits on the device at
+//                  once (C1-C3), else the work-queue k_block_stage_m
+//   k_block_pers   persistent, double-buffered TMA slice stream
+//   k_reg_tma  subdomains of <= 1024 rows with <= 8 local entries per row: TMA-streamed slices,
+//              register-resident local entries
 //   k_reg      same without TMA (BAR_KERNEL=r, for comparison)
 //   k_block    anything else: local entries staged in shared memory when they fit, else
 //              re-read through L1/L2 each sweep (BAR_KERNEL=s forces it)
