@@ -421,3 +421,24 @@ def test_graph_replay(bar, monkeypatch):
     _, info = M.solve(b, None, x, k=5, tol=1e-10, mode="async")
     assert info["converged"] and O.rel_res(A, b2, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
     M.close()
+
+
+@pytest.mark.parametrize("coded", ["1", "0"])
+def test_duo_partial_last_subdomain(bar, monkeypatch, coded):
+    """The two-blocks-per-SM kernel (coded and int32 columns) on a 2D 9-point stencil whose last
+    subdomain is partial (n = 10^6 is not a multiple of R = 512, so its last slices are short and
+    padded): sync-block-(5) and Jacobi iterates match the oracle to 1e-12, async converges."""
+    monkeypatch.setenv("BAR_DUO", "1")
+    monkeypatch.setenv("BAR_CODED", coded)
+    A = W.stencil9_2d(1000)
+    R = 512
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(11).uniform(-1, 1, A.n)
+    for mode, k in (("sync-block", 5), ("jacobi", 1)):
+        ref = x0
+        for _ in range(2):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x, _ = _solve(bar, A, b, R, k, mode, 2, 0.0, x0)
+        _close(x, ref)
+    x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10)
+    assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
