@@ -113,3 +113,25 @@ def test_history_matches_oracle(bar, mode, k):
     h = info["history"]
     assert len(h) == r.iters + 1
     np.testing.assert_allclose(h, r.history, rtol=1e-9, atol=1e-15)
+
+
+@pytest.mark.parametrize("coded", ["1", "0"])
+def test_ext_options_on_duo_kernel(bar, monkeypatch, coded):
+    """N3 tau-scaling and N1 failure windows through the two-blocks-per-SM kernel's EXT
+    instantiations (coded and int32 columns): iterates match the oracle to 1e-12."""
+    monkeypatch.setenv("BAR_DUO", "1")
+    monkeypatch.setenv("BAR_CODED", coded)
+    A = W.stencil7_3d(128)  # R = two grid lines: <= 4 local entries per row
+    R = 256
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(13).uniform(-1, 1, A.n)
+    for mode, k, meth in (("sync-block", 5, O.BLOCK_JACOBI), ("jacobi", 1, O.JACOBI)):
+        ref = x0
+        for _ in range(2):
+            ref = O.step_ex(A, b, ref, meth, R=R, k=k, tau=0.8)
+        x, _ = _gpu(bar, A, b, R, k, mode, 2, 0.0, x0, tau=0.8)
+        _close(x, ref)
+    fz = np.random.default_rng(14).random(A.n) < 0.25
+    r = O.solve(A, b, method=O.BLOCK_JACOBI, R=R, k=5, tol=0.0, max_iters=4, frozen=fz, fail_start=2, fail_stop=4)
+    x, _ = _gpu(bar, A, b, R, 5, "sync-block", 4, 0.0, fail_mask=fz, fail_start=2, fail_stop=4)
+    _close(x, r.x)
