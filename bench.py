@@ -256,11 +256,15 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-p2p", action="store_true", help="multi-GPU async: NCCL halo exchange instead of P2P")
+    ap.add_argument("--halo", default="sendrecv", choices=["sendrecv", "allgather"],
+                    help="multi-GPU NCCL halo exchange: grouped send/recv (default) or ncclAllGather")
     args = ap.parse_args()
     if args.R is None:
         args.R = WORKLOADS[args.workload][2]
     if args.impl == "reference":
         return run_reference(args)
+    if args.halo == "allgather":
+        os.environ["BAR_HALO"] = "allgather"
 
     import torch
 

@@ -255,7 +255,9 @@ bar_status bar_dist_link_loopback(bar_dist *ranks, int nranks);
 /*
  * bar_dist_solve — the collective solve (every rank calls it with the same k, limits and mode):
  * b, x0, x are this rank's owned rows (device or host, as bar_solve). Each global iteration:
- * pack the rows peers need, NCCL grouped send/recv into the ghost slots, one block sweep on the
+ * pack the rows peers need, NCCL grouped send/recv into the ghost slots (or, with the
+ * environment variable BAR_HALO=allgather set when the ranks are created, one ncclAllGather of
+ * every rank's packed send buffer and a copy of this rank's segments), one block sweep on the
  * local subdomains, all-gather of the per-rank [sum r^2, sum b^2] and a rank-ordered sum, so all
  * ranks take the same stopping decision. Async mode: blocks of a rank run asynchronously
  * (async-(k) within the GPU) and read the ghosts of the latest exchange.

@@ -36,6 +36,14 @@ struct bar_dist_s {
     int64_t n_send = 0;
     std::vector<int64_t> send_cnt, send_off, recv_cnt, recv_pos;  // recv_pos: owned-relative index
     double *part = nullptr;      // device [2]: this rank's [sum r^2, sum b^2]
+    // halo exchange by ncclAllGather (SURVEY §8(e)'s primary design; BAR_HALO=allgather): every
+    // rank contributes its whole send buffer padded to ag_max doubles, and each receiver copies
+    // its segment of every sender p out of slot p of the gathered buffer (peer_off[p] = where p's
+    // segment for this rank starts in p's send buffer). Planned on the first exchange.
+    bool halo_allgather = false, ag_ready = false;
+    int64_t ag_max = 0;
+    double *ag_buf = nullptr;            // device [nranks * ag_max]
+    std::vector<int64_t> peer_off;
     double *gathered = nullptr;  // device [2 * nranks]
     // async over peer memory (bar_dist_enable_p2p)
     bool p2p = false;
@@ -82,12 +90,88 @@ bar_status to_device(const T *src, int64_t count, T **dst) {
 
 double *own(const bar_dist D, double *ext) { return ext + D->glo_pad; }
 
+// All-gather halo plan: the largest send buffer of the group and, for this rank, the offset of
+// its segment in every sender's buffer (NCCL: one all-gather of the send counts at first use;
+// loopback: read from the linked peers).
+bar_status plan_allgather(bar_dist *ranks, int nr, cudaStream_t st) {
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        if (D->ag_ready) continue;
+        const int P = D->nranks;
+        std::vector<int64_t> cnt((size_t)P * P, 0);  // cnt[p * P + d]: what p sends to d
+        if (D->loopback) {
+            for (int p = 0; p < P; ++p)
+                for (int d = 0; d < P; ++d) cnt[(size_t)p * P + d] = D->peers[p]->send_cnt[d];
+        } else {
+#ifdef BAR_WITH_NCCL
+            int64_t *dev = nullptr;
+            BAR_CUDA(cudaMalloc(&dev, sizeof(int64_t) * (size_t)P * (P + 1)));
+            BAR_CUDA(cudaMemcpyAsync(dev, D->send_cnt.data(), sizeof(int64_t) * P, cudaMemcpyHostToDevice, st));
+            BAR_NCCL(ncclAllGather(dev, dev + P, (size_t)P, ncclInt64, D->comm, st));
+            BAR_CUDA(cudaMemcpyAsync(cnt.data(), dev + P, sizeof(int64_t) * (size_t)P * P, cudaMemcpyDeviceToHost, st));
+            BAR_CUDA(cudaStreamSynchronize(st));
+            cudaFree(dev);
+#else
+            return nccl_fail(0, "plan_allgather");
+#endif
+        }
+        D->ag_max = 1;
+        D->peer_off.assign(P, 0);
+        for (int p = 0; p < P; ++p) {
+            int64_t tot = 0, off = 0;
+            for (int d = 0; d < P; ++d) {
+                if (d == D->rank) off = tot;
+                tot += cnt[(size_t)p * P + d];
+            }
+            D->peer_off[p] = off;
+            if (tot > D->ag_max) D->ag_max = tot;
+            if (cnt[(size_t)p * P + D->rank] != D->recv_cnt[p]) {
+                set_error("all-gather plan mismatch: send/recv counts differ");
+                return BAR_ERR_INVALID_ARG;
+            }
+        }
+        BAR_CUDA(cudaMalloc(&D->ag_buf, sizeof(double) * (size_t)P * D->ag_max));
+        D->ag_ready = true;
+    }
+    return BAR_OK;
+}
+
 // Refresh the ghost slots of the extended vector `ext` of every rank in `ranks` (NCCL: the
 // calling rank only; loopback: all ranks of the process, in order, on one stream).
 bar_status exchange(bar_dist *ranks, int nr, double *const *ext, cudaStream_t st) {
     for (int i = 0; i < nr; ++i) {
         bar_dist D = ranks[i];
         BAR_CUDA(launch_pack(own(D, ext[i]), D->send_idx, D->n_send, D->send_buf, st));
+    }
+    if (ranks[0]->halo_allgather) {
+        bar_status r = plan_allgather(ranks, nr, st);
+        if (r != BAR_OK) return r;
+        const int P = ranks[0]->nranks;
+        const int64_t M = ranks[0]->ag_max;
+        if (!ranks[0]->loopback) {
+#ifdef BAR_WITH_NCCL
+            bar_dist D = ranks[0];
+            BAR_NCCL(ncclAllGather(D->send_buf, D->ag_buf, (size_t)M, ncclDouble, D->comm, st));
+#else
+            return nccl_fail(0, "exchange");
+#endif
+        } else {  // loopback: the same gathered buffer, assembled by copies into every rank's ag_buf
+            for (int i = 0; i < nr; ++i)
+                for (int p = 0; p < P; ++p)
+                    if (ranks[p]->n_send)
+                        BAR_CUDA(cudaMemcpyAsync(ranks[i]->ag_buf + (size_t)p * M, ranks[p]->send_buf,
+                                                 sizeof(double) * (size_t)ranks[p]->n_send, cudaMemcpyDeviceToDevice,
+                                                 st));
+        }
+        for (int i = 0; i < nr; ++i) {  // each receiver: its segment of every sender's slot
+            bar_dist D = ranks[i];
+            for (int p = 0; p < P; ++p) {
+                if (p == D->rank || !D->recv_cnt[p]) continue;
+                BAR_CUDA(cudaMemcpyAsync(own(D, ext[i]) + D->recv_pos[p], D->ag_buf + (size_t)p * M + D->peer_off[p],
+                                         sizeof(double) * (size_t)D->recv_cnt[p], cudaMemcpyDeviceToDevice, st));
+            }
+        }
+        return BAR_OK;
     }
     if (!ranks[0]->loopback) {
 #ifdef BAR_WITH_NCCL
@@ -516,6 +600,10 @@ bar_status bar_dist_create(int64_t n_global, int64_t row_begin, int64_t row_end,
         }
     }
     D->n_send = nsend;
+    {
+        const char *he = getenv("BAR_HALO");
+        D->halo_allgather = he && std::strcmp(he, "allgather") == 0;
+    }
     bar_status st = BAR_OK;
     // local layout: rows [0, nl), columns [-n_glo, nl + n_ghi)
     {
@@ -750,6 +838,7 @@ void bar_dist_destroy(bar_dist D) {
     cudaFree(D->xio);
     cudaFree(D->send_idx);
     cudaFree(D->send_buf);
+    cudaFree(D->ag_buf);
     cudaFree(D->part);
     cudaFree(D->gathered);
     delete D;

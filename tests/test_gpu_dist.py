@@ -140,3 +140,24 @@ def test_partitioned_duo_coded(bar, monkeypatch, P):
         assert np.array_equal(xs, xp), mode
     x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n))
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+@pytest.mark.parametrize("name,gen,args,R", MATS)
+@pytest.mark.parametrize("P", [2, 3])
+def test_halo_allgather_bitwise(bar, monkeypatch, name, gen, args, R, P):
+    """The ncclAllGather halo exchange (BAR_HALO=allgather, SURVEY §8(e)'s primary design; here
+    through the loopback transport's emulation of the gather): every rank's whole send buffer is
+    gathered and each receiver copies its segments out, so sync-block and Jacobi iterates stay
+    bitwise the one-GPU iterates, as with the grouped send/recv exchange."""
+    monkeypatch.setenv("BAR_HALO", "allgather")
+    A = gen(*args)
+    n = A.n
+    b = np.ones(n)
+    x0 = np.random.default_rng(6).uniform(-1, 1, n)
+    blocks = _split(gen, args, n, R, P)
+    for mode, k in (("sync-block", 5), ("jacobi", 1)):
+        xs, _ = _single(bar, A, b, R, k, mode, 3, 0.0, x0)
+        xp, info = _loop(blocks, n, R, b, k, mode, 3, 0.0, x0)
+        assert np.array_equal(xs, xp), (mode, np.abs(xs - xp).max())
+    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n))
+    assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
