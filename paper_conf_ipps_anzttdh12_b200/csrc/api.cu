@@ -402,26 +402,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
     bool diverged = false, nonfinite = false, bzero = false;
     double *result = buf0;
     int64_t chunk = 8;
-    // size of the next chunk of per-launch sweeps: doubling (8, 16, ..., 256), or, once two fused
-    // estimates are known, the launches the observed per-iteration rate needs to reach tol plus a
-    // margin of 2, so the chunk that reaches tol does not queue up to 255 launches that return at
-    // once (each still a full-grid launch) and needs no extra host round trip.
-    long long est_it = -1;
-    double est_rel = 0.0;
-    auto next_chunk = [&](int64_t c) -> int64_t {
-        const long long it = (long long)H.iter;
-        const double rel_now = H.last_rel;
-        int64_t nc = std::min<int64_t>(c * 2, 256);
-        if (est_it >= 0 && it > est_it && est_rel > 0.0 && rel_now > 0.0 && rel_now < est_rel && tol > 0.0 &&
-            std::isfinite(rel_now)) {
-            const double rate = std::pow(rel_now / est_rel, 1.0 / (double)(it - est_it));
-            const double need = std::ceil(std::log(tol / rel_now) / std::log(rate));
-            if (rate > 0.0 && rate < 1.0 && need >= 0.0 && need < 256.0) nc = std::max<int64_t>(1, (int64_t)need + 2);
-        }
-        est_it = it;
-        est_rel = rel_now;
-        return nc;
-    };
+    ChunkSizer sizer;  // per-launch sweeps are queued in chunks (bar_internal.cuh)
+    auto next_chunk = [&](int64_t c) -> int64_t { return sizer.next(c, (long long)H.iter, H.last_rel, tol); };
 
     if (mode != BAR_MODE_ASYNC) {
         int64_t issued = 0;  // launches m = 1..issued

@@ -13,6 +13,8 @@
 // and the diagonal (for D^-1) is found without a search.
 #pragma once
 
+#include <cmath>
+
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -53,6 +55,30 @@ struct DevState {
                                          // cannot time their kernel with host-visible events)
 };
 constexpr int kSlots = 64;
+
+// Host: size of the next chunk of per-launch sweeps queued before the host reads the state.
+// Doubling (8, 16, ..., 256), or, once two fused estimates (iteration it, rel) are known, the
+// launches the observed per-iteration rate needs to reach tol plus a margin of 2: the chunk that
+// reaches tol then does not queue up to 255 launches that return at once (each a full-grid
+// launch, and in the collective multi-GPU path a halo exchange and an all-gather) and needs no
+// extra host round trip. Deterministic in (it, rel), so ranks holding the same agreed state size
+// their chunks identically.
+struct ChunkSizer {
+    long long it = -1;
+    double rel = 0.0;
+    int64_t next(int64_t c, long long it_now, double rel_now, double tol) {
+        int64_t nc = c * 2 < 256 ? c * 2 : 256;
+        if (it >= 0 && it_now > it && rel > 0.0 && rel_now > 0.0 && rel_now < rel && tol > 0.0 &&
+            std::isfinite(rel_now)) {
+            const double rate = std::pow(rel_now / rel, 1.0 / (double)(it_now - it));
+            const double need = std::ceil(std::log(tol / rel_now) / std::log(rate));
+            if (rate > 0.0 && rate < 1.0 && need >= 0.0 && need < 256.0) nc = (int64_t)need + 2;
+        }
+        it = it_now;
+        rel = rel_now;
+        return nc;
+    }
+};
 
 struct Layout {
     int64_t n = 0, nnz = 0;

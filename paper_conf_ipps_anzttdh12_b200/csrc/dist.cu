@@ -345,6 +345,7 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
     KernelTimer &T = D0->A->W.timer;
     timer_reset(T);
     int64_t issued = 0, chunk = 8;
+    ChunkSizer sizer;  // collective path: sized from the agreed state (identical on every rank)
     int64_t iters = 0;
     double rel = 0.0;
     int converged = 0;
@@ -390,7 +391,9 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                 stopped = H.stop != 0;
             }
             if ((r = timer_collect(T, (int64_t)H.iter, 1.0)) != BAR_OK) return r;
-            chunk = std::min<int64_t>(chunk * 2, 256);
+            // p2p: each rank's estimate comes from its own board, so chunks keep doubling there
+            // (every rank must reach agree_stop's all-reduce the same number of times)
+            chunk = p2p ? std::min<int64_t>(chunk * 2, 256) : sizer.next(chunk, (long long)H.iter, H.last_rel, tol);
         }
         if (stopped && mode != BAR_MODE_ASYNC) {
             iters = H.conv_iter;
