@@ -517,10 +517,10 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             T.used = 0;
             cudaEvent_t ev0 = T.ev[0], ev1 = T.ev[1];
             auto enqueue_first = [&](cudaStream_t s) -> cudaError_t {
-                cudaError_t e = x0 == nullptr ? launch_zero_start_residual(L, db, W.state, W.partials, s)
-                                              : launch_residual(L, db, buf0, W.state, W.partials, s);
+                // the residual kernel's last block applies the x^(0) check (k_init_check's rule)
+                cudaError_t e = x0 == nullptr ? launch_zero_start_residual(L, db, W.state, W.partials, s, true)
+                                              : launch_residual(L, db, buf0, W.state, W.partials, s, nullptr, true);
                 if (e != cudaSuccess) return e;
-                if ((e = launch_init_check(W.state, s)) != cudaSuccess) return e;
                 if ((e = cudaEventRecord(ev0, s)) != cudaSuccess) return e;
                 SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
                 if ((e = launch_async_multi(a, w_end, s)) != cudaSuccess) return e;
@@ -553,7 +553,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 use_graph = Gr.exec != nullptr;
             }
             cudaError_t e = use_graph ? cudaGraphLaunch(Gr.exec, st) : enqueue_first(st);
-            launches += 4;
+            launches += 3;
             if (e == cudaErrorNotSupported) {  // no single-launch kernel: per-launch kernels below
                 cudaGetLastError();
                 multi = false;

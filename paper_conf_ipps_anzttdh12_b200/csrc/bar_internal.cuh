@@ -226,8 +226,10 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st);
 // Fully asynchronous persistent solve: claims [work, w_end) = global iterations up to w_end / q
 // in ONE launch; cudaErrorNotSupported when the layout/vectors do not fit the staged kernel.
 cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t st);
+// init_check: the last block also applies k_init_check's rule (one launch fewer on the
+// single-launch async path)
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state,
-                            double *partials, cudaStream_t st, double *dist_out = nullptr);
+                            double *partials, cudaStream_t st, double *dist_out = nullptr, bool init_check = false);
 // Multi-GPU helpers (sweep.cu): gather the values peers need; apply the stopping rule to the
 // rank-ordered sum of every rank's [sum r^2, sum b^2] (identical decision on every rank).
 cudaError_t launch_pack(const double *x_own, const int32_t *idx, int64_t cnt, double *out, cudaStream_t st);
@@ -236,7 +238,7 @@ cudaError_t launch_dist_decide(DevState *state, const double *gathered, int nran
 // exact residual of x^(0) = 0 without the SpMV: b - A 0 = b, so ||r||_2 = ||b||_2 and rel_res = 1
 // (0 for b = 0) — a read of b instead of the matrix (x0 == NULL in bar_solve)
 cudaError_t launch_zero_start_residual(const Layout &L, const double *b, DevState *state, double *partials,
-                                       cudaStream_t st);
+                                       cudaStream_t st, bool init_check = false);
 cudaError_t launch_check_finite(const double *v, int64_t n, int *flag, cudaStream_t st);
 cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st);
 // after the exact residual of x^(0): init_rel = exact_rel; if x^(0) already meets tol (or b = 0,

@@ -59,6 +59,7 @@ struct KP {
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
+    int init_check;         // residual kernels: the last block also applies the x^(0) check
 };
 
 // Static subdomain claims of persistent block c of G (k_block_pipe / k_block_duo), R15: round
@@ -127,6 +128,16 @@ __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     return v;
+}
+
+// After the exact residual of x^(0) (a7, O5: m = 0 is checked first): init_rel = exact_rel; if
+// x^(0) already meets tol (or b = 0, or it is not finite) the solve stops before the first sweep.
+__device__ __forceinline__ void init_check_rule(DevState *S) {
+    S->init_rel = S->exact_rel;
+    if (S->bnorm == 0.0 || !isfinite(S->exact_rel) || S->exact_rel <= S->tol) {
+        S->stop = 1;
+        S->work = 0x3fffffffffffffffull;  // closed: every claim is past any w_end
+    }
 }
 
 // The stopping rule (R2/R6/R14) on the global sums of r_i^2 and b_i^2.
@@ -216,6 +227,7 @@ __device__ __forceinline__ void reduce_finalize(double rr, double bb, const KP &
         return;
     }
     apply_stop_rule(S, ss, bsq, KIND == kResidual, p.hist);
+    if (KIND == kResidual && p.init_check) init_check_rule(S);
 }
 
 constexpr int U = 4;  // stored entries of a row loaded together (loads in flight per thread)
@@ -2397,13 +2409,14 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
 }
 
 cudaError_t launch_residual(const Layout &L, const double *b, const double *x, DevState *state, double *partials,
-                            cudaStream_t st, double *dist_out) {
+                            cudaStream_t st, double *dist_out, bool init_check) {
     KP p = make_kp(L);
     p.b = b;
     p.x_in = x;
     p.state = state;
     p.partials = partials;
     p.dist_out = dist_out;
+    p.init_check = init_check && dist_out == nullptr ? 1 : 0;
     return launch_rowwise<true>(p, L, st);
 }
 
@@ -2466,22 +2479,17 @@ __global__ void __launch_bounds__(256) k_zero_start(KP p) {
 }
 
 cudaError_t launch_zero_start_residual(const Layout &L, const double *b, DevState *state, double *partials,
-                                       cudaStream_t st) {
+                                       cudaStream_t st, bool init_check) {
     KP p = make_kp(L);
     p.b = b;
     p.state = state;
     p.partials = partials;
+    p.init_check = init_check ? 1 : 0;
     k_zero_start<<<(unsigned)rowwise_grid(L), 256, 0, st>>>(p);
     return cudaGetLastError();
 }
 
-__global__ void k_init_check(DevState *S) {
-    S->init_rel = S->exact_rel;
-    if (S->bnorm == 0.0 || !isfinite(S->exact_rel) || S->exact_rel <= S->tol) {
-        S->stop = 1;
-        S->work = 0x3fffffffffffffffull;  // closed: every claim is past any w_end
-    }
-}
+__global__ void k_init_check(DevState *S) { init_check_rule(S); }
 
 cudaError_t launch_init_check(DevState *state, cudaStream_t st) {
     k_init_check<<<1, 1, 0, st>>>(state);
