@@ -157,6 +157,23 @@ def test_iteration_count_and_solution(bar, name, mode, k, R):
     _close(x, r.x)
 
 
+@pytest.mark.parametrize("mode,k,R", [("jacobi", 1, 448), ("sync-block", 5, 128)])
+def test_few_launches_queued_past_the_stop(bar, mode, k, R):
+    """The per-launch solve loop sizes its last chunk from the observed residual rate
+    (ChunkSizer, csrc/bar_internal.cuh): on fv1 (Jacobi 146, sync-block-(5) 92 iterations) doubling
+    chunks 8, 16, 32, 64, 128 would queue 248 / 120 sweeps; the sized chunk stays within a few
+    launches of iters + 1 (the stop is detected in the sweep after x^(iters)). Same iterate and
+    count as the oracle either way."""
+    A = MATS["fv1"]()
+    b = np.ones(A.n)
+    meth = O.JACOBI if mode == "jacobi" else O.BLOCK_JACOBI
+    r = O.solve(A, b, method=meth, R=R, k=k, tol=1e-10)
+    x, info = _solve(bar, A, b, R, k, mode, 20000, 1e-10)
+    assert info["converged"] == 1 and info["iters"] == r.iters
+    _close(x, r.x)
+    assert info["kernel_launches"] <= r.iters + 1 + 12, (info["kernel_launches"], r.iters)
+
+
 def test_dyadic_bitwise(bar):
     """Exact dyadic iterates: GPU == oracle bit for bit, any order/FMA."""
     A = W.dyadic_stencil9_2d(40, p=4)
