@@ -278,23 +278,30 @@ bar_status p2p_iteration(bar_dist D, const SweepArgs &a, bar_mode mode, cudaStre
 }
 
 // Chunk-boundary agreement on the stop requests of all ranks (the only synchronisation of the
-// asynchronous multi-GPU mode besides the exact confirming residual).
-bar_status agree_stop(bar_dist *ranks, int nr, cudaStream_t st, bool &any) {
+// asynchronous multi-GPU mode besides the exact confirming residual), and on the size of the next
+// chunk: every rank sizes it from its own estimate (ChunkSizer) and all take the largest, so every
+// rank reaches this all-reduce equally often.
+bar_status agree_stop(bar_dist *ranks, int nr, cudaStream_t st, bool &any, ChunkSizer *sizers, int64_t chunk,
+                      double tol, int64_t &next) {
     any = false;
+    next = 1;
     for (int i = 0; i < nr; ++i) {
         bar_status r = read_state(ranks[i]->A, st);
         if (r != BAR_OK) return r;
-        any = any || ranks[i]->A->W.h_state->stop != 0;
+        const DevState &h = *ranks[i]->A->W.h_state;
+        any = any || h.stop != 0;
+        next = std::max<int64_t>(next, sizers[i].next(chunk, (long long)h.iter, h.last_rel, tol));
     }
     if (!ranks[0]->loopback) {
 #ifdef BAR_WITH_NCCL
         bar_dist D = ranks[0];
-        int v = any ? 1 : 0, out = 0;
-        BAR_CUDA(cudaMemcpyAsync(D->d_flag, &v, sizeof(int), cudaMemcpyHostToDevice, st));
-        BAR_NCCL(ncclAllReduce(D->d_flag, D->d_flag, 1, ncclInt32, ncclMax, D->comm, st));
-        BAR_CUDA(cudaMemcpyAsync(&out, D->d_flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+        int v[2] = {any ? 1 : 0, (int)next}, out[2] = {0, 0};
+        BAR_CUDA(cudaMemcpyAsync(D->d_flag, v, sizeof(v), cudaMemcpyHostToDevice, st));
+        BAR_NCCL(ncclAllReduce(D->d_flag, D->d_flag, 2, ncclInt32, ncclMax, D->comm, st));
+        BAR_CUDA(cudaMemcpyAsync(out, D->d_flag, sizeof(out), cudaMemcpyDeviceToHost, st));
         BAR_CUDA(cudaStreamSynchronize(st));
-        any = out != 0;
+        any = out[0] != 0;
+        next = out[1];
 #endif
     }
     return BAR_OK;
@@ -346,6 +353,8 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
     timer_reset(T);
     int64_t issued = 0, chunk = 8;
     ChunkSizer sizer;  // collective path: sized from the agreed state (identical on every rank)
+    std::vector<ChunkSizer> p2p_sizers(nr);  // p2p: one per rank, agreed in agree_stop
+    int64_t p2p_next = 8;
     int64_t iters = 0;
     double rel = 0.0;
     int converged = 0;
@@ -385,15 +394,16 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
             }
             issued += c;
             if (p2p) {
-                if ((r = agree_stop(ranks, nr, st, stopped)) != BAR_OK) return r;
+                if ((r = agree_stop(ranks, nr, st, stopped, p2p_sizers.data(), chunk, tol, p2p_next)) != BAR_OK)
+                    return r;
             } else {
                 if ((r = read_state(D0->A, st)) != BAR_OK) return r;
                 stopped = H.stop != 0;
             }
             if ((r = timer_collect(T, (int64_t)H.iter, 1.0)) != BAR_OK) return r;
-            // p2p: each rank's estimate comes from its own board, so chunks keep doubling there
-            // (every rank must reach agree_stop's all-reduce the same number of times)
-            chunk = p2p ? std::min<int64_t>(chunk * 2, 256) : sizer.next(chunk, (long long)H.iter, H.last_rel, tol);
+            // p2p: each rank's estimate comes from its own board; the ranks agree on the largest
+            // of their chunk sizes in agree_stop
+            chunk = p2p ? p2p_next : sizer.next(chunk, (long long)H.iter, H.last_rel, tol);
         }
         if (stopped && mode != BAR_MODE_ASYNC) {
             iters = H.conv_iter;
@@ -753,8 +763,8 @@ bar_status bar_dist_enable_p2p(bar_dist D, const int32_t *ghost_src_idx, const v
     }
     DeviceGuard g(D->device);
     if (!D->board) BAR_CUDA(cudaMalloc(&D->board, sizeof(double) * 2 * (size_t)D->nranks));
-    if (!D->d_flag) BAR_CUDA(cudaMalloc(&D->d_flag, sizeof(int)));
-    BAR_CUDA(cudaMemset(D->d_flag, 0, sizeof(int)));
+    if (!D->d_flag) BAR_CUDA(cudaMalloc(&D->d_flag, 2 * sizeof(int)));  // [stop request, next chunk]
+    BAR_CUDA(cudaMemset(D->d_flag, 0, 2 * sizeof(int)));
     // ghost j's owner: ghosts are ordered by owner (recv_counts), owners' ranges are contiguous
     std::vector<int32_t> grank(ng), gidx(ng);
     {
