@@ -156,9 +156,10 @@ bar_status bar_solve(bar_matrix A, const double *b, const double *x0, double *x,
  *   res_history  HOST double[max_global_iters + 1] (nullable): sync modes rel_res(x^(m)) for
  *              m = 0..iters (exact up to the summation order); async the fused per-iteration
  *              estimate (x as each block saw it). Entries past iters are left untouched.
- *   async_single_launch  -1 auto, 0 one launch per global iteration, 1 the fully asynchronous
- *              single-launch kernel (falls back silently where it does not apply). Options
- *              tau != 1, fail_mask and res_history imply 0.
+ *   async_single_launch  -1 the handle's choice (bar_tuning.single_launch), 0 one launch per
+ *              global iteration, 1 the fully asynchronous single-launch kernel (falls back
+ *              silently where it does not apply). Options tau != 1, fail_mask and res_history
+ *              imply 0.
  */
 typedef struct {
     double tau;
@@ -194,6 +195,43 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
 /* bar_matrix_get_info — sizes and the contract bytes per global iteration of a handle. */
 bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info);
 
+/*
+ * bar_tuning — explicit per-handle overrides of the library's kernel and schedule choices
+ * (DESIGN.md §5). The library reads NO environment variables: every choice that is not the
+ * default is made here, on one handle, by the caller (profiling, A/B runs, and the tests that
+ * force each kernel path). All-zero = the defaults. Choices that do not apply to a layout fall
+ * back silently to the next kernel in the dispatch order; sync-block and Jacobi
+ * iterates do not depend on any field here (bitwise), async iterates depend on the schedule.
+ */
+typedef struct {
+    int32_t kernel;         /* 0 auto; force a fallback family: 1 k_block (shared-memory staged),
+                               2 k_reg, 3 k_reg_tma, 4 k_block_pers                              */
+    int32_t duo;            /* 0 auto, 1 two-blocks-per-SM kernel wherever it fits, -1 never      */
+    int32_t pipe;           /* 0 auto, 1 two-ahead pipelined kernel wherever it fits, -1 never    */
+    int32_t coded;          /* 0 auto (coded columns when the layout has them), -1 int32 columns  */
+    int32_t async_order;    /* per-launch async subdomain order: 0 auto (contiguous chunks per
+                               block, R15), 1 chunks, 2 round robin, 3 strided chunks (chunks of
+                               the plane-transposed sequence, where the layout has a plane stride) */
+    int32_t async_queue;    /* 0 static claims, 1 device work-queue claims (k_block_stage)       */
+    int32_t resident;       /* 0 auto, -1 never use the block-owns-subdomain single-launch kernel */
+    int32_t lead;           /* k_block_resident: max sweeps a block may lead the last completed
+                               global iteration (0 = default 3; 1..48)                           */
+    int32_t ghost_prefetch; /* L2 bulk prefetch of the gather ranges: 0 auto (R >= 512), 1, -1   */
+    int32_t graph;          /* single-launch async: 0 capture + replay as a CUDA graph, -1 never  */
+    int32_t single_launch;  /* async: 0 auto (one launch for all iterations when one iteration
+                               moves < 256 MB), 1 always where it applies, -1 never              */
+    int32_t jacobi_rowwise; /* 1: Jacobi by the row-wise kernel even where the staged kernels apply */
+    int32_t grid_cap;       /* > 0: at most this many persistent blocks                          */
+    int32_t warps;          /* k_block: warps per block (0 auto)                                 */
+    int32_t halo;           /* multi-GPU sync / collective exchange: 0 NCCL grouped send/recv,
+                               1 one ncclAllGather per iteration                                 */
+    int32_t peer;           /* multi-GPU async: 0 peer memory when mapped, -1 the collective path */
+} bar_tuning;
+
+/* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a
+ * concurrent call on the same handle. Errors: BAR_ERR_INVALID_ARG. */
+bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning);
+
 /* bar_destroy — free the handle and its device memory (NULL-safe). */
 void bar_destroy(bar_matrix A);
 
@@ -203,42 +241,95 @@ void bar_destroy(bar_matrix A);
  * of rows ... assigned to the different thread blocks" (§3.4). row_begin must be a
  * multiple of rows_per_block, so subdomains never straddle ranks and the per-row arithmetic
  * is identical to the one-GPU solve (sync-block / Jacobi iterates are bitwise independent of
- * the number of ranks). Columns a rank reads but does not own ("ghosts") are refreshed once
- * per global iteration: halo exchange by NCCL grouped send/recv over NVLink, replacing the
- * paper's AMC / DC / DK host- or master-GPU transfers. Local numbering is
- * order-preserving: [ghosts below row_begin | owned rows | ghosts above], stored relative to
+ * the number of ranks). Columns a rank reads but does not own are its "ghosts". Local numbering
+ * is order-preserving: [ghosts below row_begin | owned rows | ghosts above], stored relative to
  * the owned block (ghosts below are negative), so a row's entries keep their global order.
  *
- * Planning (host only, no GPU, usable before any device exists):
+ * Two ways a rank reads its ghosts, replacing the paper's AMC / DC / DK host- or master-GPU
+ * transfers:
+ *   collective    sync-block and Jacobi (and async when peer memory is unavailable): once per
+ *                 global iteration, NCCL grouped send/recv over NVLink (bar_tuning.halo = 0) or
+ *                 one ncclAllGather (halo = 1) refreshes the ghost slots; the per-rank residual
+ *                 sums are all-gathered and added in rank order, so every rank takes the same
+ *                 stopping decision from the same bits.
+ *   peer memory   async (the default when every rank can map every other rank's memory; north
+ *                 star: "an async mode reads peers' x over NVLink P2P with no barrier"; the paper's
+ *                 DK idea, without a master GPU): before each local sweep a rank PULLS its
+ *                 ghosts from the owners' live iterates (relaxed system-scope loads: x "as it
+ *                 stands", eq. 3) and pushes its residual partial into every rank's board (a small
+ *                 array in each rank's memory, mapped through CUDA IPC). No collective and no
+ *                 barrier while iterating: a rank whose estimate meets tol writes a tagged stop
+ *                 request into every board, and the ranks meet only for the exact confirming
+ *                 residual (two board barriers: device-side release/acquire waits, 20 s timeout
+ *                 -> BAR_ERR_NCCL instead of a hang). info.iters = min over ranks of the global
+ *                 iterations each ran; info.cta_iters_max = the max.
+ */
+
+/*
+ * bar_create_csr_dist — §8(b)'s multi-GPU entry point: this rank's share of a row-partitioned
+ * matrix, planned inside the library. Collective: every rank of the group calls it.
+ *   n_global        rows of the global system
+ *   row_begin/end   this rank's rows (row_begin a multiple of rows_per_block; the ranks' ranges
+ *                   contiguous and ascending in rank order, together [0, n_global))
+ *   nnz_local, rowptr, col, val   the local rows in CSR with GLOBAL column ids (rowptr relative,
+ *                   rowptr[0] = 0), host or device memory, copied
+ *   rows_per_block  R; device: this rank's GPU
+ *   nccl_unique_id  128 bytes from bar_nccl_unique_id on rank 0, given to every rank (required)
+ *   rank, nranks    this rank and the group size
+ * Inside: ncclCommInitRank; an all-gather of every rank's row range, ghost count and device, and
+ * of the ghost lists; the exchange plan and local numbering; the local layout; and, when every
+ * rank can reach every other rank's memory (cudaDeviceCanAccessPeer, agreed by a min
+ * all-reduce), an all-gather of CUDA IPC handles that maps every rank's iterate and board.
+ * The returned handle works with bar_solve / bar_residual (collective: b, x0, x are this rank's
+ * rows; every rank calls with the same k, limits and mode), bar_matrix_get_info (local sizes),
+ * bar_set_tuning, bar_sweep (local launches on this rank's rows, no exchange: kernel timing) and
+ * bar_destroy (frees the communicator). bar_solve_ex options tau, fail_mask and res_history are
+ * not supported on it (BAR_ERR_INVALID_ARG).
+ * Errors: as bar_create_csr, plus BAR_ERR_NCCL; BAR_ERR_INVALID_ARG for a bad partition.
+ */
+bar_status bar_create_csr_dist(int64_t n_global, int64_t row_begin, int64_t row_end, int64_t nnz_local,
+                               const int32_t *rowptr, const int32_t *col, const double *val, int32_t rows_per_block,
+                               int device, const void *nccl_unique_id, int rank, int nranks, bar_matrix *out);
+
+/* bar_nccl_unique_id — rank 0 creates the NCCL id (128 bytes) that every rank passes to
+ * bar_create_csr_dist / bar_dist_create (broadcast it by any means). BAR_ERR_NCCL without NCCL. */
+bar_status bar_nccl_unique_id(void *id128);
+
+/* ---- lower-level building blocks (explicit plans; tests, in-process loopback groups) -------- */
+typedef struct bar_dist_s *bar_dist; /* opaque, one per rank */
+
+/* Planning, host only (no GPU needed):
  *   bar_dist_ghosts    sorted distinct ghost columns of the local rows: the n_ghost_lo ones
  *                      below row_begin, then the n_ghost_hi ones at or above row_end. Call with
  *                      ghosts = NULL for the counts. rowptr is relative (rowptr[0] = 0), col global.
  *   bar_dist_localize  col_local[e] = col[e] - row_begin for owned columns, -n_ghost_lo + j for
  *                      the j-th ghost below, (row_end - row_begin) + j for the j-th ghost above.
- * The caller exchanges ghost lists with its process group (tests: gloo; bench: NCCL) to get
- *   recv_counts[p]  how many of this rank's ghosts rank p owns (they are consecutive in ghost order)
- *   send_counts[p]  how many owned rows rank p needs, and send_idx (their local row indices, in p's
- *                   ghost order, concatenated by p).
+ *   bar_dist_plan      from every rank's row range (row_ranges[2p], [2p+1]), ghost count and
+ *                      ghost list (ghosts_all: the lists concatenated in rank order): this rank's
+ *                      recv_counts[p] (its ghosts owned by p; consecutive in ghost order),
+ *                      send_counts[p] and send_idx (owned local rows p needs, in p's ghost order,
+ *                      concatenated by p; NULL to get the counts first) and ghost_src_idx[j]
+ *                      (owner-local row of ghost j, for bar_dist_enable_p2p; nullable).
  */
-typedef struct bar_dist_s *bar_dist; /* opaque, one per rank */
-
 bar_status bar_dist_ghosts(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
                            const int32_t *col, int64_t *n_ghost_lo, int64_t *n_ghost_hi, int32_t *ghosts);
 bar_status bar_dist_localize(int64_t row_begin, int64_t row_end, int64_t nnz_local, const int32_t *rowptr,
                              const int32_t *col, int64_t n_ghost_lo, int64_t n_ghost_hi, const int32_t *ghosts,
                              int32_t *col_local);
-
-/* bar_nccl_unique_id — rank 0 creates the NCCL id (128 bytes) that every rank passes to
- * bar_dist_create (broadcast it with the caller's process group). BAR_ERR_NCCL without NCCL. */
-bar_status bar_nccl_unique_id(void *id128);
+bar_status bar_dist_plan(int nranks, int rank, const int64_t *row_ranges, const int64_t *ghost_counts,
+                         const int32_t *ghosts_all, int64_t *recv_counts, int64_t *send_counts, int32_t *send_idx,
+                         int32_t *ghost_src_idx);
 
 /*
- * bar_dist_create — this rank's share: the local CSR (n_local = row_end - row_begin rows,
- * col_local from bar_dist_localize, values), the exchange plan, and the transport.
- *   nccl_id   128-byte ncclUniqueId from bar_nccl_unique_id, or NULL for the in-process
- *             LOOPBACK transport (several ranks in one process on one device, linked with
- *             bar_dist_link_loopback and driven by bar_dist_solve_loopback — for testing the
- *             partitioned path on a single GPU).
+ * bar_dist_create — this rank's share from an explicit plan: the local CSR (n_local = row_end -
+ * row_begin rows, col_local from bar_dist_localize, values), the plan (bar_dist_plan), and the
+ * transport.
+ *   nccl_id   128-byte ncclUniqueId (an NCCL communicator for the collective path), or NULL: no
+ *             communicator — then either link the ranks of one process into a LOOPBACK group
+ *             (bar_dist_link_loopback; several ranks on one device, device copies as the exchange,
+ *             driven by bar_dist_solve_loopback — the partitioned path on a single GPU), or, for
+ *             separate processes, enable peer memory (bar_dist_enable_p2p with IPC handles): then
+ *             only the async mode is available.
  *   send_idx  int32[sum send_counts] local row indices; send/recv_counts int64[nranks].
  * Arrays may be host or device memory and are copied. Errors as bar_create_csr, plus
  * BAR_ERR_NCCL, BAR_ERR_INVALID_ARG (row_begin not a multiple of R, inconsistent counts).
@@ -253,14 +344,12 @@ bar_status bar_dist_create(int64_t n_global, int64_t row_begin, int64_t row_end,
 bar_status bar_dist_link_loopback(bar_dist *ranks, int nranks);
 
 /*
- * bar_dist_solve — the collective solve (every rank calls it with the same k, limits and mode):
- * b, x0, x are this rank's owned rows (device or host, as bar_solve). Each global iteration:
- * pack the rows peers need, NCCL grouped send/recv into the ghost slots (or, with the
- * environment variable BAR_HALO=allgather set when the ranks are created, one ncclAllGather of
- * every rank's packed send buffer and a copy of this rank's segments), one block sweep on the
- * local subdomains, all-gather of the per-rank [sum r^2, sum b^2] and a rank-ordered sum, so all
- * ranks take the same stopping decision. Async mode: blocks of a rank run asynchronously
- * (async-(k) within the GPU) and read the ghosts of the latest exchange.
+ * bar_dist_solve — the solve of one rank (every rank calls it with the same k, limits and mode):
+ * b, x0, x are this rank's owned rows (device or host, as bar_solve). Collective path per global
+ * iteration: halo exchange, one block sweep of the local subdomains, all-gather of the per-rank
+ * [sum r^2, sum b^2] and a rank-ordered sum. Async over peer memory: see above. Async without
+ * peer memory: blocks of a rank run asynchronously (async-(k) within the GPU) and read the
+ * ghosts of the latest collective exchange.
  */
 bar_status bar_dist_solve(bar_dist D, const double *b, const double *x0, double *x, int32_t k,
                           int64_t max_global_iters, double tol, bar_mode mode, void *cuda_stream,
@@ -273,18 +362,12 @@ bar_status bar_dist_solve_loopback(bar_dist *ranks, int nranks, const double *co
                                    bar_mode mode, void *cuda_stream, bar_solve_info *info);
 
 /*
- * Asynchronous multi-GPU mode over peer memory (north star: "an async mode reads peers' x over
- * NVLink P2P with no barrier"; the paper's DK idea, without a master GPU). After
- * bar_dist_enable_p2p, bar_dist_solve / bar_dist_solve_loopback in BAR_MODE_ASYNC no longer
- * exchange halos collectively: before every local sweep each rank PULLS its ghost values from
- * the owners' live iterates with relaxed system-scope loads (x "as it stands", eq. 3) and
- * pushes its residual partial into every peer's board; ranks only synchronise at chunk
- * boundaries (a one-int all-reduce of the stop requests) and for the exact confirming residual.
+ * Peer memory for the async mode (bar_create_csr_dist does this itself):
  *   bar_dist_p2p_handles  128 bytes: CUDA IPC handles of this rank's iterate and board (publish
  *                         them to the group), and *own_offset (its owned-block offset, in doubles).
  *   bar_dist_enable_p2p   ghost_src_idx[j] = owner-local row of ghost j (ghost order); handles =
  *                         nranks * 128 bytes and own_offsets = nranks offsets gathered from every
- *                         rank, or both NULL for linked loopback ranks (same process).
+ *                         rank, or both NULL for linked loopback ranks (same process) and 1-rank groups.
  */
 bar_status bar_dist_p2p_handles(bar_dist D, void *handles128, int64_t *own_offset);
 bar_status bar_dist_enable_p2p(bar_dist D, const int32_t *ghost_src_idx, const void *handles,
@@ -294,6 +377,9 @@ bar_status bar_dist_enable_p2p(bar_dist D, const int32_t *ghost_src_idx, const v
  * block-sweep kernel on its current iterate (no halo exchange, no convergence control, no sync;
  * ghost values are whatever the last exchange left). Local, not collective. */
 bar_status bar_dist_sweep(bar_dist D, int32_t k, int64_t nsweeps, bar_mode mode, void *cuda_stream);
+
+/* bar_dist_set_tuning — bar_set_tuning of the rank's local handle (kernel choice, halo mode). */
+bar_status bar_dist_set_tuning(bar_dist D, const bar_tuning *tuning);
 
 /* bar_dist_destroy — free one rank's share (NULL-safe; also destroys its NCCL communicator). */
 void bar_dist_destroy(bar_dist D);

@@ -4,9 +4,10 @@ Every step of the solve runs in the library's CUDA kernels; this module only con
 numpy arrays / torch tensors into pointers. It never falls back to a CPU path: if
 ``libbar.so`` is missing or fails to load, importing this module raises.
 
-The C names are kept: ``bar_create_csr``, ``bar_solve``, ``bar_residual``,
-``bar_matrix_get_info``, ``bar_destroy``, ``bar_last_error``. ``Matrix`` is a small
-RAII wrapper over them.
+The C names are kept: ``bar_create_csr``, ``bar_solve``, ``bar_solve_ex``, ``bar_sweep``,
+``bar_residual``, ``bar_matrix_get_info``, ``bar_set_tuning``, ``bar_destroy``,
+``bar_last_error``. ``Matrix`` is a small RAII wrapper over them. The library reads no
+environment variable: kernel / schedule overrides go through ``Matrix.set_tuning``.
 """
 from __future__ import annotations
 
@@ -30,10 +31,11 @@ STATUS = {0: "BAR_OK", 1: "BAR_ERR_INVALID_ARG", 2: "BAR_ERR_BAD_CSR", 3: "BAR_E
 MAX_ROWS_PER_BLOCK = 8192
 
 # every symbol include/bar.h declares (tests check the export table against the header)
-EXPORTS = ("bar_create_csr", "bar_solve", "bar_solve_ex", "bar_sweep", "bar_residual", "bar_matrix_get_info", "bar_destroy",
-           "bar_last_error", "bar_dist_ghosts", "bar_dist_localize", "bar_nccl_unique_id", "bar_dist_create",
-           "bar_dist_link_loopback", "bar_dist_solve", "bar_dist_solve_loopback", "bar_dist_sweep",
-           "bar_dist_p2p_handles", "bar_dist_enable_p2p", "bar_dist_destroy")
+EXPORTS = ("bar_create_csr", "bar_solve", "bar_solve_ex", "bar_sweep", "bar_residual", "bar_matrix_get_info",
+           "bar_set_tuning", "bar_destroy", "bar_last_error", "bar_create_csr_dist", "bar_nccl_unique_id",
+           "bar_dist_ghosts", "bar_dist_localize", "bar_dist_plan", "bar_dist_create", "bar_dist_link_loopback",
+           "bar_dist_solve", "bar_dist_solve_loopback", "bar_dist_sweep", "bar_dist_p2p_handles",
+           "bar_dist_enable_p2p", "bar_dist_set_tuning", "bar_dist_destroy")
 
 
 class SolveInfo(ctypes.Structure):
@@ -65,7 +67,40 @@ class MatrixInfo(ctypes.Structure):
         return d
 
 
+class Tuning(ctypes.Structure):
+    """bar_tuning (include/bar.h): explicit per-handle kernel / schedule overrides; zero = defaults."""
+
+    _fields_ = [(f, ctypes.c_int32) for f in (
+        "kernel", "duo", "pipe", "coded", "async_order", "async_queue", "resident", "lead", "ghost_prefetch", "graph",
+        "single_launch", "jacobi_rowwise", "grid_cap", "warps", "halo", "peer")]
+
+    KERNELS = {"auto": 0, "block": 1, "reg": 2, "reg_tma": 3, "pers": 4}
+    ORDERS = {"auto": 0, "chunks": 1, "round_robin": 2, "strided": 3}
+
+    @classmethod
+    def make(cls, **kw):
+        """Tuning(kernel="block", duo=-1, async_order="round_robin", halo="allgather", ...)."""
+        t = cls()
+        for k, v in kw.items():
+            if k == "kernel" and isinstance(v, str):
+                v = cls.KERNELS[v]
+            elif k == "async_order" and isinstance(v, str):
+                v = cls.ORDERS[v]
+            elif k == "async_queue" and isinstance(v, str):
+                v = {"static": 0, "queue": 1}[v]
+            elif k == "halo" and isinstance(v, str):
+                v = {"sendrecv": 0, "allgather": 1}[v]
+            elif isinstance(v, bool):
+                v = 1 if v else -1
+            if k not in dict(cls._fields_):
+                raise KeyError(f"unknown bar_tuning field {k}")
+            setattr(t, k, int(v))
+        return t
+
+
 _vp, _i64, _i32, _f64 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_double
+_lib.bar_set_tuning.restype = ctypes.c_int
+_lib.bar_set_tuning.argtypes = [_vp, ctypes.POINTER(Tuning)]
 _lib.bar_create_csr.restype = ctypes.c_int
 _lib.bar_create_csr.argtypes = [_i64, _i64, _vp, _vp, _vp, _i32, ctypes.c_int, ctypes.POINTER(_vp)]
 _lib.bar_solve.restype = ctypes.c_int
@@ -173,6 +208,13 @@ def bar_matrix_get_info(A):
     return info
 
 
+def bar_set_tuning(A, tuning=None):
+    """tuning: a Tuning, a dict of its fields, or None (defaults)."""
+    if isinstance(tuning, dict):
+        tuning = Tuning.make(**tuning)
+    _check(_lib.bar_set_tuning(A, ctypes.byref(tuning) if tuning is not None else None))
+
+
 def bar_destroy(A):
     _lib.bar_destroy(A)
 
@@ -191,17 +233,24 @@ def _stream_handle(stream):
 class Matrix:
     """A CSR matrix resident on a B200 in the library's layout (owns a bar_matrix handle)."""
 
-    def __init__(self, rowptr, col, val, rows_per_block: int = 128, device: int = 0, n: int | None = None):
+    def __init__(self, rowptr, col, val, rows_per_block: int = 128, device: int = 0, n: int | None = None,
+                 tuning=None):
         n = (len(rowptr) - 1) if n is None else n
         nnz = int(rowptr[-1]) if isinstance(rowptr, np.ndarray) else int(rowptr[-1].item())
         self.handle = bar_create_csr(n, nnz, rowptr, col, val, rows_per_block, device)
         self.n, self.nnz, self.R, self.device = n, nnz, rows_per_block, device
+        if tuning:
+            self.set_tuning(tuning)
 
     @classmethod
-    def from_csr(cls, A, rows_per_block: int = 128, device: int = 0):
+    def from_csr(cls, A, rows_per_block: int = 128, device: int = 0, tuning=None):
         """From a workloads.CSR (host numpy arrays)."""
         return cls(np.ascontiguousarray(A.rowptr, dtype=np.int32), np.ascontiguousarray(A.col, dtype=np.int32),
-                   np.ascontiguousarray(A.val, dtype=np.float64), rows_per_block, device, n=A.n)
+                   np.ascontiguousarray(A.val, dtype=np.float64), rows_per_block, device, n=A.n, tuning=tuning)
+
+    def set_tuning(self, tuning=None, **kw):
+        """bar_set_tuning: a Tuning, a dict, keyword fields, or nothing (defaults)."""
+        bar_set_tuning(self.handle, tuning if tuning is not None or not kw else dict(kw))
 
     def info(self) -> dict:
         return bar_matrix_get_info(self.handle).as_dict()

@@ -66,9 +66,9 @@ double model_bytes(const Layout &L) { return (double)L.nnz * (8 + 4) + (double)L
 // Async driver choice. The fully asynchronous single-launch kernel removes per-iteration
 // launches and host round trips, which dominate when one global iteration moves little data;
 // for large systems the per-launch kernel streams faster (fewer registers on the hot path).
-// BAR_ASYNC_MULTI=1/0 forces either.
+// bar_tuning.single_launch = 1 / -1 forces either.
 bool use_async_multi(const Layout &L) {
-    if (const char *ev = getenv("BAR_ASYNC_MULTI")) return ev[0] == '1';
+    if (L.tune.single_launch) return L.tune.single_launch > 0;
     return model_bytes(L) < 256e6;
 }
 
@@ -205,6 +205,10 @@ fail:
 
 void bar_destroy(bar_matrix A) {
     if (!A) return;
+    if (A->dist) {  // a rank's share (bar_create_csr_dist): its communicator, mappings, buffers
+        dist_destroy_handle(A);
+        return;
+    }
     DeviceGuard g(A->device);
     free_layout(A->L);
     Workspace &W = A->W;
@@ -219,6 +223,26 @@ void bar_destroy(bar_matrix A) {
     cudaFree(W.state);
     cudaFreeHost(W.h_state);
     delete A;
+}
+
+bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning) {
+    g_err.clear();
+    if (!A) {
+        set_error("NULL handle");
+        return BAR_ERR_INVALID_ARG;
+    }
+    bar_tuning t{};
+    if (tuning) t = *tuning;
+    if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 3 || t.async_queue < 0 ||
+        t.async_queue > 1 || t.lead < 0 || t.lead > 48 || t.grid_cap < 0 || t.warps < 0 || t.warps > 32 ||
+        t.halo < 0 || t.halo > 1 || t.peer > 0) {
+        set_error("bar_tuning field out of range");
+        return BAR_ERR_INVALID_ARG;
+    }
+    A->L.tune = t;
+    A->W.graph.b = nullptr;  // a captured solve may have used other kernels: capture again
+    A->W.graph.x = nullptr;
+    return BAR_OK;
 }
 
 bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info) {
@@ -249,6 +273,7 @@ bar_status bar_residual(bar_matrix A, const double *b, const double *x, void *cu
         set_error("NULL argument");
         return BAR_ERR_INVALID_ARG;
     }
+    if (A->dist) return dist_residual_handle(A, b, x, (cudaStream_t)cuda_stream, res_norm2, b_norm2);
     DeviceGuard g(A->device);
     cudaStream_t st = (cudaStream_t)cuda_stream;
     bar_status r = ensure_workspace(A);
@@ -287,6 +312,7 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
         set_error("bar_sweep takes device pointers only");
         return BAR_ERR_INVALID_ARG;
     }
+    if (A->dist) return dist_sweep_handle(A, b, x, k, nsweeps, mode, (cudaStream_t)cuda_stream);
     cudaStream_t st = (cudaStream_t)cuda_stream;
     bar_status r = ensure_workspace(A);
     if (r != BAR_OK) return r;
@@ -333,6 +359,13 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         return BAR_ERR_INVALID_ARG;
     }
     if (mode == BAR_MODE_JACOBI) k = 1;
+    if (A->dist) {  // one rank of a row-partitioned solve (collective over its group)
+        if (opts && (opts->tau != 1.0 || opts->fail_mask || opts->res_history)) {
+            set_error("bar_solve_ex options are not supported on multi-GPU handles");
+            return BAR_ERR_INVALID_ARG;
+        }
+        return dist_solve_handle(A, b, x0, x, k, max_global_iters, tol, mode, (cudaStream_t)cuda_stream, info);
+    }
     const double tau = opts ? opts->tau : 1.0;
     if (!(tau > 0.0) || !std::isfinite(tau)) {
         set_error("tau must be a positive finite number");
@@ -463,6 +496,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             else if (r0 <= tol) converged = 1;
         };
         bool used_multi = false;
+        bool fallback = false;  // the single-launch kernel aborted (blocks not co-resident)
         const long long w_end = (long long)max_global_iters * (long long)L.q;
         unsigned long long claimed_before = 0;
         long long m0 = 0;  // static-ownership single-launch kernels: restart iteration after a resume
@@ -495,6 +529,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             rel = H.exact_rel;
             if (!std::isfinite(rel) || rel > 1e30) diverged = true;
             else if (rel <= tol) converged = 1;
+            else if (H.aborted) fallback = true;  // continue below with per-launch kernels
             else if (!H.stop || (!resident && (long long)H.work_resume >= w_end)) return BAR_OK;  // max iters
             else {
                 m0 = H.iters_done;
@@ -529,10 +564,9 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 return cudaMemcpyAsync(W.h_state, W.state, sizeof(DevState), cudaMemcpyDeviceToHost, s);
             };
             SolveGraph &Gr = W.graph;
-            const char *ge = getenv("BAR_GRAPH");
             const bool same = Gr.b == db && Gr.x0 == x0 && Gr.x == buf0 && Gr.k == k &&
                               Gr.max_iters == max_global_iters && Gr.tol == tol;
-            bool use_graph = !(ge && ge[0] == '0') && !(same && Gr.unsupported);
+            bool use_graph = L.tune.graph >= 0 && !(same && Gr.unsupported);
             if (use_graph && !(same && Gr.exec)) {  // (re)capture for this call
                 if (Gr.exec) cudaGraphExecDestroy(Gr.exec);
                 Gr.exec = nullptr;
@@ -551,7 +585,9 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 if (graph) cudaGraphDestroy(graph);
                 cudaGetLastError();
                 use_graph = Gr.exec != nullptr;
+                Gr.kernel = L.last_kernel;
             }
+            if (use_graph) L.last_kernel = Gr.kernel;  // what the replayed graph launches
             cudaError_t e = use_graph ? cudaGraphLaunch(Gr.exec, st) : enqueue_first(st);
             launches += 3;
             if (e == cudaErrorNotSupported) {  // no single-launch kernel: per-launch kernels below
@@ -587,6 +623,15 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                     }
                 }
             }
+        }
+        if (fallback) {
+            // the single-launch kernel's blocks were not all resident (other work on the device):
+            // continue from the current iterate, counting from the completed global iterations
+            BAR_CUDA(launch_continue_per_launch(W.state, st));
+            ++launches;
+            if ((r = read_state(A, st)) != BAR_OK) return r;
+            used_multi = false;
+            multi = false;
         }
         if (used_multi) {
             // global iterations needed: the iteration whose fused estimate met tol (the returned

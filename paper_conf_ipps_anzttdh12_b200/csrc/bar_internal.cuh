@@ -18,6 +18,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <string>
 
 #include "bar.h"
@@ -32,7 +33,9 @@ struct DevState {
     unsigned int counter;   // last-block ticket
     int stop;               // kernels return immediately when set
     int diverged;
-    int pad0;
+    int aborted;            // k_block_resident: blocks were not co-resident (a block waited > ~2 ms
+                            // for lagging ones); every block stopped, the host continues with
+                            // per-launch kernels from the current iterate (R12)
     long long iter;         // launches that executed (sync: m of the latest x^(m) produced)
     long long conv_iter;    // sync: m with rel_res(x^(m)) <= tol
     double bnorm;           // ||b||_2
@@ -72,7 +75,8 @@ struct ChunkSizer {
             std::isfinite(rel_now)) {
             const double rate = std::pow(rel_now / rel, 1.0 / (double)(it_now - it));
             const double need = std::ceil(std::log(tol / rel_now) / std::log(rate));
-            if (rate > 0.0 && rate < 1.0 && need >= 0.0 && need < 256.0) nc = (int64_t)need + 2;
+            // (need + 2 <= KernelTimer::kMax: every launch of a chunk gets its timer events)
+            if (rate > 0.0 && rate < 1.0 && need >= 0.0 && need < 256.0) nc = std::min<int64_t>((int64_t)need + 2, 256);
         }
         it = it_now;
         rel = rel_now;
@@ -90,6 +94,9 @@ struct Layout {
     int64_t local_entries = 0;
     int max_wl = 0, max_wo = 0;
     int max_w = 0;              // widest slice: max over slices of wl + wo
+    int64_t plane_stride = 0;   // S: the farthest frequent off-block coupling of a middle subdomain,
+                                // in subdomains, when it is a whole multiple of R (3D grid: a plane);
+                                // used by the strided claim order (tuning.async_order = 3)
     int sms = 148;              // SMs of the device (persistent grids)
     // device arrays
     double *val = nullptr;      // [entries]
@@ -107,6 +114,7 @@ struct Layout {
     int32_t *dict = nullptr;    // [dptr[q]]
     int32_t *dptr = nullptr;    // [q + 1]
     int64_t dict_entries = 0;
+    bar_tuning tune{};          // explicit kernel / schedule overrides (bar_set_tuning); zero = defaults
     mutable int64_t rw_grid = -1;  // cached rowwise_grid (occupancy queries cost API round trips)
     mutable const char *last_kernel = "none";  // name of the most recently launched sweep kernel
 };
@@ -131,6 +139,7 @@ struct SolveGraph {
     cudaStream_t cap = nullptr;      // capture stream (library-private)
     cudaGraphExec_t exec = nullptr;
     bool unsupported = false;        // the key's call has no single-launch kernel: do not capture
+    const char *kernel = "none";     // the sweep kernel the graph launches (Layout::last_kernel at capture)
     const double *b = nullptr, *x0 = nullptr;
     double *x = nullptr;
     int32_t k = 0;
@@ -157,6 +166,7 @@ struct bar_matrix_s {
     int device = 0;
     bar::Layout L;
     bar::Workspace W;
+    struct bar_dist_s *dist = nullptr;  // set on handles from bar_create_csr_dist (one rank's share)
 };
 
 namespace bar {
@@ -198,6 +208,15 @@ void timer_free(KernelTimer &T);
         cudaError_t _e = (call);                                    \
         if (_e != cudaSuccess) return ::bar::cuda_fail(_e, #call);  \
     } while (0)
+
+// Handles from bar_create_csr_dist (dist.cu): the collective solve / residual of one rank.
+bar_status dist_solve_handle(bar_matrix A, const double *b, const double *x0, double *x, int32_t k,
+                             int64_t max_global_iters, double tol, bar_mode mode, cudaStream_t st, bar_solve_info *info);
+bar_status dist_residual_handle(bar_matrix A, const double *b, const double *x, cudaStream_t st, double *res_norm2,
+                                double *b_norm2);
+void dist_destroy_handle(bar_matrix A);
+bar_status dist_sweep_handle(bar_matrix A, const double *b, double *x, int32_t k, int64_t nsweeps, bar_mode mode,
+                             cudaStream_t st);
 
 // Layout construction (layout.cu). rowptr/col/val are DEVICE pointers.
 // Columns in [col_lo, col_hi) (default [0, n)); row i's diagonal is column i.
@@ -248,5 +267,7 @@ cudaError_t launch_init_check(DevState *state, cudaStream_t st);
 // reopen a closed async queue; clear_slots: also zero the per-iteration residual slots
 // (k_block_resident restarts every block at the last completed iteration)
 cudaError_t launch_resume_queue(DevState *state, cudaStream_t st, bool clear_slots = false);
+// after an aborted single-launch solve (DevState::aborted): iter = iters_done, stop / aborted cleared
+cudaError_t launch_continue_per_launch(DevState *state, cudaStream_t st);
 
 }  // namespace bar

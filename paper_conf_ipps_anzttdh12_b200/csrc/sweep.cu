@@ -19,7 +19,9 @@
 // with coalesced warp-wide loads from the sliced layout (bar_internal.cuh).
 #include <algorithm>
 #include <cstdlib>
+#include <map>
 #include <mutex>
+#include <utility>
 
 #include "bar_internal.cuh"
 #include "tma.cuh"
@@ -56,6 +58,8 @@ struct KP {
     const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
     int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
+    int32_t stride;         // > 0: strided (transposed) chunk order, S subdomains per plane (claim_at)
+    int32_t stride_q;       //   and Q = q / S planes
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
@@ -68,14 +72,32 @@ struct KP {
 // sweeps its chunk in order, so a subdomain sees this iteration's values of its predecessors in
 // the chunk: eq. 4's shift s(k+1, j) > 0, the block Gauss-Seidel flavour of P:209, on every
 // coupling shorter than the chunk). Either way each subdomain is swept exactly once per launch (R7).
+// A third order (tuning.async_order = 3, "strided"): with S = Layout::plane_stride subdomains
+// between a subdomain and its farthest frequent coupling (C5: a grid plane = 256 subdomains of
+// two lines), the chunks are cut from the TRANSPOSED sequence t = s Q + p of l = p S + s
+// (Q = q / S): a block sweeps one position s through consecutive planes p, so the plane below was
+// swept one claim earlier (Gauss-Seidel along the far coupling, its x still in L2) and the
+// plane above, read as ghosts, is the next claim's x_J.
 struct Claims {
     long long l0, step, lend;
 };
+constexpr long long kNoClaim = 0x7fffffffffffffffll;
 
 __device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
     const long long G = gridDim.x, c = blockIdx.x;
     if (p.claim_chunk) return {c * (long long)q / G, 1, (c + 1) * (long long)q / G};
     return {c, G, (long long)q};
+}
+
+// The j-th subdomain block c claims, or kNoClaim past its last.
+__device__ __forceinline__ long long claim_at(const KP &p, const Claims &C, long long j, int64_t q) {
+    const long long t = C.l0 + j * C.step;
+    if (t >= C.lend) return kNoClaim;
+    if (p.stride > 0) {  // q < 2^31: 32-bit arithmetic
+        const uint32_t tt = (uint32_t)t, Q = (uint32_t)p.stride_q;
+        return (long long)(tt % Q) * p.stride + tt / Q;
+    }
+    return t;
 }
 
 // Thread 0: start copying subdomain l's ghost-range entry (kGhostRanges pairs, 32 B) into
@@ -828,7 +850,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const Claims C = claims_of(p, q);
-    auto lof = [&](long long j) { return C.l0 + j * C.step; };
+    auto lof = [&](long long j) { return claim_at(p, C, j, q); };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto stage_bytes = [&](long long l, int64_t E0, int64_t E1) -> uint32_t {
         const int nrows = (int)min((int64_t)R, p.n - (int64_t)l * R);
@@ -839,7 +861,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // part w (0..3) of the stage of l_j (see above); one lane per warp
     auto issue_part = [&](int w, long long j, const int64_t *bd, const int32_t *gr) {
         const long long l = lof(j);
-        if (l >= C.lend) return;
+        if (l >= q) return;
         const int vs = (int)(j & 1), bs = (int)(j % 3);
         const int64_t TS = l * (int64_t)R;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
@@ -866,7 +888,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= C.lend) return;
+        if (l >= q) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -888,14 +910,14 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         fence_mbar_init();
         for (int j = 0; j < 4; ++j) {
             const long long l = lof(j);
-            if (l >= C.lend) break;
+            if (l >= q) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
         }
         for (int j = 0; j < 2; ++j) {
             const long long l = lof(j);
-            if (l >= C.lend) break;
+            if (l >= q) break;
             mbar_arrive_expect_tx(&bars[j], stage_bytes(l, bnd[j][0], bnd[j][1]));
             for (int w = 0; w < 4; ++w) issue_part(w, j, bnd[j], j == 1 && p.gr ? gsm[j] : nullptr);
         }
@@ -907,7 +929,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     for (int i = 0;; ++i) {
         const int vs = i & 1, bs = i % 3;
         const long long l = lof(i);
-        if (l >= C.lend) break;
+        if (l >= q) break;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
         const int64_t TS = l * (int64_t)R;
@@ -969,7 +991,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         }
         // post the byte count of l_{i+2}'s stage before the barrier that frees its buffers, so
         // that no copy of it can complete bytes before its phase expects them
-        if (threadIdx.x == 0 && lof(i + 2) < C.lend) {
+        if (threadIdx.x == 0 && lof(i + 2) < q) {
             const int r = (i + 2) & 3;
             mbar_arrive_expect_tx(&bars[(i + 2) % 3], stage_bytes(lof(i + 2), bnd[r][0], bnd[r][1]));
         }
@@ -1052,7 +1074,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     double *ya = reinterpret_cast<double *>(smraw + g.o_ya);
     double *yb = reinterpret_cast<double *>(smraw + g.o_yb);
     const Claims C = claims_of(p, q);
-    auto lof = [&](long long j) { return C.l0 + j * C.step; };
+    auto lof = [&](long long j) { return claim_at(p, C, j, q); };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto slab_bytes = [&](long long l, const int64_t *bd, const int32_t *db) -> uint32_t {
         const uint32_t nsl = (uint32_t)nsl_of(l);
@@ -1063,7 +1085,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
     auto issue_part = [&](int w, long long j) {
         const long long l = lof(j);
-        if (l >= C.lend) return;
+        if (l >= q) return;
         const int64_t *bd = bnd[j & 3];
         if (w == 3) {  // what l_j's first phase reads directly: b_J, x_J and its ghost x ranges
             const int64_t TS = l * (int64_t)R;
@@ -1098,7 +1120,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= C.lend) return;
+        if (l >= q) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -1126,7 +1148,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         fence_mbar_init();
         for (int j = 0; j < 3; ++j) {
             const long long l = lof(j);
-            if (l >= C.lend) break;
+            if (l >= q) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
@@ -1144,7 +1166,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     double rr = 0.0, bb = 0.0;
     for (int i = 0;; ++i) {
         const long long l = lof(i);
-        if (l >= C.lend) break;
+        if (l >= q) break;
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
@@ -1203,7 +1225,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             bb += bi * bi;
         }
         // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
-        if (threadIdx.x == 0 && lof(i + 1) < C.lend)
+        if (threadIdx.x == 0 && lof(i + 1) < q)
             mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3], dbd[(i + 1) & 3]));
         __syncthreads();
         if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
@@ -1661,8 +1683,12 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // loads), k local sweeps, relaxed write-back of x_J, residual publication for iteration m
 // (iteration_publish: the block completing iteration m evaluates rel_res_m and stops the solve).
 // Blocks stop on the stop flag (read one iteration ahead, so its latency is hidden) or after
-// max_global_iters sweeps; state->res_sweeps counts the sweeps for the host's accounting. A block may run at most 48 iterations ahead of the
-// last completed one (the 64 residual slots; P:109's bounded delay), spinning otherwise.
+// max_global_iters sweeps; state->res_sweeps counts the sweeps for the host's accounting. A block
+// may run at most p.lead (<= 48) iterations ahead of the last completed one (the 64 residual
+// slots; P:109's bounded delay), waiting otherwise. The kernel relies on all q blocks being
+// resident at once; if they are not (other work on the device holds SMs), a waiting block
+// times out after ~2 ms, raises state->aborted and the stop flag, every block exits, and the
+// host continues the solve from the current iterate with per-launch kernels (R12).
 template <int WLR>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_resident(KP p) {
     extern __shared__ __align__(128) unsigned char smraw[];
@@ -1731,24 +1757,23 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
     long long done_ld = p.m0;  // thread 0: iters_done, loaded one iteration ahead of its use
     unsigned long long sweeps = 0;
-    int unpaced = 0;  // thread 0: gave up waiting for lagging blocks (see below)
     for (long long m = p.m0;; ++m) {
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
             // bounded lead over the last completed iteration (p.lead sweeps; residual slots are
             // reused mod 64). The lead is checked against iters_done as loaded one iteration ago
-            // and only re-read (waited on) when exceeded. The wait is itself bounded (~2 ms): if
-            // other work on the device keeps some blocks from being resident, this block goes on
-            // iterating without publishing residuals (unpaced) instead of waiting for them
-            // forever; the solve then ends at max_global_iters and the exact residual decides.
-            if (g && !unpaced && m - done_ld > p.lead) {
-                const long long t0c = clock64();
+            // and only re-read (waited on) when exceeded. The wait is itself bounded (~2 ms of
+            // %globaltimer): a lagging block that long behind is not resident, so the launch gives
+            // up (aborted + stop) instead of waiting on work that cannot run
+            if (g && m - done_ld > p.lead) {
+                const unsigned long long t0c = globaltimer_ns();
                 while (g && m - *(volatile long long *)&p.state->iters_done > p.lead) {
                     if (*(volatile int *)&p.state->stop) g = 0;
-                    if (clock64() - t0c > 4000000ll) {
-                        unpaced = 1;
-                        break;
+                    else if (globaltimer_ns() - t0c > 2000000ull) {
+                        atomicExch(&p.state->aborted, 1);
+                        atomicExch(&p.state->stop, 1);
+                        g = 0;
                     }
                 }
             }
@@ -1803,7 +1828,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             const int W = blockDim.x >> 5;
             double a0 = 0.0;
             for (int w = 0; w < W; ++w) a0 += sred[0][w];
-            if (!unpaced) iteration_publish(p, m, 1u, a0, bsum, q);
+            iteration_publish(p, m, 1u, a0, bsum, q);
             stop_seen = stop_ld;
         }
     }
@@ -1922,6 +1947,7 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->counter = 0;
     S->stop = 0;
     S->diverged = 0;
+    S->aborted = 0;
     S->iter = 0;
     S->conv_iter = -1;
     S->tol = tol;
@@ -1956,24 +1982,65 @@ KP make_kp(const Layout &L) {
     // measured on B200 (round 1, tools/kernel_ab.py): the L2 prefetch of the gather ranges pays
     // for large subdomains (C5, R = 1024: 2.78 vs 2.87 ms per sync-block-(5) launch) and costs
     // for small ones (C4, R = 128: 0.45 vs 0.41 ms), whose ranges are 1 KB
-    p.gr = (getenv("BAR_NO_GHOST_PREFETCH") || L.R < 512) ? nullptr : L.gr;
+    const int gp = L.tune.ghost_prefetch;
+    p.gr = (gp ? gp > 0 : L.R >= 512) ? L.gr : nullptr;
+    p.grid_cap = L.tune.grid_cap > 0 ? L.tune.grid_cap : 0;
     return p;
+}
+
+// Launch caches per (kernel, device): the dynamic shared-memory attribute (cudaFuncSetAttribute
+// applies to the current device only) and the occupancy query results. Guarded by g_launch_mu.
+struct FnState {
+    size_t attr = 0, c_smem = 0;
+    int c_threads = 0, occ = 0;
+};
+std::map<std::pair<const void *, int>, FnState> g_fn;
+
+FnState &fn_state(const void *fn) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        cudaGetLastError();
+        dev = 0;
+    }
+    return g_fn[{fn, dev}];
+}
+
+template <class F>
+cudaError_t ensure_smem(F *fn, size_t smem) {
+    FnState &s = fn_state(reinterpret_cast<const void *>(fn));
+    if (smem > s.attr) {
+        cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        s.attr = smem;
+    }
+    return cudaSuccess;
+}
+
+// Co-resident blocks of fn per SM at (threads, smem); 0 if the query fails or nothing fits.
+template <class F>
+int occupancy(F *fn, int threads, size_t smem) {
+    FnState &s = fn_state(reinterpret_cast<const void *>(fn));
+    if (s.c_smem != smem || s.c_threads != threads) {
+        int o = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, fn, threads, smem) != cudaSuccess) {
+            cudaGetLastError();
+            o = 0;
+        }
+        s.occ = o;
+        s.c_smem = smem;
+        s.c_threads = threads;
+    }
+    return s.occ;
 }
 
 template <bool ASYNC, bool STAGE>
 cudaError_t launch_block_t(const KP &p, int threads, size_t smem, unsigned grid, cudaStream_t st) {
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaError_t e =
-            cudaFuncSetAttribute(k_block<ASYNC, STAGE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr = smem;
-    }
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(k_block<ASYNC, STAGE>, smem);
+    if (e != cudaSuccess) return e;
     k_block<ASYNC, STAGE><<<grid, threads, smem, st>>>(p);
     return cudaGetLastError();
 }
-
 
 // Block geometry: one 32-row slice per warp and pass; local entries staged in shared memory
 // when they fit (otherwise re-read through L1/L2 in every sweep).
@@ -1993,43 +2060,29 @@ cudaError_t launch_reg_w(const KP &p, const Layout &L, cudaStream_t st) {
 
 template <bool ASYNC, int WLR>
 cudaError_t launch_reg_tma_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaError_t e =
-            cudaFuncSetAttribute(k_reg_tma<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr = smem;
-    }
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(k_reg_tma<ASYNC, WLR>, smem);
+    if (e != cudaSuccess) return e;
     k_reg_tma<ASYNC, WLR><<<(unsigned)L.q, L.spb * kSlice, smem, st>>>(p);
     return cudaGetLastError();
 }
 
-// Persistent grid of k_block_pers: every block that fits on the device at once.
-template <bool ASYNC, int WLR>
-int64_t pers_grid(const Layout &L, size_t smem) {
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr = 0;
-    if (smem > attr) {
-        if (cudaFuncSetAttribute(k_block_pers<ASYNC, WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-            cudaSuccess)
-            return -1;
-        attr = smem;
-    }
-    int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_block_pers<ASYNC, WLR>, L.spb * kSlice, smem) !=
-            cudaSuccess ||
-        per_sm < 1)
-        per_sm = 1;
-    const int64_t g = (int64_t)per_sm * L.sms;
+// Persistent grid: every block that fits on the device at once (at least one per SM), capped by
+// the subdomain count and the tuning's grid cap.
+int64_t persistent_grid(int per_sm, const KP &p, const Layout &L) {
+    int64_t g = (int64_t)(per_sm < 1 ? 1 : per_sm) * L.sms;
+    if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
     return g < L.q ? g : L.q;
 }
 
 template <bool ASYNC, int WLR>
 cudaError_t launch_pers_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
-    const int64_t g = pers_grid<ASYNC, WLR>(L, smem);
-    if (g < 0) return cudaGetLastError();
-    k_block_pers<ASYNC, WLR><<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    auto kfn = k_block_pers<ASYNC, WLR>;
+    cudaError_t e = ensure_smem(kfn, smem);
+    if (e != cudaSuccess) return e;
+    const int64_t g = persistent_grid(occupancy(kfn, L.spb * kSlice, smem), p, L);
+    kfn<<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -2038,26 +2091,10 @@ cudaError_t launch_stage_m(const KP &p, const Layout &L, size_t smem, cudaStream
     const bool ext = !MULTI && (p.frozen != nullptr || p.tau != 1.0);  // N1 / N3 requested
     auto kfn = MULTI ? k_block_stage_m<true, WLR, true>
                      : (ext ? k_block_stage<ASYNC, WLR, true> : k_block_stage<ASYNC, WLR, false>);
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr[2] = {0, 0};
-    static size_t c_smem[2] = {0, 0};
-    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
-    const int v = ext ? 1 : 0;
-    if (smem > attr[v]) {
-        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr[v] = smem;
-    }
-    if (c_smem[v] != smem || c_threads[v] != L.spb * kSlice) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, L.spb * kSlice, smem) != cudaSuccess ||
-            occ[v] < 1)
-            occ[v] = 1;
-        c_smem[v] = smem;
-        c_threads[v] = L.spb * kSlice;
-    }
-    const int per_sm = occ[v];
-    int64_t g = (int64_t)per_sm * L.sms;
-    if (g > L.q) g = L.q;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(kfn, smem);
+    if (e != cudaSuccess) return e;
+    const int64_t g = persistent_grid(occupancy(kfn, L.spb * kSlice, smem), p, L);
     KP pp = p;
     // a block prefetches x_J two claims ahead; with fewer than ~3 claims of other blocks in
     // between, that could predate the subdomain's own previous update
@@ -2070,26 +2107,10 @@ template <bool ASYNC, int WLR>
 cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
     auto kfn = ext ? k_block_pipe<ASYNC, WLR, true> : k_block_pipe<ASYNC, WLR, false>;
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr[2] = {0, 0};
-    static size_t c_smem[2] = {0, 0};
-    static int c_threads[2] = {0, 0}, occ[2] = {0, 0};
-    const int v = ext ? 1 : 0;
-    if (smem > attr[v]) {
-        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr[v] = smem;
-    }
-    if (c_smem[v] != smem || c_threads[v] != L.spb * kSlice) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, L.spb * kSlice, smem) != cudaSuccess ||
-            occ[v] < 1)
-            occ[v] = 1;
-        c_smem[v] = smem;
-        c_threads[v] = L.spb * kSlice;
-    }
-    int64_t g = (int64_t)occ[v] * L.sms;
-    if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
-    if (g > L.q) g = L.q;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(kfn, smem);
+    if (e != cudaSuccess) return e;
+    const int64_t g = persistent_grid(occupancy(kfn, L.spb * kSlice, smem), p, L);
     kfn<<<(unsigned)g, L.spb * kSlice, smem, st>>>(p);
     return cudaGetLastError();
 }
@@ -2100,65 +2121,36 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     const bool coded = p.codes != nullptr;
     auto kfn = coded ? (ext ? k_block_duo<ASYNC, WLR, true, true> : k_block_duo<ASYNC, WLR, false, true>)
                      : (ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>);
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr[4] = {0, 0, 0, 0};
-    static size_t c_smem[4] = {0, 0, 0, 0};
-    static int c_threads[4] = {0, 0, 0, 0}, occ[4] = {0, 0, 0, 0};
-    const int v = (ext ? 1 : 0) + (coded ? 2 : 0);
     const int threads = L.spb / 2 * kSlice;
-    if (smem > attr[v]) {
-        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr[v] = smem;
-    }
-    if (c_smem[v] != smem || c_threads[v] != threads) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[v], kfn, threads, smem) != cudaSuccess || occ[v] < 1)
-            occ[v] = 1;
-        c_smem[v] = smem;
-        c_threads[v] = threads;
-    }
-    int64_t g = (int64_t)occ[v] * L.sms;
-    if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
-    if (g > L.q) g = L.q;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(kfn, smem);
+    if (e != cudaSuccess) return e;
+    const int64_t g = persistent_grid(occupancy(kfn, threads, smem), p, L);
     kfn<<<(unsigned)g, threads, smem, st>>>(p);
     return cudaGetLastError();
 }
 
 // k_block_resident for a single-launch async solve when all q subdomains fit on the device at
-// once (grid = q blocks co-resident); BAR_RESIDENT=0 keeps the work-queue kernel.
+// once (grid = q blocks co-resident); tuning.resident = -1 keeps the work-queue kernel.
 template <int WLR>
 bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_t &err) {
-    const char *re = getenv("BAR_RESIDENT");
-    if (re && re[0] == '0') return false;
+    if (L.tune.resident < 0) return false;
     const int threads = L.spb * kSlice;
     const size_t smem = 2 * (size_t)L.R * sizeof(double) + (size_t)L.max_w * threads * 12;
     if (smem > kSmemMax) return false;
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr = 0;
-    static size_t c_smem = 0;
-    static int c_threads = 0, occ = 0;
-    if (smem > attr) {
-        if (cudaFuncSetAttribute(k_block_resident<WLR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-            cudaSuccess) {
-            cudaGetLastError();
-            return false;
-        }
-        attr = smem;
-    }
-    if (c_smem != smem || c_threads != threads) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_block_resident<WLR>, threads, smem) != cudaSuccess)
-            occ = 0;
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    if (ensure_smem(k_block_resident<WLR>, smem) != cudaSuccess) {
         cudaGetLastError();
-        c_smem = smem;
-        c_threads = threads;
+        return false;
     }
-    if ((int64_t)occ * L.sms < L.q) return false;  // every subdomain's block must be co-resident
+    // every subdomain's block must fit at once (if other work keeps some of them from being
+    // resident, the kernel aborts and the host continues with per-launch kernels: DESIGN.md R12)
+    if ((int64_t)occupancy(k_block_resident<WLR>, threads, smem) * L.sms < L.q) return false;
     L.last_kernel = "k_block_resident<async>";
     // lead 3 (B200, round 1, tools/kernel_ab.py): C2 51 vs 56-59 global iterations with lead 40
     // (0.29 vs 0.33 ms), C3 0.205 vs 0.217 ms; blocks racing far ahead sweep on stale ghosts
     KP pp = p;
-    pp.lead = 3;
-    if (const char *le = getenv("BAR_LEAD")) pp.lead = std::max(1, std::min(48, atoi(le)));
+    pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 3;
     k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(pp);
     err = cudaGetLastError();
     return true;
@@ -2169,6 +2161,7 @@ cudaError_t launch_stage_t(const KP &p, const Layout &L, size_t smem, cudaStream
     if (ASYNC && p.w_end > 0) {
         cudaError_t e = cudaSuccess;
         if (launch_resident_t<WLR>(p, L, st, e)) return e;
+        L.last_kernel = "k_block_stage_m<async>";
         return launch_stage_m<true, WLR, true>(p, L, smem, st);
     }
     return launch_stage_m<ASYNC, WLR, false>(p, L, smem, st);
@@ -2194,29 +2187,28 @@ bool staged_ok(const KP &p, const Layout &L) {
 //   k_block_pers   persistent, double-buffered TMA slice stream
 //   k_reg_tma  subdomains of <= 1024 rows with <= 8 local entries per row: TMA-streamed slices,
 //              register-resident local entries
-//   k_reg      same without TMA (BAR_KERNEL=r, for comparison)
+//   k_reg      same without TMA (tuning.kernel = 2, for comparison)
 //   k_block    anything else: local entries staged in shared memory when they fit, else
-//              re-read through L1/L2 each sweep (BAR_KERNEL=s forces it)
+//              re-read through L1/L2 each sweep (tuning.kernel = 1 forces it)
+// The choice depends only on the layout, the vectors' alignment and the handle's bar_tuning.
 template <bool ASYNC>
 cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
-    const char *kv = getenv("BAR_KERNEL");
-    const char kind = kv ? kv[0] : 't';
+    const bar_tuning &T = L.tune;
+    const int kind = T.kernel;  // 0 auto, 1 k_block, 2 k_reg, 3 k_reg_tma, 4 k_block_pers
     p.wlmax = L.max_wl;
     p.wmax = L.max_w;
-    // async subdomain order of the per-launch kernels: static round robin (block c sweeps c,
-    // c + G, ...) by default. Measured on B200 (round 1): the device work queue's atomic claims
-    // cost 0.6 ms/iteration on some boxes (C5 k=5: 3.57 vs 2.91 ms) and converged no faster
-    // (59 vs 57 global iterations). BAR_ASYNC_STATIC=0 selects the queue.
-    const char *sc = getenv("BAR_ASYNC_STATIC");
-    p.static_claims = !(sc && sc[0] == '0');
-    if (const char *ge = getenv("BAR_GRID")) p.grid_cap = atoi(ge);  // tuning: cap persistent grids
+    // async subdomain order of the per-launch kernels: static claims by default. Measured on
+    // B200 (round 1): the device work queue's atomic claims cost 0.6 ms/iteration on some boxes
+    // (C5 k=5: 3.57 vs 2.91 ms) and converged no faster (59 vs 57 global iterations).
+    p.static_claims = T.async_queue != 1;
     // async claim order of k_block_pipe / k_block_duo: contiguous chunks by default. Measured on
     // B200 (round 1, tools/kernel_ab.py, async-(5) to 1e-10): C5 (R = 1024) 44 global iterations
     // vs 59 with round robin, C4 (R = 512) 63 vs 105 — each block sweeps its chunk in order, so
     // the neighbouring lines / planes below a subdomain already hold this iteration's values.
-    // BAR_ORDER=r/c overrides (sync modes: the order does not change the iterates; round robin)
-    p.claim_chunk = ASYNC ? 1 : 0;
-    if (const char *oe = getenv("BAR_ORDER")) p.claim_chunk = oe[0] == 'c';
+    // (sync modes: the order does not change the iterates; round robin)
+    p.claim_chunk = T.async_order == 0 ? (ASYNC ? 1 : 0) : (T.async_order != 2 ? 1 : 0);
+    p.stride = (T.async_order == 3 && L.plane_stride > 0 && L.q % L.plane_stride == 0) ? (int32_t)L.plane_stride : 0;
+    p.stride_q = p.stride ? (int32_t)(L.q / p.stride) : 1;
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
@@ -2230,27 +2222,23 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // for sync-block (C5: 2.64 vs 3.51 ms/iteration) and, since async claims are static (no
     // work-queue atomic on the issuing thread), for async and Jacobi with R >= 256 too (C5:
     // 2.65 vs 3.35 and 2.58 vs 2.69 ms; C4 at R = 256: 0.38 vs 0.42 ms); with R = 128 (C4) the
-    // one-ahead kernel is 2% faster for async. BAR_PIPE=0/1 overrides
-    const char *pe = getenv("BAR_PIPE");
-    const bool pipe_on = (pe ? pe[0] == '1' : ((!ASYNC && p.k >= 3) || L.R >= 256)) &&
+    // one-ahead kernel is 2% faster for async.
+    const bool pipe_on = (T.pipe ? T.pipe > 0 : ((!ASYNC && p.k >= 3) || L.R >= 256)) &&
                          (!ASYNC || p.static_claims);  // the pipeline claims statically
     // two-blocks-per-SM variant (k_block_duo) where the pipelined kernel holds a whole SM (C5
     // sync modes, B200 round 1, tools/kernel_ab.py: Jacobi 2.45 vs 2.58 ms, sync-block-(5) 2.56-2.67
-    // vs 2.67 ms per launch); BAR_DUO=0/1 overrides
-    // coded columns (Layout::codes, 1 byte per entry instead of 4) for the duo kernel when the
-    // layout has them; BAR_CODED=0 reads the int32 columns instead
-    const char *ce = getenv("BAR_CODED");
-    const bool coded = L.codes != nullptr && !(ce && ce[0] == '0');
+    // vs 2.67 ms per launch); coded columns (Layout::codes, 1 byte per entry instead of 4) when
+    // the layout has them
+    const bool coded = L.codes != nullptr && T.coded >= 0;
     const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w, coded).bytes;
-    const char *de = getenv("BAR_DUO");
     const bool duo_fits = L.spb % 2 == 0 && L.spb >= 8 && L.max_wl <= 4 && 2 * (duo_smem + 2048) <= 228 * 1024;
     // Async: two blocks per SM whenever they fit (C5 R = 1024: 2.69 vs 2.93 ms per launch with
     // chunked claims; C4 R = 512: 0.40 vs 0.52 ms). With round-robin claims the 2 x 148
     // subdomains in flight (303K rows on C5) exceeded the plane coupling distance (262K) and cost
     // global iterations (63 vs 59); chunked claims do not depend on the window.
-    const bool duo_on = (de ? de[0] == '1' : ((ASYNC && p.claim_chunk) || pipe_smem > 113 * 1024)) && duo_fits &&
+    const bool duo_on = (T.duo ? T.duo > 0 : ((ASYNC && p.claim_chunk) || pipe_smem > 113 * 1024)) && duo_fits &&
                         (!ASYNC || p.static_claims);
-    if (kind == 't' && duo_on && p.w_end == 0 && geom_ok && aligned) {
+    if (kind == 0 && duo_on && p.w_end == 0 && geom_ok && aligned) {
         L.last_kernel = coded ? (ASYNC ? "k_block_duo<async,coded>" : "k_block_duo<sync,coded>")
                               : (ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>");
         KP pc = p;
@@ -2261,7 +2249,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         }
         return launch_duo_t<ASYNC, 4>(pc, L, duo_smem, st);  // two rows per thread: <= 4 local entries
     }
-    if (kind == 't' && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
+    if (kind == 0 && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
         L.last_kernel = ASYNC ? "k_block_pipe<async>" : "k_block_pipe<sync>";
         if (L.max_wl <= 4) return launch_pipe_t<ASYNC, 4>(p, L, pipe_smem, st);
         if (L.max_wl <= 6) return launch_pipe_t<ASYNC, 6>(p, L, pipe_smem, st);
@@ -2269,8 +2257,8 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         if (L.max_wl <= 12) return launch_pipe_t<ASYNC, 12>(p, L, pipe_smem, st);  // <= 512 threads
         return launch_pipe_t<ASYNC, 16>(p, L, pipe_smem, st);
     }
-    if (kind == 't' && geom_ok && aligned && stage_smem <= kSmemMax) {
-        L.last_kernel = p.w_end > 0 ? "k_block_stage_m<async>" : ASYNC ? "k_block_stage<async>" : "k_block_stage<sync>";
+    if (kind == 0 && geom_ok && aligned && stage_smem <= kSmemMax) {
+        L.last_kernel = ASYNC ? "k_block_stage<async>" : "k_block_stage<sync>";
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
         if (L.max_wl <= 6) return launch_stage_t<ASYNC, 6>(p, L, stage_smem, st);
         if (L.max_wl <= 8) return launch_stage_t<ASYNC, 8>(p, L, stage_smem, st);
@@ -2279,19 +2267,19 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     }
     if (p.w_end > 0) return cudaErrorNotSupported;  // no persistent multi-iteration kernel here
     const bool ext = p.frozen != nullptr || p.tau != 1.0;  // N1/N3: only k_block_stage and k_block
-    if (!ext && (kind == 't' || kind == 'p') && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
+    if (!ext && (kind == 0 || kind == 4) && L.spb <= 32 && L.max_wl <= 8 && pers_smem <= kSmemBudget) {
         L.last_kernel = ASYNC ? "k_block_pers<async>" : "k_block_pers<sync>";
         if (L.max_wl <= 4) return launch_pers_t<ASYNC, 4>(p, L, pers_smem, st);
         if (L.max_wl <= 6) return launch_pers_t<ASYNC, 6>(p, L, pers_smem, st);
         return launch_pers_t<ASYNC, 8>(p, L, pers_smem, st);
     }
-    if (!ext && (kind == 't' || kind == 'n') && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
+    if (!ext && (kind == 0 || kind == 3) && L.spb <= 32 && L.max_wl <= 8 && tma_smem <= kSmemBudget) {
         L.last_kernel = ASYNC ? "k_reg_tma<async>" : "k_reg_tma<sync>";
         if (L.max_wl <= 4) return launch_reg_tma_t<ASYNC, 4>(p, L, tma_smem, st);
         if (L.max_wl <= 6) return launch_reg_tma_t<ASYNC, 6>(p, L, tma_smem, st);
         return launch_reg_tma_t<ASYNC, 8>(p, L, tma_smem, st);
     }
-    if (!ext && kind != 's' && L.spb <= 32 && L.max_wl <= 8) {
+    if (!ext && kind != 1 && L.spb <= 32 && L.max_wl <= 8) {
         L.last_kernel = ASYNC ? "k_reg<async>" : "k_reg<sync>";
         return launch_reg_w<ASYNC, 1>(p, L, st);
     }
@@ -2301,10 +2289,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const bool stage = row_bytes + stage_bytes <= kSmemBudget;
     const size_t smem = row_bytes + (stage ? stage_bytes : 0);
     int W = L.spb < 32 ? L.spb : 32;
-    if (const char *ev = getenv("BAR_WARPS")) {
-        int w = atoi(ev);
-        if (w >= 1 && w <= 32) W = w < L.spb ? w : L.spb;
-    }
+    if (T.warps >= 1 && T.warps <= 32) W = T.warps < L.spb ? T.warps : L.spb;
     if (stage) return launch_block_t<ASYNC, true>(p, W * 32, smem, (unsigned)L.q, st);
     return launch_block_t<ASYNC, false>(p, W * 32, smem, (unsigned)L.q, st);
 }
@@ -2316,22 +2301,18 @@ bool rowwise_tma_ok(const Layout &L) { return 16 * (size_t)slice_buf_bytes(L.max
 template <bool RES>
 cudaError_t launch_rowwise(KP p, const Layout &L, cudaStream_t st) {
     p.wmax = L.max_w;
-    const char *kv = getenv("BAR_KERNEL");
-    if (!rowwise_tma_ok(L) || (kv && kv[0] == 'r')) {
+    if (!rowwise_tma_ok(L) || L.tune.kernel == 2) {
         if (!RES) L.last_kernel = "k_rowwise<jacobi>";
         k_rowwise<RES><<<(unsigned)((L.nslices + 7) / 8), 256, 0, st>>>(p);
         return cudaGetLastError();
     }
     const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
-    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);  // the static caches below
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_rowwise_tma<RES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr = smem;
-    }
+    const int64_t grid = rowwise_grid(L);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
+    cudaError_t e = ensure_smem(k_rowwise_tma<RES>, smem);
+    if (e != cudaSuccess) return e;
     if (!RES) L.last_kernel = "k_rowwise_tma<jacobi>";
-    k_rowwise_tma<RES><<<(unsigned)rowwise_grid(L), 256, smem, st>>>(p);
+    k_rowwise_tma<RES><<<(unsigned)grid, 256, smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -2342,14 +2323,13 @@ int64_t rowwise_grid(const Layout &L) {
     const int64_t groups = (L.nslices + 7) / 8;
     if (!rowwise_tma_ok(L)) return L.rw_grid = groups;
     const size_t smem = 16 * (size_t)slice_buf_bytes(L.max_w);
+    std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
     int a = 0, b = 0;
-    cudaFuncSetAttribute(k_rowwise_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBudget);
-    cudaFuncSetAttribute(k_rowwise_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBudget);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, k_rowwise_tma<true>, 256, smem) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_rowwise_tma<false>, 256, smem) != cudaSuccess) {
-        cudaGetLastError();
-        a = b = 1;
+    if (ensure_smem(k_rowwise_tma<true>, smem) == cudaSuccess && ensure_smem(k_rowwise_tma<false>, smem) == cudaSuccess) {
+        a = occupancy(k_rowwise_tma<true>, 256, smem);
+        b = occupancy(k_rowwise_tma<false>, 256, smem);
     }
+    cudaGetLastError();
     int64_t per_sm = a < b ? a : b;  // the same grid for both (deterministic reductions)
     if (per_sm < 1) per_sm = 1;
     const int64_t g = per_sm * L.sms;
@@ -2380,8 +2360,7 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     if (mode == BAR_MODE_JACOBI) {
         // Jacobi (eq. 2) is sync-block-(1) for any R, with the same per-row arithmetic
         // (off-block entries, then local ones, diagonal included): use the staged stream
-        const char *jv = getenv("BAR_JACOBI_ROWWISE");
-        if (!(jv && jv[0] == '1') && staged_ok(p, *a.L)) {
+        if (a.L->tune.jacobi_rowwise != 1 && staged_ok(p, *a.L)) {
             p.k = 1;
             return launch_block<false>(p, *a.L, st);
         }
@@ -2490,6 +2469,21 @@ cudaError_t launch_zero_start_residual(const Layout &L, const double *b, DevStat
 }
 
 __global__ void k_init_check(DevState *S) { init_check_rule(S); }
+
+// After an aborted single-launch solve: continue counting global iterations from the completed
+// ones with per-launch kernels (S->iter is the per-launch kernels' counter).
+__global__ void k_continue_per_launch(DevState *S) {
+    S->iter = S->iters_done;
+    S->stop = 0;
+    S->aborted = 0;
+    S->counter = 0;
+    S->work = 0;
+}
+
+cudaError_t launch_continue_per_launch(DevState *state, cudaStream_t st) {
+    k_continue_per_launch<<<1, 1, 0, st>>>(state);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_init_check(DevState *state, cudaStream_t st) {
     k_init_check<<<1, 1, 0, st>>>(state);

@@ -27,6 +27,7 @@ def test_reference_arm_line():
     assert d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
     assert d["config"]["workload"].startswith("c1")
+    assert d["extrapolated"] is False and d["oracle_iters"] == 28  # a full oracle sync-block-(5) solve
 
 
 @pytest.mark.gpu
@@ -45,6 +46,8 @@ def test_our_arm_line(bar):
     c = d["cpu_baseline"]
     assert c["kind"] == "oracle" and c["cores"] == 1 and c["value"] > 0 and c["sample"]
     assert c["jacobi"]["iters"] == 137 and c["gauss_seidel"]["iters"] == 14  # SURVEY P12 counts
+    assert c["sync_block_5"]["iters"] == 28 and d["oracle_iters"] == 28 and not c["extrapolated"]
+    assert d["partitioned_1rank"]["converged"] and d["lead_48"]["global_iters"] > 0
     e = d["e2e"]
     assert e["h2d_bytes_per_step"] == 8 * 2000 and e["d2h_bytes_per_step"] == 8 * 2000 and e["value"] > 0
     assert d["clocks"]["sm_max_mhz"]

@@ -20,10 +20,10 @@ def _split(gen, args, n, R, P):
     return [gen(*args, row_lo=a, row_hi=b) for a, b in D.partition(n, R, P)]
 
 
-def _single(bar, A, b, R, k, mode, iters, tol, x0):
+def _single(bar, A, b, R, k, mode, iters, tol, x0, tuning=None):
     import torch
 
-    M = bar.Matrix.from_csr(A, R)
+    M = bar.Matrix.from_csr(A, R, tuning=tuning)
     x = torch.empty(A.n, dtype=torch.float64, device="cuda")
     _, info = M.solve(torch.from_numpy(b).cuda(), torch.from_numpy(x0).cuda(), x, k=k, max_global_iters=iters,
                       tol=tol, mode=mode)
@@ -31,12 +31,12 @@ def _single(bar, A, b, R, k, mode, iters, tol, x0):
     return x.cpu().numpy(), info
 
 
-def _loop(blocks, n, R, b, k, mode, iters, tol, x0):
+def _loop(blocks, n, R, b, k, mode, iters, tol, x0, tuning=None):
     import torch
 
     from paper_conf_ipps_anzttdh12_b200 import dist as D
 
-    G = D.LoopbackGroup(blocks, n, R)
+    G = D.LoopbackGroup(blocks, n, R, tuning=tuning)
     bs = [torch.from_numpy(b[a:c].copy()).cuda() for a, c in G.ranges]
     x0s = [torch.from_numpy(x0[a:c].copy()).cuda() for a, c in G.ranges]
     xs, info = G.solve(bs, x0s, None, k=k, max_global_iters=iters, tol=tol, mode=mode)
@@ -102,9 +102,8 @@ def test_partitioned_async_p2p(bar, name, gen, args, R, P):
     G.close()
     assert info["converged"] and info["rel_res"] <= 1e-10
     assert O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
-    # no collective exchange inside the iteration: 4 launches per rank per global iteration
-    # (pull, sweep, publish, estimate), plus the confirming exchange/residual; the chunk sizes the
-    # ranks agree on (agree_stop) keep the launches queued past the stop to a few per rank
+    # no collective exchange inside the iteration: 3 launches per rank per global iteration
+    # (pull, sweep, publish + estimate), plus the confirming barriers / pull / residual
     assert info["iters"] > 0
     assert info["kernel_launches"] <= 4 * P * (info["iters"] + 12) + 16 * P, (info["kernel_launches"], info["iters"])
 
@@ -125,11 +124,11 @@ def test_plan_errors(bar):
 
 
 @pytest.mark.parametrize("P", [2, 3])
-def test_partitioned_duo_coded(bar, monkeypatch, P):
+def test_partitioned_duo_coded(bar, P):
     """The two-blocks-per-SM kernel with coded columns on rank-local layouts (ghost columns below
     the owned block are negative local indices, the offsets d = col - row stay valid): sync-block
     and Jacobi bitwise the one-GPU iterates, async (chunked claims) converges."""
-    monkeypatch.setenv("BAR_DUO", "1")
+    tune = {"duo": 1}
     gen, args, R = W.stencil7_3d, (128,), 256  # two grid lines per subdomain: <= 4 local entries
     A = gen(*args)
     n = A.n
@@ -137,21 +136,21 @@ def test_partitioned_duo_coded(bar, monkeypatch, P):
     x0 = np.random.default_rng(7).uniform(-1, 1, n)
     blocks = _split(gen, args, n, R, P)
     for mode, k in (("sync-block", 5), ("jacobi", 1)):
-        xs, _ = _single(bar, A, b, R, k, mode, 3, 0.0, x0)
-        xp, _ = _loop(blocks, n, R, b, k, mode, 3, 0.0, x0)
+        xs, _ = _single(bar, A, b, R, k, mode, 3, 0.0, x0, tuning=tune)
+        xp, _ = _loop(blocks, n, R, b, k, mode, 3, 0.0, x0, tuning=tune)
         assert np.array_equal(xs, xp), mode
-    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n))
+    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n), tuning=tune)
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
 
 
 @pytest.mark.parametrize("name,gen,args,R", MATS)
 @pytest.mark.parametrize("P", [2, 3])
-def test_halo_allgather_bitwise(bar, monkeypatch, name, gen, args, R, P):
-    """The ncclAllGather halo exchange (BAR_HALO=allgather, SURVEY §8(e)'s primary design; here
+def test_halo_allgather_bitwise(bar, name, gen, args, R, P):
+    """The ncclAllGather halo exchange (bar_tuning.halo = 1, SURVEY §8(e)'s primary design; here
     through the loopback transport's emulation of the gather): every rank's whole send buffer is
     gathered and each receiver copies its segments out, so sync-block and Jacobi iterates stay
     bitwise the one-GPU iterates, as with the grouped send/recv exchange."""
-    monkeypatch.setenv("BAR_HALO", "allgather")
+    tune = {"halo": "allgather"}
     A = gen(*args)
     n = A.n
     b = np.ones(n)
@@ -159,7 +158,174 @@ def test_halo_allgather_bitwise(bar, monkeypatch, name, gen, args, R, P):
     blocks = _split(gen, args, n, R, P)
     for mode, k in (("sync-block", 5), ("jacobi", 1)):
         xs, _ = _single(bar, A, b, R, k, mode, 3, 0.0, x0)
-        xp, info = _loop(blocks, n, R, b, k, mode, 3, 0.0, x0)
+        xp, info = _loop(blocks, n, R, b, k, mode, 3, 0.0, x0, tuning=tune)
         assert np.array_equal(xs, xp), (mode, np.abs(xs - xp).max())
-    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n))
+    x, info = _loop(blocks, n, R, b, 5, "async", 20000, 1e-10, np.zeros(n), tuning=tune)
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+# ------------------------------------------------------------------ bar_create_csr_dist over NCCL
+@pytest.mark.parametrize("name,gen,args,R", MATS)
+@pytest.mark.parametrize("halo", ["sendrecv", "allgather"])
+def test_create_csr_dist_one_rank_nccl(bar, name, gen, args, R, halo):
+    """§8(b)'s bar_create_csr_dist through the C ABI only (ctypes; no torch.distributed): a
+    1-rank NCCL group (the box has one GPU). The library plans the share over NCCL (all-gathers
+    of the row ranges, ghost counts, devices and ghost lists; a min all-reduce of the peer-access
+    flags; an all-gather of the IPC handles), and the solve runs the collective path
+    (ncclGroupStart/End of the halo exchange or an in-place ncclAllGather, an ncclAllGather of the
+    residual partials per iteration): sync-block and Jacobi iterates and iteration counts are
+    bitwise those of bar_solve; async runs the peer-memory path (board barriers with itself)."""
+    import ctypes
+
+    import torch
+
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    A = gen(*args)
+    n = A.n
+    b = np.ones(n)
+    x0 = np.random.default_rng(8).uniform(-1, 1, n)
+    nid = ctypes.create_string_buffer(128)
+    assert bar._lib.bar_nccl_unique_id(nid) == 0, bar.bar_last_error()
+    h = ctypes.c_void_p()
+    rp, col, val = (np.ascontiguousarray(a) for a in (A.rowptr, A.col, A.val))
+    st = bar._lib.bar_create_csr_dist(n, 0, n, A.nnz, rp.ctypes.data, col.ctypes.data, val.ctypes.data, R, 0, nid, 0,
+                                      1, ctypes.byref(h))
+    assert st == 0, bar.bar_last_error()
+    bar.bar_set_tuning(h, {"halo": halo})
+    bd, x0d = torch.from_numpy(b).cuda(), torch.from_numpy(x0).cuda()
+    for mode, k in (("sync-block", 5), ("jacobi", 1)):
+        for m, tol in ((3, 0.0), (20000, 1e-10)):
+            xs, i1 = _single(bar, A, b, R, k, mode, m, tol, x0)
+            xd = torch.empty_like(bd)
+            _, i2 = bar.bar_solve(h, bd, x0d, xd, k, m, tol, mode)
+            assert np.array_equal(xs, xd.cpu().numpy()), (mode, m)
+            assert i1["iters"] == i2.iters
+    xd = torch.empty_like(bd)
+    _, info = bar.bar_solve(h, bd, None, xd, 5, 20000, 1e-10, "async")
+    assert info.converged and O.rel_res(A, b, xd.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    r, bn = bar.bar_residual(h, bd, xd)
+    ref = O.rel_res(A, b, xd.cpu().numpy())  # b - A x cancels near convergence: DESIGN.md R16
+    assert abs(r / bn - ref) <= 1e-6 * ref + 1e-15, (r / bn, ref)
+    # bar_sweep on the share: local launches (one rank: the whole matrix), oracle's iterates
+    xd = x0d.clone()
+    bar.bar_sweep(h, bd, xd, 5, 2, "sync-block")
+    torch.cuda.synchronize()
+    ref = O.block_jacobi_step(A, b, O.block_jacobi_step(A, b, x0, R, 5), R, 5)
+    assert np.abs(xd.cpu().numpy() - ref).max() <= 1e-12 * np.abs(ref).max()
+    bar.bar_destroy(h)
+    # the Python wrapper (marshalling only) over the same call
+    M = D.DistMatrix(A, n, R, 0, D.nccl_unique_id(), 0, 1)
+    xm, info = M.solve(bd, None, None, k=5, mode="sync-block")
+    xs, i1 = _single(bar, A, b, R, 5, "sync-block", 20000, 1e-10, np.zeros(n))
+    assert np.array_equal(xs, xm.cpu().numpy()) and info["iters"] == i1["iters"]
+    M.close()
+
+
+def test_create_csr_dist_errors(bar):
+    import ctypes
+
+    from paper_conf_ipps_anzttdh12_b200 import dist as D  # noqa: F401  (sets the argtypes)
+
+    A = W.stencil7_3d(8)
+    rp, col, val = (np.ascontiguousarray(a) for a in (A.rowptr, A.col, A.val))
+    nid = ctypes.create_string_buffer(128)
+    assert bar._lib.bar_nccl_unique_id(nid) == 0
+    h = ctypes.c_void_p()
+    # no NCCL id
+    assert bar._lib.bar_create_csr_dist(A.n, 0, A.n, A.nnz, rp.ctypes.data, col.ctypes.data, val.ctypes.data, 64, 0,
+                                        None, 0, 1, ctypes.byref(h)) == 1
+    # row_begin not a multiple of R
+    blk = W.stencil7_3d(8, row_lo=100, row_hi=200)
+    brp, bcol, bval = (np.ascontiguousarray(a) for a in (blk.rowptr, blk.col, blk.val))
+    assert bar._lib.bar_create_csr_dist(A.n, 100, 200, blk.nnz, brp.ctypes.data, bcol.ctypes.data, bval.ctypes.data,
+                                        64, 0, nid, 0, 2, ctypes.byref(h)) == 1
+    # a column outside [0, n_global)
+    bad = col.copy()
+    bad[5] = A.n + 3
+    assert bar._lib.bar_create_csr_dist(A.n, 0, A.n, A.nnz, rp.ctypes.data, bad.ctypes.data, val.ctypes.data, 64, 0,
+                                        nid, 0, 1, ctypes.byref(h)) == 2
+
+
+# ------------------------------------------------------------------ separate processes, peer memory
+def _peer_worker(rank, world, store, case, q):
+    import os
+    import sys
+
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import workloads as W
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    torch.cuda.set_device(0)
+    # a file store (no TCP port to race for); gloo only carries the ghost lists and IPC handles
+    dist.init_process_group("gloo", init_method=f"file://{store}", rank=rank, world_size=world)
+    try:
+        kind, size, R, k = case
+        gen = {"s7": W.stencil7_3d, "s9": W.stencil9_2d, "tref": W.trefethen}[kind]
+        n = gen(size).n
+        a, c = D.partition(n, R, world)[rank]
+        A = gen(size, row_lo=a, row_hi=c)
+
+        def allgather(o):
+            out = [None] * world
+            dist.all_gather_object(out, o)
+            return out
+
+        Pr = D.PeerRank(A, n, R, 0, rank, world, allgather)
+        b = torch.ones(c - a, dtype=torch.float64, device="cuda")
+        outs = []
+        for _ in range(2):  # twice: epochs and stop tags carry over between solves
+            x, info = Pr.solve(b, None, None, k=k, tol=1e-10, mode="async")
+            outs.append((x.cpu().numpy(), info))
+        Pr.close()
+        q.put((rank, outs))
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("case", [("s7", 24, 128, 5), ("tref", 2000, 128, 5), ("s9", 98, 128, 2)])
+@pytest.mark.parametrize("world", [2, 3])
+def test_peer_processes_one_gpu(bar, case, world):
+    """The peer-memory async mode with SEPARATE PROCESSES sharing the one GPU: real CUDA IPC
+    mappings of every rank's iterate and board (handles exchanged over gloo), ghost pulls with
+    relaxed system-scope loads, stop requests through the boards, and the confirming residual
+    behind two board barriers — no NCCL, no collective while iterating. Every rank returns
+    converged with the same exact residual; the assembled x meets it by the oracle."""
+    import multiprocessing as mp
+    import tempfile
+
+    import workloads as W
+
+    store = tempfile.mktemp(prefix="bar_peer_store_")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_peer_worker, args=(r, world, store, case, q), daemon=True) for r in range(world)]
+    for p in ps:
+        p.start()
+    try:
+        res = dict(q.get(timeout=240) for _ in ps)
+    finally:
+        for p in ps:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r in range(world):
+        assert not isinstance(res[r], str), res[r]
+    kind, size, R, k = case
+    gen = {"s7": W.stencil7_3d, "s9": W.stencil9_2d, "tref": W.trefethen}[kind]
+    A = gen(size)
+    b = np.ones(A.n)
+    for s_ in range(2):
+        infos = [res[r][s_][1] for r in range(world)]
+        x = np.concatenate([res[r][s_][0] for r in range(world)])
+        for i in infos:
+            assert i["converged"] and i["rel_res"] <= 1e-10, i
+        assert len({i["rel_res"] for i in infos}) == 1  # the same bits on every rank
+        assert len({i["iters"] for i in infos}) == 1  # min over ranks, agreed through the boards
+        assert O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)

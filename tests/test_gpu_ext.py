@@ -15,8 +15,8 @@ def _dev(a):
     return torch.from_numpy(np.ascontiguousarray(a)).cuda()
 
 
-def _gpu(bar, A, b, R, k, mode, iters, tol, x0=None, **kw):
-    M = bar.Matrix.from_csr(A, R)
+def _gpu(bar, A, b, R, k, mode, iters, tol, x0=None, tuning=None, **kw):
+    M = bar.Matrix.from_csr(A, R, tuning=tuning)
     x, info = M.solve(_dev(b), None if x0 is None else _dev(x0), None, k=k, max_global_iters=iters, tol=tol,
                       mode=mode, **kw)
     M.close()
@@ -69,6 +69,42 @@ def test_tau_rho_gt_1(bar):
     _close(x, r.x, 1e-10)
 
 
+def test_tau_async(bar):
+    """N3 in async mode (§8(f): "all three modes").
+    * The SPD system with rho(B) > 1: with tau = 2/(lambda_1 + lambda_n) async-(1)
+      converges to the direct solution. Across several subdomains nothing guarantees that
+      (rho(|B_tau|) = 1 - tau + tau rho(|B|) > 1 for every tau <= 1, so Chazan-Miranker allows
+      divergent orders), so it runs on one subdomain (R >= n), where async-(1) is tau-Jacobi.
+    * With tau != 1 the fixed point is preserved (start at x*, tol = 0: x stays at x*), and
+      for tau < 1 on Trefethen_2000 (rho(|B_tau|) = 1 - tau + 0.86 tau < 1) async-(5) over 16
+      subdomains converges to x*."""
+    n = 48
+    Ad = np.eye(n) + 0.3 * np.ones((n, n))
+    nz = [np.nonzero(Ad[i])[0] for i in range(n)]
+    A = W.CSR(n, np.concatenate([[0], np.cumsum([len(z) for z in nz])]).astype(np.int32),
+              np.concatenate(nz).astype(np.int32), np.concatenate([Ad[i, z] for i, z in enumerate(nz)]))
+    DA = Ad / np.diag(Ad)[:, None]
+    lam = np.linalg.eigvals(DA).real
+    tau = 2.0 / (lam.min() + lam.max())
+    b = np.ones(n)
+    xs = np.linalg.solve(Ad, b)
+    for R in (64, 1024):
+        x, info = _gpu(bar, A, b, R, 1, "async", 20000, 1e-10, tau=tau)
+        assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+        _close(x, xs, 1e-8)
+    B = W.trefethen(2000)
+    bb = np.ones(B.n)
+    xb = np.linalg.solve(B.to_dense(), bb)
+    for tau_ in (0.7, 1.2):
+        x, info = _gpu(bar, B, bb, 128, 5, "async", 10, 0.0, xb, tau=tau_)
+        assert info["iters"] == 10
+        assert np.abs(x - xb).max() <= 1e-13 * np.abs(xb).max()
+        # and from x0 = 0 the tau-scaled async iteration converges (rho(|B_tau|) < 1 for tau <= 1)
+        if tau_ < 1:
+            x, info = _gpu(bar, B, bb, 128, 5, "async", 20000, 1e-10, tau=tau_)
+            assert info["converged"] and np.abs(x - xb).max() <= 1e-8 * np.abs(xb).max()
+
+
 @pytest.mark.parametrize("name", list(MATS))
 @pytest.mark.parametrize("mode,k", [("sync-block", 5), ("jacobi", 1)])
 def test_failure_window_iterates(bar, name, mode, k):
@@ -116,11 +152,10 @@ def test_history_matches_oracle(bar, mode, k):
 
 
 @pytest.mark.parametrize("coded", ["1", "0"])
-def test_ext_options_on_duo_kernel(bar, monkeypatch, coded):
+def test_ext_options_on_duo_kernel(bar, coded):
     """N3 tau-scaling and N1 failure windows through the two-blocks-per-SM kernel's EXT
     instantiations (coded and int32 columns): iterates match the oracle to 1e-12."""
-    monkeypatch.setenv("BAR_DUO", "1")
-    monkeypatch.setenv("BAR_CODED", coded)
+    tune = {"duo": 1, "coded": 0 if coded == "1" else -1}
     A = W.stencil7_3d(128)  # R = two grid lines: <= 4 local entries per row
     R = 256
     b = np.ones(A.n)
@@ -129,9 +164,39 @@ def test_ext_options_on_duo_kernel(bar, monkeypatch, coded):
         ref = x0
         for _ in range(2):
             ref = O.step_ex(A, b, ref, meth, R=R, k=k, tau=0.8)
-        x, _ = _gpu(bar, A, b, R, k, mode, 2, 0.0, x0, tau=0.8)
+        x, _ = _gpu(bar, A, b, R, k, mode, 2, 0.0, x0, tuning=tune, tau=0.8)
         _close(x, ref)
     fz = np.random.default_rng(14).random(A.n) < 0.25
     r = O.solve(A, b, method=O.BLOCK_JACOBI, R=R, k=5, tol=0.0, max_iters=4, frozen=fz, fail_start=2, fail_stop=4)
-    x, _ = _gpu(bar, A, b, R, 5, "sync-block", 4, 0.0, fail_mask=fz, fail_start=2, fail_stop=4)
+    x, _ = _gpu(bar, A, b, R, 5, "sync-block", 4, 0.0, tuning=tune, fail_mask=fz, fail_start=2, fail_stop=4)
     _close(x, r.x)
+
+
+def test_n2_harness_small(bar):
+    """tools/nondeterminism.py (N2, Tables 2-3) at a small size: every run of a fixed
+    iteration count returns a finite exact residual, residuals fall with m, and the spread is
+    reported (run-to-run variation of the asynchronous schedule)."""
+    from tools import nondeterminism
+
+    name, rows = nondeterminism.table("c1", runs=4, checkpoints=[5, 15, 25])
+    assert [m for m, _ in rows] == [5, 15, 25]
+    avgs = [r.mean() for _, r in rows]
+    for _, r in rows:
+        assert len(r) == 4 and np.all(np.isfinite(r)) and np.all(r > 0)
+    assert avgs[0] > avgs[1] > avgs[2]
+    # sync-block-(5) after m iterations bounds the async average within a factor 30 (P5, R15)
+    A = W.trefethen(2000)
+    for m, r in rows:
+        sb = O.solve(A, np.ones(A.n), method=O.BLOCK_JACOBI, R=128, k=5, tol=0.0, max_iters=m).rel_res
+        assert r.mean() <= 30 * sb, (m, r.mean(), sb)
+
+
+def test_n4_harness_small(bar):
+    """tools/local_iters.py (N4, Table 4, P:711 / P:863-867) on C2: positive per-iteration times
+    for k = 1, 5, 9 that do not fall with k (each extra local sweep adds work, no HBM bytes)."""
+    from tools import local_iters
+
+    info, kernel, rows = local_iters.table("c2", ks=(1, 5, 9))
+    ts = [t for _, t in rows]
+    assert all(t > 0 for t in ts), rows
+    assert ts[2] >= 0.9 * ts[0], rows

@@ -91,3 +91,21 @@ def test_async_full_size_converges(big):
     # the solution is symmetric under the grid's reflection (b = 1, symmetric stencil): a property
     # of x* that a wrong index/partition would break
     assert np.abs(xh - xh[::-1]).max() <= 1e-8 * np.abs(xh).max()
+
+
+def test_async_known_solution_full_size(big):
+    """SURVEY §8(c) reading 1's second run at the bench configurations: x* = 1, b = A 1 (the CSR
+    row sums, computed here on the host), async-(5) to rel_res 1e-10 in bench.py's launch
+    configuration; the returned x must be within 1e-8 of x* = 1 in the max norm (cond_2(A) ~ 13
+    for these stencils, so 1e-10 in the residual bounds the error near 1e-9)."""
+    import torch
+
+    wl, R, n, M, x0, b = big
+    A = make_matrix(wl)
+    b1 = np.add.reduceat(A.val, A.rowptr[:-1])  # (A 1)_i, exact in fp64 up to one rounding per entry
+    del A
+    bd = torch.from_numpy(b1).cuda()
+    x, info = M.solve(bd, None, None, k=5, tol=1e-10, mode="async")
+    assert info["converged"] and info["rel_res"] <= 1e-10
+    err = (x - 1.0).abs().max().item()
+    assert err <= 1e-8, err

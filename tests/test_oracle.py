@@ -305,6 +305,44 @@ def test_tau_jacobi_matches_matrix_form():
     assert np.array_equal(O.step_ex(A, b, x, O.JACOBI, tau=1.0), O.jacobi_step(A, b, x))
 
 
+def _block_step_ex_matrix_form(Ad, b, x, R, k, tau, frozen):
+    """sb-(k) with N3 / N1 in splitting form: M = block-diagonal part (row//R == col//R),
+    N = A - M, F = diag(frozen), s = b - N x, y^0 = x and, k times, the correction form
+    y <- y + tau (I - F) D^-1 (s - M y)  (every update x + tau (v - x), R17; frozen rows keep
+    their value and are read by the others, R18)."""
+    n = Ad.shape[0]
+    blk = np.arange(n) // R
+    M = np.where(blk[:, None] == blk[None, :], Ad, 0.0)
+    s = b - (Ad - M) @ x
+    free = 1.0 - np.asarray(frozen, dtype=float)
+    y = x.copy()
+    for _ in range(k):
+        y = y + tau * free * (s - M @ y) / np.diag(Ad)
+    return y
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_block_step_ex_matches_matrix_form(seed):
+    """oracle_block_jacobi_step_ex per step, at R < n (off-block entries present), tau != 1 and
+    a frozen mask, against the splitting's matrix form — the function the GPU N1 / N3 parity
+    tests compare with."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(20, 90))
+    A = W.random_dd(n, 6, seed=seed, symmetric_pattern=bool(seed % 2))
+    Ad = _dense(A)
+    b, x = rng.standard_normal(n), rng.standard_normal(n)
+    frozen = (rng.random(n) < 0.3).astype(np.uint8)
+    for R in (1, 3, 7, 16, n - 1):
+        for k in (1, 2, 5):
+            for tau in (0.6, 1.0, 1.3):
+                for fz in (None, frozen):
+                    got = O.step_ex(A, b, x, O.BLOCK_JACOBI, R=R, k=k, tau=tau, frozen=fz)
+                    ref = _block_step_ex_matrix_form(Ad, b, x, R, k, tau, np.zeros(n) if fz is None else fz)
+                    np.testing.assert_allclose(got, ref, rtol=0, atol=1e-12 * (1 + np.abs(ref).max()))
+                    if fz is not None:
+                        assert np.array_equal(got[fz == 1], x[fz == 1])
+
+
 def test_tau_block_R_ge_n_is_k_tau_jacobi():
     A = W.random_dd(40, 5, seed=22)
     b, x = np.ones(40), np.random.default_rng(2).standard_normal(40)

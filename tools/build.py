@@ -88,10 +88,21 @@ def build_bar(force: bool = False) -> str:
     return out
 
 
+def build_test_helpers(force: bool = False) -> str:
+    """tests/helpers/libspin.so: a test-only kernel that occupies SMs (tests of the single-launch
+    kernel's behaviour when other work holds the device)."""
+    src = os.path.join(ROOT, "tests", "helpers", "spin.cu")
+    out = os.path.join(ROOT, "tests", "helpers", "libspin.so")
+    if force or _stale(out, [src]):
+        _run([NVCC, *ARCH, "-O2", "-Xcompiler", "-fPIC", "-shared", "-o", out, src])
+    return out
+
+
 def build_all(force: bool = False) -> None:
     build_workloads(force)
     build_oracle(force)
     build_bar(force)
+    build_test_helpers(force)
 
 
 if __name__ == "__main__":

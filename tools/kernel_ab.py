@@ -1,12 +1,13 @@
-"""A/B timing of kernel variants selected by environment switches (tuning aid, not a bench value).
+"""A/B timing of kernel variants selected by bar_tuning fields (tuning aid, not a bench value).
 
-For one matrix, each variant (a set of BAR_* environment variables, read by libbar.so at every
-launch) is timed two ways with CUDA events on the launching stream:
+For one matrix, each variant (a set of bar_tuning fields, set on the handle with bar_set_tuning;
+the library reads no environment variable) is timed two ways with CUDA events on the launching
+stream:
   * per launch: slope of 8 vs 40 back-to-back bar_sweep launches (cancels fixed overheads);
   * whole solve: bar_solve to tol, median of --reps solves, with its global-iteration count.
 
     python tools/kernel_ab.py --workload c5 --modes async,sync-block \
-        --variants 'base:;nopf:BAR_NO_GHOST_PREFETCH=1;pipe:BAR_PIPE=1'
+        --variants 'base:;nopf:ghost_prefetch=-1;pipe:pipe=1,duo=-1;strided:async_order=3'
 """
 import argparse
 import json
@@ -23,13 +24,14 @@ def parse_variants(spec):
     for item in spec.split(";"):
         if not item.strip():
             continue
-        name, _, envs = item.partition(":")
-        env = {}
-        for kv in envs.split(","):
+        name, _, fields = item.partition(":")
+        tune = {}
+        for kv in fields.split(","):
             if kv.strip():
                 k, _, v = kv.partition("=")
-                env[k.strip()] = v.strip()
-        out.append((name.strip(), env))
+                v = v.strip()
+                tune[k.strip()] = int(v) if v.lstrip("-").isdigit() else v
+        out.append((name.strip(), tune))
     return out
 
 
@@ -75,16 +77,9 @@ def main():
     del src, dst
     clk = os.popen("nvidia-smi --query-gpu=clocks.sm,clocks.mem,power.draw --format=csv,noheader").read().strip()
     print(json.dumps({"box": {"copy_GBs": round(copy_gbs, 1), "clocks": clk}}), flush=True)
-    base_env = {k: os.environ.get(k) for k in ("BAR_PIPE", "BAR_NO_GHOST_PREFETCH", "BAR_KERNEL", "BAR_ASYNC_STATIC",
-                                          "BAR_DUO", "BAR_JACOBI_ROWWISE", "BAR_GRID", "BAR_ORDER", "BAR_CODED", "BAR_RESIDENT", "BAR_LEAD")}
     for mode in a.modes.split(","):
-        for name, env in parse_variants(a.variants):
-            for k_, v in base_env.items():
-                if v is None:
-                    os.environ.pop(k_, None)
-                else:
-                    os.environ[k_] = v
-            os.environ.update(env)
+        for name, tune in parse_variants(a.variants):
+            M.set_tuning(tune or None)
             M.sweep(b, x, k=a.k, nsweeps=4, mode=mode)
             lo, hi = 8, 40
             t_lo = min(ev_time(lambda: M.sweep(b, x, k=a.k, nsweeps=lo, mode=mode))[0] for _ in range(3))
@@ -94,7 +89,7 @@ def main():
             solves = [ev_time(lambda: M.solve(b, None, x, k=a.k, mode=mode)) for _ in range(a.reps)]
             ms = statistics.median(s[0] for s in solves)
             iters = [s[1][1]["iters"] for s in solves]
-            print(json.dumps({"workload": a.workload, "R": R, "k": a.k, "mode": mode, "variant": name, "env": env,
+            print(json.dumps({"workload": a.workload, "R": R, "k": a.k, "mode": mode, "variant": name, "tuning": tune,
                               "launch_ms": round(per_launch, 4),
                               "contract_GBs": round(info["model_bytes_per_iter"] / per_launch / 1e6, 1),
                               "frac_of_copy": round(info["model_bytes_per_iter"] / per_launch / 1e6 / copy_gbs, 3),

@@ -48,7 +48,15 @@ def full(rep, out, traffic_json=None):
                                                          for v, k in stalls))
     open(out, "w").write("\n".join(lines) + "\n")
     if traffic_json and dram:
-        json.dump({"dram_bytes_per_launch": sum(dram) / len(dram), "source": rep}, open(traffic_json, "w"))
+        # stamped with the build, kernel and R it was captured from: bench.py only uses a capture
+        # whose stamp matches the run (a capture of another build is stale)
+        sys.path.insert(0, __import__("os").path.dirname(__import__("os").path.dirname(__import__("os").path.abspath(__file__))))
+        import bench
+
+        kern = d.get("Kernel Name", "?")
+        json.dump({"dram_bytes_per_launch": sum(dram) / len(dram), "source": rep, "libbar_sha256": bench.lib_hash(),
+                   "kernel": KERNEL_NAMES.get(kern.split("(")[0].split("::")[-1], kern), "R": R_ARG},
+                  open(traffic_json, "w"))
     print("\n".join(lines))
 
 
@@ -76,7 +84,14 @@ def launches(csv_path, out):
     print("\n".join(lines))
 
 
+# ncu kernel names -> the names libbar reports (bar_matrix_info.last_sweep_kernel)
+KERNEL_NAMES = {"k_block_duo<1, 4, 0, 1>": "k_block_duo<async,coded>", "k_block_duo<0, 4, 0, 1>": "k_block_duo<sync,coded>",
+                "k_block_duo<1, 4, 0, 0>": "k_block_duo<async>", "k_block_duo<0, 4, 0, 0>": "k_block_duo<sync>"}
+R_ARG = None
+
 if __name__ == "__main__":
+    if "--R" in sys.argv:
+        R_ARG = int(sys.argv[sys.argv.index("--R") + 1])
     mode = sys.argv[1]
     if mode == "full":
         tj = sys.argv[sys.argv.index("--traffic-json") + 1] if "--traffic-json" in sys.argv else None

@@ -17,6 +17,7 @@ def main():
     ap.add_argument("--k", type=int, default=5)
     ap.add_argument("--R", type=int, default=None)
     ap.add_argument("--sweeps", type=int, default=6)
+    ap.add_argument("--tune", default="", help="bar_tuning fields, e.g. async_order=3")
     a = ap.parse_args()
     import torch
 
@@ -25,7 +26,11 @@ def main():
 
     R = a.R or bench.WORKLOADS[a.workload][2]
     A = bench.make_matrix(a.workload)
-    M = bar.Matrix.from_csr(A, rows_per_block=R)
+    tune = {}
+    for kv in filter(None, a.tune.split(",")):
+        k, v = kv.split("=")
+        tune[k] = int(v) if v.lstrip("-").isdigit() else v
+    M = bar.Matrix.from_csr(A, rows_per_block=R, tuning=tune or None)
     del A
     b = torch.ones(M.n, dtype=torch.float64, device="cuda")
     x = torch.zeros(M.n, dtype=torch.float64, device="cuda")
