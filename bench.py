@@ -135,6 +135,22 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+class quiet_stdout:
+    """Redirect file descriptor 1 to /dev/null (C libraries write there directly)."""
+
+    def __enter__(self):
+        sys.stdout.flush()
+        self.saved = os.dup(1)
+        dn = os.open(os.devnull, os.O_WRONLY)
+        os.dup2(dn, 1)
+        os.close(dn)
+
+    def __exit__(self, *a):
+        sys.stdout.flush()
+        os.dup2(self.saved, 1)
+        os.close(self.saved)
+
+
 def cpu_info():
     cores = len(os.sched_getaffinity(0))
     model = ""
@@ -360,7 +376,8 @@ def main():
         A = make_matrix(args.workload, rows[0], rows[1])
         t_gen = time.time() - t0
         t0 = time.time()
-        M = bdist.DistMatrix.from_process_group(A, n, args.R, local_rank, tuning=tune)
+        with quiet_stdout():
+            M = bdist.DistMatrix.from_process_group(A, n, args.R, local_rank, tuning=tune)
         t_setup = time.time() - t0
         n_loc = rows[1] - rows[0]
         local_bytes = A.nnz * 12.0 + n_loc * 28.0
@@ -481,7 +498,9 @@ def main():
             from paper_conf_ipps_anzttdh12_b200 import dist as bdist
 
             t0 = time.time()
-            Md = bdist.DistMatrix(A_host, n, args.R, local_rank, bdist.nccl_unique_id(), 0, 1, tuning=tune or None)
+            with quiet_stdout():  # NCCL prints its version line on stdout; the bench prints ONE line
+                Md = bdist.DistMatrix(A_host, n, args.R, local_rank, bdist.nccl_unique_id(), 0, 1,
+                                      tuning=tune or None)
             t_dc = time.time() - t0
             for _ in range(2):
                 step(Mx=Md)

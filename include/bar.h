@@ -210,8 +210,7 @@ typedef struct {
     int32_t pipe;           /* 0 auto, 1 two-ahead pipelined kernel wherever it fits, -1 never    */
     int32_t coded;          /* 0 auto (coded columns when the layout has them), -1 int32 columns  */
     int32_t async_order;    /* per-launch async subdomain order: 0 auto (contiguous chunks per
-                               block, R15), 1 chunks, 2 round robin, 3 strided chunks (chunks of
-                               the plane-transposed sequence, where the layout has a plane stride) */
+                               block, R15), 1 chunks, 2 round robin                               */
     int32_t async_queue;    /* 0 static claims, 1 device work-queue claims (k_block_stage)       */
     int32_t resident;       /* 0 auto, -1 never use the block-owns-subdomain single-launch kernel */
     int32_t lead;           /* k_block_resident: max sweeps a block may lead the last completed

@@ -75,7 +75,7 @@ class Tuning(ctypes.Structure):
         "single_launch", "jacobi_rowwise", "grid_cap", "warps", "halo", "peer")]
 
     KERNELS = {"auto": 0, "block": 1, "reg": 2, "reg_tma": 3, "pers": 4}
-    ORDERS = {"auto": 0, "chunks": 1, "round_robin": 2, "strided": 3}
+    ORDERS = {"auto": 0, "chunks": 1, "round_robin": 2}
 
     @classmethod
     def make(cls, **kw):

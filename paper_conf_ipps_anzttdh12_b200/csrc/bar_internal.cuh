@@ -94,9 +94,6 @@ struct Layout {
     int64_t local_entries = 0;
     int max_wl = 0, max_wo = 0;
     int max_w = 0;              // widest slice: max over slices of wl + wo
-    int64_t plane_stride = 0;   // S: the farthest frequent off-block coupling of a middle subdomain,
-                                // in subdomains, when it is a whole multiple of R (3D grid: a plane);
-                                // used by the strided claim order (tuning.async_order = 3)
     int sms = 148;              // SMs of the device (persistent grids)
     // device arrays
     double *val = nullptr;      // [entries]

@@ -496,17 +496,6 @@ bar_status build_layout(Layout &L, int64_t n, int64_t nnz, const int32_t *d_rowp
     k_ghost_ranges<<<(unsigned)L.q, 256, 0, st>>>(n, R, col_lo, col_hi, d_rowptr, d_col, L.gr);
     BAR_CK(cudaGetLastError());
     BAR_CK(cudaStreamSynchronize(st));
-    {  // plane stride: the farthest full-width ghost range of the middle subdomain, in subdomains
-        const int64_t lm = L.q / 2;
-        int32_t g[2 * kGhostRanges];
-        BAR_CK(cudaMemcpy(g, L.gr + 2 * lm * kGhostRanges, sizeof(g), cudaMemcpyDeviceToHost));
-        int64_t far = 0;
-        for (int r = 0; r < kGhostRanges; ++r) {
-            const int64_t d = (int64_t)g[2 * r] - lm * (int64_t)R;
-            if (g[2 * r + 1] == R && d % R == 0 && (d < 0 ? -d : d) > far) far = d < 0 ? -d : d;
-        }
-        L.plane_stride = far / R;
-    }
     build_codes(L, st);
 
 done:

@@ -58,8 +58,6 @@ struct KP {
     const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
     int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
-    int32_t stride;         // > 0: strided (transposed) chunk order, S subdomains per plane (claim_at)
-    int32_t stride_q;       //   and Q = q / S planes
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
@@ -72,16 +70,9 @@ struct KP {
 // sweeps its chunk in order, so a subdomain sees this iteration's values of its predecessors in
 // the chunk: eq. 4's shift s(k+1, j) > 0, the block Gauss-Seidel flavour of P:209, on every
 // coupling shorter than the chunk). Either way each subdomain is swept exactly once per launch (R7).
-// A third order (tuning.async_order = 3, "strided"): with S = Layout::plane_stride subdomains
-// between a subdomain and its farthest frequent coupling (C5: a grid plane = 256 subdomains of
-// two lines), the chunks are cut from the TRANSPOSED sequence t = s Q + p of l = p S + s
-// (Q = q / S): a block sweeps one position s through consecutive planes p, so the plane below was
-// swept one claim earlier (Gauss-Seidel along the far coupling, its x still in L2) and the
-// plane above, read as ghosts, is the next claim's x_J.
 struct Claims {
     long long l0, step, lend;
 };
-constexpr long long kNoClaim = 0x7fffffffffffffffll;
 
 __device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
     const long long G = gridDim.x, c = blockIdx.x;
@@ -89,16 +80,7 @@ __device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
     return {c, G, (long long)q};
 }
 
-// The j-th subdomain block c claims, or kNoClaim past its last.
-__device__ __forceinline__ long long claim_at(const KP &p, const Claims &C, long long j, int64_t q) {
-    const long long t = C.l0 + j * C.step;
-    if (t >= C.lend) return kNoClaim;
-    if (p.stride > 0) {  // q < 2^31: 32-bit arithmetic
-        const uint32_t tt = (uint32_t)t, Q = (uint32_t)p.stride_q;
-        return (long long)(tt % Q) * p.stride + tt / Q;
-    }
-    return t;
-}
+
 
 // Thread 0: start copying subdomain l's ghost-range entry (kGhostRanges pairs, 32 B) into
 // shared memory with cp.async (completion: cp.async.wait_all before reading it).
@@ -850,7 +832,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const Claims C = claims_of(p, q);
-    auto lof = [&](long long j) { return claim_at(p, C, j, q); };
+    auto lof = [&](long long j) { return C.l0 + j * C.step; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto stage_bytes = [&](long long l, int64_t E0, int64_t E1) -> uint32_t {
         const int nrows = (int)min((int64_t)R, p.n - (int64_t)l * R);
@@ -861,7 +843,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // part w (0..3) of the stage of l_j (see above); one lane per warp
     auto issue_part = [&](int w, long long j, const int64_t *bd, const int32_t *gr) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int vs = (int)(j & 1), bs = (int)(j % 3);
         const int64_t TS = l * (int64_t)R;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
@@ -888,7 +870,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -910,14 +892,14 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         fence_mbar_init();
         for (int j = 0; j < 4; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
         }
         for (int j = 0; j < 2; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             mbar_arrive_expect_tx(&bars[j], stage_bytes(l, bnd[j][0], bnd[j][1]));
             for (int w = 0; w < 4; ++w) issue_part(w, j, bnd[j], j == 1 && p.gr ? gsm[j] : nullptr);
         }
@@ -929,7 +911,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     for (int i = 0;; ++i) {
         const int vs = i & 1, bs = i % 3;
         const long long l = lof(i);
-        if (l >= q) break;
+        if (l >= C.lend) break;
         unsigned char *V = smraw + (size_t)vs * g.vc_bytes;
         unsigned char *B = smraw + g.o_bx + (size_t)bs * g.bx_bytes;
         const int64_t TS = l * (int64_t)R;
@@ -991,7 +973,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         }
         // post the byte count of l_{i+2}'s stage before the barrier that frees its buffers, so
         // that no copy of it can complete bytes before its phase expects them
-        if (threadIdx.x == 0 && lof(i + 2) < q) {
+        if (threadIdx.x == 0 && lof(i + 2) < C.lend) {
             const int r = (i + 2) & 3;
             mbar_arrive_expect_tx(&bars[(i + 2) % 3], stage_bytes(lof(i + 2), bnd[r][0], bnd[r][1]));
         }
@@ -1074,7 +1056,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     double *ya = reinterpret_cast<double *>(smraw + g.o_ya);
     double *yb = reinterpret_cast<double *>(smraw + g.o_yb);
     const Claims C = claims_of(p, q);
-    auto lof = [&](long long j) { return claim_at(p, C, j, q); };
+    auto lof = [&](long long j) { return C.l0 + j * C.step; };
     auto nsl_of = [&](long long l) { return (int)((min((int64_t)R, p.n - (int64_t)l * R) + kSlice - 1) / kSlice); };
     auto slab_bytes = [&](long long l, const int64_t *bd, const int32_t *db) -> uint32_t {
         const uint32_t nsl = (uint32_t)nsl_of(l);
@@ -1085,7 +1067,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
     auto issue_part = [&](int w, long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int64_t *bd = bnd[j & 3];
         if (w == 3) {  // what l_j's first phase reads directly: b_J, x_J and its ghost x ranges
             const int64_t TS = l * (int64_t)R;
@@ -1120,7 +1102,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
     auto fetch_ring = [&](long long j) {
         const long long l = lof(j);
-        if (l >= q) return;
+        if (l >= C.lend) return;
         const int r = (int)(j & 3);
         asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(&bnd[r][0])), "l"(p.sptr + l * spb)
                      : "memory");
@@ -1148,7 +1130,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         fence_mbar_init();
         for (int j = 0; j < 3; ++j) {
             const long long l = lof(j);
-            if (l >= q) break;
+            if (l >= C.lend) break;
             bnd[j][0] = p.sptr[l * spb];
             bnd[j][1] = p.sptr[l * spb + nsl_of(l)];
             for (int t = 0; t < 2 * kGhostRanges; ++t) gsm[j][t] = p.gr ? p.gr[2 * l * kGhostRanges + t] : 0;
@@ -1166,7 +1148,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     double rr = 0.0, bb = 0.0;
     for (int i = 0;; ++i) {
         const long long l = lof(i);
-        if (l >= q) break;
+        if (l >= C.lend) break;
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
@@ -1225,7 +1207,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             bb += bi * bi;
         }
         // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
-        if (threadIdx.x == 0 && lof(i + 1) < q)
+        if (threadIdx.x == 0 && lof(i + 1) < C.lend)
             mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3], dbd[(i + 1) & 3]));
         __syncthreads();
         if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
@@ -2206,9 +2188,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // vs 59 with round robin, C4 (R = 512) 63 vs 105 — each block sweeps its chunk in order, so
     // the neighbouring lines / planes below a subdomain already hold this iteration's values.
     // (sync modes: the order does not change the iterates; round robin)
-    p.claim_chunk = T.async_order == 0 ? (ASYNC ? 1 : 0) : (T.async_order != 2 ? 1 : 0);
-    p.stride = (T.async_order == 3 && L.plane_stride > 0 && L.q % L.plane_stride == 0) ? (int32_t)L.plane_stride : 0;
-    p.stride_q = p.stride ? (int32_t)(L.q / p.stride) : 1;
+    p.claim_chunk = T.async_order == 0 ? (ASYNC ? 1 : 0) : (T.async_order == 1 ? 1 : 0);
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);

@@ -399,7 +399,7 @@ def test_forced_kernel_paths(bar, tune, name, R):
 def test_tuning_validation(bar):
     A = W.trefethen(64)
     M = bar.Matrix.from_csr(A, 16)
-    for bad in ({"kernel": 9}, {"lead": 49}, {"async_order": 3}, {"halo": 2}, {"warps": 33}):
+    for bad in ({"kernel": 9}, {"lead": 49}, {"async_order": 3}, {"halo": 2}, {"warps": 33}, {"peer": 1}):
         with pytest.raises(bar.BarError):
             M.set_tuning(bad)
     with pytest.raises(KeyError):

@@ -52,13 +52,14 @@ def test_single_launch_with_device_held(bar, spin, n, envelope, graph):
     assert "resident" in M.info()["last_sweep_kernel"] and info0["converged"]
     s_spin, s_solve = torch.cuda.Stream(), torch.cuda.Stream()
     sms = spin.spin_sm_count(0)
-    assert spin.spin_launch(sms - 2, 1024, 200 * 1024, 400_000_000, ctypes.c_void_p(s_spin.cuda_stream)) == 0
-    time.sleep(0.05)  # the spinner now holds sms - 2 SMs for ~0.35 s more
-    t0 = time.perf_counter()
-    _, info = M.solve(bd, None, x, k=5, tol=1e-10, mode="async", stream=s_solve, max_global_iters=20000)
-    s_solve.synchronize()
-    dt = time.perf_counter() - t0
-    torch.cuda.synchronize()
+    for rep in range(2):  # the first pass also loads the fallback kernels (lazy module loading)
+        assert spin.spin_launch(sms - 2, 1024, 200 * 1024, 400_000_000, ctypes.c_void_p(s_spin.cuda_stream)) == 0
+        time.sleep(0.05)  # the spinner now holds sms - 2 SMs for ~0.35 s more
+        t0 = time.perf_counter()
+        _, info = M.solve(bd, None, x, k=5, tol=1e-10, mode="async", stream=s_solve, max_global_iters=20000)
+        s_solve.synchronize()
+        dt = time.perf_counter() - t0
+        torch.cuda.synchronize()
     assert info["converged"] and info["rel_res"] <= 1e-10, info
     assert O.rel_res(A, b, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
     assert envelope[0] <= info["iters"] <= envelope[1], info
