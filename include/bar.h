@@ -208,9 +208,13 @@ typedef struct {
                                2 k_reg, 3 k_reg_tma, 4 k_block_pers                              */
     int32_t duo;            /* 0 auto, 1 two-blocks-per-SM kernel wherever it fits, -1 never      */
     int32_t pipe;           /* 0 auto, 1 two-ahead pipelined kernel wherever it fits, -1 never    */
-    int32_t coded;          /* 0 auto (coded columns when the layout has them), -1 int32 columns  */
+    int32_t coded;          /* 0 auto = 1: coded columns when the layout has them, off-block x
+                               gathered entry by entry; 2 staged gathers (each subdomain's off-block
+                               x intervals copied to shared memory first, where the layout has
+                               them); -1 int32 columns                                            */
     int32_t async_order;    /* per-launch async subdomain order: 0 auto (contiguous chunks per
-                               block, R15), 1 chunks, 2 round robin                               */
+                               block, R15), 1 chunks, 2 round robin, 3 fronts: `fronts` contiguous
+                               ranges, each swept round robin by its share of the blocks         */
     int32_t async_queue;    /* 0 static claims, 1 device work-queue claims (k_block_stage)       */
     int32_t resident;       /* 0 auto, -1 never use the block-owns-subdomain single-launch kernel */
     int32_t lead;           /* k_block_resident: max sweeps a block may lead the last completed
@@ -225,6 +229,7 @@ typedef struct {
     int32_t halo;           /* multi-GPU sync / collective exchange: 0 NCCL grouped send/recv,
                                1 one ncclAllGather per iteration                                 */
     int32_t peer;           /* multi-GPU async: 0 peer memory when mapped, -1 the collective path */
+    int32_t fronts;         /* async_order = 3: number of fronts (0 = 8)                          */
 } bar_tuning;
 
 /* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a

@@ -233,9 +233,9 @@ bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning) {
     }
     bar_tuning t{};
     if (tuning) t = *tuning;
-    if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 2 || t.async_queue < 0 ||
+    if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 3 || t.fronts < 0 || t.async_queue < 0 ||
         t.async_queue > 1 || t.lead < 0 || t.lead > 48 || t.grid_cap < 0 || t.warps < 0 || t.warps > 32 ||
-        t.halo < 0 || t.halo > 1 || t.peer > 0) {
+        t.halo < 0 || t.halo > 1 || t.peer > 0 || t.coded > 2) {
         set_error("bar_tuning field out of range");
         return BAR_ERR_INVALID_ARG;
     }
@@ -262,7 +262,8 @@ bar_status bar_matrix_get_info(bar_matrix A, bar_matrix_info *info) {
     info->last_sweep_kernel = L.last_kernel;
     info->coded = L.codes != nullptr;
     info->layout_bytes_per_iter = (double)L.entries * (8 + (L.codes ? 1 : 4)) + (double)L.n * 24 +
-                                  (double)L.nslices * 12 + (L.codes ? (double)L.dict_entries * 4 + (double)L.q * 4 : 0.0);
+                                  (double)L.nslices * 12 + (L.codes ? (double)L.dict_entries * 4 + (double)L.q * 4 : 0.0) +
+                                  (L.xs_len > 0 ? (double)L.q * kMaxIv * 16 : 0.0);
     return BAR_OK;
 }
 

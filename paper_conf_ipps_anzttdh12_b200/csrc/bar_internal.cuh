@@ -111,12 +111,20 @@ struct Layout {
     int32_t *dict = nullptr;    // [dptr[q]]
     int32_t *dptr = nullptr;    // [q + 1]
     int64_t dict_entries = 0;
+    // Staged gathers (coded layouts whose every subdomain's off-block columns lie in <= kMaxIv
+    // x intervals of total length <= 4 R; else xs_len = 0): iv[l] = kMaxIv x (lo, len, base, 0)
+    // and sdict (dictionary of shared-memory index offsets, layout.cu k_codes); xs_len = the
+    // largest interval buffer (>= R) in doubles
+    int32_t *sdict = nullptr;   // [dptr[q]]
+    int32_t *iv = nullptr;      // [q][kMaxIv][4]
+    int64_t xs_len = 0;
     bar_tuning tune{};          // explicit kernel / schedule overrides (bar_set_tuning); zero = defaults
     mutable int64_t rw_grid = -1;  // cached rowwise_grid (occupancy queries cost API round trips)
     mutable const char *last_kernel = "none";  // name of the most recently launched sweep kernel
 };
 constexpr int kGhostRanges = 4;
 constexpr int kDictMax = 256;
+constexpr int kMaxIv = 4;
 
 // Device time of the sweep-kernel launches of one solve, taken with CUDA events on the
 // launching stream around each launch (the bench's live per-launch duration inside its timed

@@ -203,32 +203,54 @@ __global__ void k_ghost_ranges(int64_t n, int32_t R, int64_t col_lo, int64_t col
 }
 
 // Per subdomain (one block): the dictionary of its column offsets d = col - row (off-block
-// entries store global columns, local ones col - TS; padding has d = 0) and each entry's 1-byte
-// code. dcount[l] = dictionary size, or -1 if it exceeds kDictMax (then no coded layout).
-// Entries of the rows past n in the last subdomain are never read: code 0.
+// entries store global columns, local ones col - TS; padding has d = 0), keyed by (d, local):
+// an offset that is local for some rows of the subdomain and off-block for others (a 3D
+// stencil's -512 in a two-line subdomain) gets two codes. dcount[l] = dictionary size, or -1 if
+// it exceeds kDictMax (then no coded layout). Entries of the rows past n in the last subdomain
+// are never read: code 0.
+//
+// Staged gathers: the off-block columns of the subdomain's real (non-padding) entries with
+// offset d span [TS + d + loc_min(d), TS + d + loc_max(d)]; merged (gaps <= kIvGap), these
+// spans give at most kMaxIv intervals of x that the sweep copies into shared memory once per
+// visit (one pass of coalesced relaxed loads) instead of gathering entry by entry. sdict[code]
+// is then, for an off-block code, the shared-memory index offset TS + d - lo_r + base_r of its
+// interval r (x of entry (loc, code) at xs[loc + sdict[code]]), for a local code d itself, and
+// 0 for off-block padding (value 0; xs[loc] is finite since the buffer holds >= R values).
+// iv[l] = kMaxIv x (lo, len, base, 0); ivlen[l] = buffer length, or -1 when the subdomain's
+// off-block columns do not fit kMaxIv intervals of total length <= kIvCap * R.
 constexpr int kDictSlots = 2 * kDictMax;
+constexpr int kIvGap = 16;
+constexpr int kIvCap = 4;
 __global__ void k_codes(int64_t n, int32_t R, int32_t spb, const int64_t *__restrict__ sptr,
                         const int32_t *__restrict__ sw, const int32_t *__restrict__ col, uint8_t *__restrict__ codes,
-                        int32_t *__restrict__ dtmp, int32_t *__restrict__ dcount) {
-    __shared__ int32_t key[kDictSlots];
+                        int32_t *__restrict__ dtmp, int32_t *__restrict__ stmp, int32_t *__restrict__ dcount,
+                        int32_t *__restrict__ iv, int32_t *__restrict__ ivlen) {
+    __shared__ long long key[kDictSlots];
     __shared__ int32_t code[kDictSlots];
+    __shared__ int32_t mnl[kDictSlots], mxl[kDictSlots];
+    __shared__ long long st[kDictMax], en[kDictMax];  // thread 0: spans of the off-block offsets
     __shared__ int overflow;
-    const int32_t kEmpty = INT32_MIN;
-    for (int t = threadIdx.x; t < kDictSlots; t += blockDim.x) key[t] = kEmpty;
+    const long long kEmpty = (long long)0x8000000000000000ull;
+    for (int t = threadIdx.x; t < kDictSlots; t += blockDim.x) {
+        key[t] = kEmpty;
+        mnl[t] = INT32_MAX;
+        mxl[t] = -1;
+    }
     if (threadIdx.x == 0) overflow = 0;
     __syncthreads();
     const int64_t l = blockIdx.x, TS = l * (int64_t)R;
     const int nrows = (int)min((int64_t)R, n - TS);
     const int nsl = (nrows + kSlice - 1) / kSlice;
-    auto slot_of = [&](int32_t d, bool insert) -> int {
-        int h = (int)(((uint32_t)d * 2654435761u) >> 23) & (kDictSlots - 1);  // 9 bits
+    auto slot_of = [&](long long k, bool insert) -> int {
+        int h = (int)(((unsigned long long)k * 0x9E3779B97F4A7C15ull) >> 55) & (kDictSlots - 1);  // 9 bits
         for (int probe = 0; probe < kDictSlots; ++probe, h = (h + 1) & (kDictSlots - 1)) {
-            const int32_t k = key[h];
-            if (k == d) return h;
-            if (k == kEmpty) {
+            const long long kk = key[h];
+            if (kk == k) return h;
+            if (kk == kEmpty) {
                 if (!insert) return -1;
-                const int32_t old = atomicCAS(&key[h], kEmpty, d);
-                if (old == kEmpty || old == d) return h;
+                const long long old = (long long)atomicCAS((unsigned long long *)&key[h], (unsigned long long)kEmpty,
+                                                           (unsigned long long)k);
+                if (old == kEmpty || old == k) return h;
             }
         }
         return -1;
@@ -244,13 +266,20 @@ __global__ void k_codes(int64_t n, int32_t R, int32_t spb, const int64_t *__rest
                     continue;
                 }
                 const int32_t c = col[E + t];
-                const int32_t d = e < wo ? (int32_t)(c - (TS + loc)) : c - loc;
-                const int h = slot_of(d, pass == 0);
+                const bool local = e >= wo;
+                const int32_t d = local ? c - loc : (int32_t)(c - (TS + loc));
+                const int h = slot_of(((long long)d << 1) | (local ? 1 : 0), pass == 0);
                 if (h < 0) {
                     overflow = 1;
                     continue;
                 }
-                if (pass == 1) codes[E + t] = (uint8_t)code[h];
+                if (pass == 1) {
+                    codes[E + t] = (uint8_t)code[h];
+                    if (!local && (c < TS || c >= TS + nrows)) {  // a real off-block entry
+                        atomicMin(&mnl[h], loc);
+                        atomicMax(&mxl[h], loc);
+                    }
+                }
             }
         }
         __syncthreads();
@@ -258,7 +287,7 @@ __global__ void k_codes(int64_t n, int32_t R, int32_t spb, const int64_t *__rest
             int cnt = 0;
             for (int h = 0; h < kDictSlots; ++h) {
                 if (key[h] == kEmpty) continue;
-                if (cnt < kDictMax) dtmp[l * kDictMax + cnt] = key[h];
+                if (cnt < kDictMax) dtmp[l * kDictMax + cnt] = (int32_t)(key[h] >> 1);
                 code[h] = cnt++;
             }
             if (cnt == 0) dtmp[l * kDictMax + cnt++] = 0;
@@ -267,6 +296,69 @@ __global__ void k_codes(int64_t n, int32_t R, int32_t spb, const int64_t *__rest
         }
         __syncthreads();
         if (overflow) return;
+    }
+    if (threadIdx.x != 0) return;
+    // intervals: spans of the real off-block offsets, sorted by start and merged
+    int ns = 0;
+    for (int h = 0; h < kDictSlots; ++h) {
+        if (key[h] == kEmpty || (key[h] & 1) || mxl[h] < 0) continue;
+        const long long d = key[h] >> 1;
+        long long a = TS + d + mnl[h], b = TS + d + mxl[h] + 1;
+        int i = ns++;
+        while (i > 0 && st[i - 1] > a) {  // insertion sort by start
+            st[i] = st[i - 1];
+            en[i] = en[i - 1];
+            --i;
+        }
+        st[i] = a;
+        en[i] = b;
+    }
+    long long lo[kMaxIv], hi[kMaxIv];
+    int ni = 0;
+    bool ok = true;
+    for (int i = 0; i < ns && ok; ++i) {
+        if (ni > 0 && st[i] <= hi[ni - 1] + kIvGap) {
+            if (en[i] > hi[ni - 1]) hi[ni - 1] = en[i];
+        } else if (ni == kMaxIv) {
+            ok = false;
+        } else {
+            lo[ni] = st[i];
+            hi[ni] = en[i];
+            ++ni;
+        }
+    }
+    long long tot = 0;
+    for (int r = 0; r < ni; ++r) tot += hi[r] - lo[r];
+    if (tot > (long long)kIvCap * R) ok = false;
+    long long base[kMaxIv];
+    {
+        long long acc = 0;
+        for (int r = 0; r < ni; ++r) {
+            base[r] = acc;
+            acc += hi[r] - lo[r];
+        }
+    }
+    for (int r = 0; r < kMaxIv; ++r) {
+        int32_t *o = iv + 4 * (l * kMaxIv + r);
+        o[0] = ok && r < ni ? (int32_t)lo[r] : 0;
+        o[1] = ok && r < ni ? (int32_t)(hi[r] - lo[r]) : 0;
+        o[2] = ok && r < ni ? (int32_t)base[r] : 0;
+        o[3] = 0;
+    }
+    ivlen[l] = ok ? (int32_t)(tot > R ? tot : R) : -1;
+    for (int h = 0; h < kDictSlots; ++h) {
+        if (key[h] == kEmpty) continue;
+        const long long d = key[h] >> 1;
+        int32_t v = (int32_t)d;  // local code: the local offset
+        if (!(key[h] & 1)) {
+            v = 0;  // off-block padding only
+            if (mxl[h] >= 0 && ok) {
+                const long long a = TS + d + mnl[h];
+                for (int r = 0; r < ni; ++r)
+                    if (a >= lo[r] && a < hi[r]) v = (int32_t)(TS + d - lo[r] + base[r]);
+            }
+        }
+        stmp[l * kDictMax + code[h]] = v;
     }
 }
 
@@ -277,11 +369,15 @@ __global__ void k_dict_pad(int64_t q, const int32_t *__restrict__ dcount, int32_
     if (l == q) dsize[l] = 0;
 }
 
-__global__ void k_dict_compact(int64_t q, const int32_t *__restrict__ dtmp, const int32_t *__restrict__ dcount,
-                               const int32_t *__restrict__ dptr, int32_t *__restrict__ dict) {
+__global__ void k_dict_compact(int64_t q, const int32_t *__restrict__ dtmp, const int32_t *__restrict__ stmp,
+                               const int32_t *__restrict__ dcount, const int32_t *__restrict__ dptr,
+                               int32_t *__restrict__ dict, int32_t *__restrict__ sdict) {
     const int64_t l = blockIdx.x;
     const int cnt = dcount[l], sz = dptr[l + 1] - dptr[l];
-    for (int c = threadIdx.x; c < sz; c += blockDim.x) dict[dptr[l] + c] = c < cnt ? dtmp[l * kDictMax + c] : 0;
+    for (int c = threadIdx.x; c < sz; c += blockDim.x) {
+        dict[dptr[l] + c] = c < cnt ? dtmp[l * kDictMax + c] : 0;
+        sdict[dptr[l] + c] = c < cnt ? stmp[l * kDictMax + c] : 0;
+    }
 }
 
 template <class T>
@@ -305,32 +401,46 @@ void free_layout(Layout &L) {
     cudaFree(L.codes);
     cudaFree(L.dict);
     cudaFree(L.dptr);
+    cudaFree(L.sdict);
+    cudaFree(L.iv);
     L.codes = nullptr;
     L.dict = nullptr;
     L.dptr = nullptr;
+    L.sdict = nullptr;
+    L.iv = nullptr;
     L.dict_entries = 0;
+    L.xs_len = 0;
 }
 
 // Coded columns (Layout::codes); leaves them NULL when a subdomain has more than kDictMax
-// distinct offsets or memory is short (the kernels then read the int32 columns).
+// distinct offsets or memory is short (the kernels then read the int32 columns). With them, the
+// staged-gather tables (Layout::sdict / iv / xs_len) when every subdomain's off-block columns fit
+// its intervals (else xs_len = 0: the coded kernels gather from global memory).
 static void build_codes(Layout &L, cudaStream_t st) {
     const int64_t q = L.q;
-    int32_t *dtmp = nullptr, *dcount = nullptr, *dsize = nullptr;
+    int32_t *dtmp = nullptr, *stmp = nullptr, *dcount = nullptr, *dsize = nullptr, *ivlen = nullptr, *red = nullptr;
     void *tmp = nullptr;
     size_t tb = 0;
-    int32_t mn = 0, total = 0;
+    int32_t mn = 0, total = 0, ivmin = -1, ivmax = 0;
     bool ok = false;
     if (cudaMalloc(&L.codes, (size_t)L.entries + 16) != cudaSuccess ||
         cudaMalloc(&dtmp, sizeof(int32_t) * (size_t)q * kDictMax) != cudaSuccess ||
+        cudaMalloc(&stmp, sizeof(int32_t) * (size_t)q * kDictMax) != cudaSuccess ||
         cudaMalloc(&dcount, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess ||
         cudaMalloc(&dsize, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess ||
+        cudaMalloc(&ivlen, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess ||
+        cudaMalloc(&red, sizeof(int32_t) * 2) != cudaSuccess ||
+        cudaMalloc(&L.iv, sizeof(int32_t) * 4 * (size_t)q * kMaxIv) != cudaSuccess ||
         cudaMalloc(&L.dptr, sizeof(int32_t) * (size_t)(q + 1)) != cudaSuccess)
         goto out;
-    k_codes<<<(unsigned)q, 256, 0, st>>>(L.n, L.R, L.spb, L.sptr, L.sw, L.col, L.codes, dtmp, dcount);
+    k_codes<<<(unsigned)q, 256, 0, st>>>(L.n, L.R, L.spb, L.sptr, L.sw, L.col, L.codes, dtmp, stmp, dcount, L.iv,
+                                        ivlen);
     if (cub::DeviceReduce::Min(nullptr, tb, dcount, dsize + q, q, st) != cudaSuccess) goto out;
     {
         size_t tb2 = 0;
         if (cub::DeviceScan::ExclusiveSum(nullptr, tb2, dsize, L.dptr, q + 1, st) != cudaSuccess) goto out;
+        if (tb2 > tb) tb = tb2;
+        if (cub::DeviceReduce::Max(nullptr, tb2, ivlen, red + 1, q, st) != cudaSuccess) goto out;
         if (tb2 > tb) tb = tb2;
     }
     if (cudaMalloc(&tmp, tb) != cudaSuccess) goto out;
@@ -340,6 +450,13 @@ static void build_codes(Layout &L, cudaStream_t st) {
         if (cudaMemcpyAsync(&mn, dsize + q, sizeof(int32_t), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
             cudaStreamSynchronize(st) != cudaSuccess || mn < 1)
             goto out;
+        t = tb;
+        if (cub::DeviceReduce::Min(tmp, t, ivlen, red, q, st) != cudaSuccess) goto out;
+        t = tb;
+        if (cub::DeviceReduce::Max(tmp, t, ivlen, red + 1, q, st) != cudaSuccess) goto out;
+        if (cudaMemcpyAsync(&ivmin, red, sizeof(int32_t), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+            cudaMemcpyAsync(&ivmax, red + 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st) != cudaSuccess)
+            goto out;
         k_dict_pad<<<(unsigned)((q + 1 + 255) / 256), 256, 0, st>>>(q, dcount, dsize);
         t = tb;
         if (cub::DeviceScan::ExclusiveSum(tmp, t, dsize, L.dptr, q + 1, st) != cudaSuccess) goto out;
@@ -347,24 +464,35 @@ static void build_codes(Layout &L, cudaStream_t st) {
             cudaStreamSynchronize(st) != cudaSuccess)
             goto out;
     }
-    if (cudaMalloc(&L.dict, sizeof(int32_t) * (size_t)(total + 4)) != cudaSuccess) goto out;
-    k_dict_compact<<<(unsigned)q, 64, 0, st>>>(q, dtmp, dcount, L.dptr, L.dict);
+    if (cudaMalloc(&L.dict, sizeof(int32_t) * (size_t)(total + 4)) != cudaSuccess ||
+        cudaMalloc(&L.sdict, sizeof(int32_t) * (size_t)(total + 4)) != cudaSuccess)
+        goto out;
+    k_dict_compact<<<(unsigned)q, 64, 0, st>>>(q, dtmp, stmp, dcount, L.dptr, L.dict, L.sdict);
     ok = cudaStreamSynchronize(st) == cudaSuccess && cudaGetLastError() == cudaSuccess;
     L.dict_entries = total;
+    L.xs_len = ivmin >= 0 ? ((ivmax + 1) & ~1) : 0;  // staged gathers for every subdomain, or none
 out:
     cudaGetLastError();
     cudaFree(dtmp);
+    cudaFree(stmp);
     cudaFree(dcount);
     cudaFree(dsize);
+    cudaFree(ivlen);
+    cudaFree(red);
     cudaFree(tmp);
     if (!ok) {
         cudaFree(L.codes);
         cudaFree(L.dict);
         cudaFree(L.dptr);
+        cudaFree(L.sdict);
+        cudaFree(L.iv);
         L.codes = nullptr;
         L.dict = nullptr;
         L.dptr = nullptr;
+        L.sdict = nullptr;
+        L.iv = nullptr;
         L.dict_entries = 0;
+        L.xs_len = 0;
     }
 }
 

@@ -58,9 +58,13 @@ struct KP {
     const int32_t *gr;      // ghost-range table (Layout::gr): L2 prefetch targets of the a3 gathers
     int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
+    int fronts;             // > 0: F fronts (claims_of), async_order = 3
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
+    const int32_t *sdict;   // staged gathers (Layout::sdict / iv / xs_len): shared-memory index
+    const int32_t *iv;      //   offsets per code, the subdomain's x intervals, their buffer length
+    int32_t xs_len;
     int init_check;         // residual kernels: the last block also applies the x^(0) check
 };
 
@@ -74,8 +78,18 @@ struct Claims {
     long long l0, step, lend;
 };
 
+// A third order, F "fronts" (tuning.async_order = 3): the subdomains are cut into F contiguous
+// ranges and the G / F blocks of front f sweep range f round robin, so each front advances as one
+// narrow window of G / F subdomains (F = 1 is round robin over the whole matrix, F = G the chunks).
+// A subdomain's far couplings (the plane below on a 3D grid) then lie many rounds back in its
+// front, and the x written meanwhile is F windows of about one plane — small enough for L2.
 __device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
     const long long G = gridDim.x, c = blockIdx.x;
+    if (p.fronts > 0) {
+        const long long F = p.fronts, Gf = G / F, f = c / Gf;
+        if (f >= F) return {0, 1, 0};  // G not a multiple of F: the remainder blocks idle
+        return {f * (long long)q / F + c % Gf, Gf, (f + 1) * (long long)q / F};
+    }
     if (p.claim_chunk) return {c * (long long)q / G, 1, (c + 1) * (long long)q / G};
     return {c, G, (long long)q};
 }
@@ -1022,12 +1036,13 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
 // Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
 struct DuoGeom {
-    uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, bytes;
+    uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, o_xs, bytes;
 };
 
-// CODED: the column block holds 1-byte codes and is followed by the subdomain's dictionary
-// (<= kDictMax int32 offsets); otherwise int32 columns.
-__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, bool coded = false) {
+// coded: the column block holds 1-byte codes and is followed by the subdomain's dictionary
+// (<= kDictMax int32 offsets); otherwise int32 columns. xs_len > 0 (staged gathers): a buffer
+// of xs_len doubles for the subdomain's off-block x intervals.
+__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, bool coded = false, int xs_len = 0) {
     DuoGeom g;
     g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
     g.o_col = g.vcap * 8;
@@ -1036,11 +1051,16 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
     g.o_sw = g.o_sptr + (((uint32_t)spb * 8 + 15) & ~15u);
     g.o_ya = (g.o_sw + (((uint32_t)spb * 4 + 15) & ~15u) + 127) & ~127u;
     g.o_yb = g.o_ya + (uint32_t)R * 8;
-    g.bytes = g.o_yb + (uint32_t)R * 8;
+    g.o_xs = g.o_yb + (uint32_t)R * 8;
+    g.bytes = g.o_xs + (uint32_t)xs_len * 8;
     return g;
 }
 
-template <bool ASYNC, int WLR, bool EXT = false, bool CODED = false>
+// CODED: 0 int32 columns; 1 coded columns, off-block x gathered entry by entry from global
+// memory (relaxed loads); 2 coded columns with STAGED gathers: at the start of each subdomain the
+// block copies its off-block x intervals (Layout::iv, at most kMaxIv, x "as it stands", relaxed
+// loads, one coalesced pass) into shared memory, and phase 1 reads x there (Layout::sdict).
+template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     if (*(volatile int *)&p.state->stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
@@ -1048,8 +1068,9 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
     __shared__ __align__(16) int32_t gsm[4][2 * kGhostRanges];  // [j % 4]: ghost ranges of l_j
     __shared__ __align__(16) int32_t dbd[4][2];                 // [j % 4]: dictionary D0, D1 (CODED)
+    __shared__ __align__(16) int32_t ivs[CODED == 2 ? 4 : 1][4 * kMaxIv];  // [j % 4]: x intervals of l_j
     const int R = p.R, spb = p.spb;
-    const DuoGeom g = duo_geom(R, spb, p.wmax, CODED);
+    const DuoGeom g = duo_geom(R, spb, p.wmax, CODED != 0, CODED == 2 ? p.xs_len : 0);
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;  // = spb / 2
@@ -1089,7 +1110,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             if (CODED) {
                 const int32_t *db = dbd[j & 3];
                 bulk_g2s_hint(smraw + g.o_col, p.codes + bd[0], ne, &bar, policy_evict_first());
-                bulk_g2s(smraw + g.o_dict, p.dict + db[0], (uint32_t)(db[1] - db[0]) * 4, &bar);
+                bulk_g2s(smraw + g.o_dict, (CODED == 2 ? p.sdict : p.dict) + db[0], (uint32_t)(db[1] - db[0]) * 4,
+                         &bar);
             } else {
                 bulk_g2s_hint(smraw + g.o_col, p.col + bd[0], ne * 4, &bar, policy_evict_first());
             }
@@ -1123,6 +1145,13 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(&dbd[r][1])), "l"(p.dptr + l + 1)
                          : "memory");
         }
+        if (CODED == 2) {
+#pragma unroll
+            for (int t = 0; t < kMaxIv; ++t)
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(&ivs[r & 3][4 * t])),
+                             "l"(p.iv + 4 * (l * kMaxIv + t))
+                             : "memory");
+        }
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
     if (threadIdx.x == 0) {  // prologue: ring slots of l_0 .. l_2, the slab of l_0
@@ -1138,10 +1167,16 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 dbd[j][0] = p.dptr[l];
                 dbd[j][1] = p.dptr[l + 1];
             }
+            if (CODED == 2)
+                for (int t = 0; t < 4 * kMaxIv; ++t) ivs[j & 3][t] = p.iv[4 * l * kMaxIv + t];
         }
         mbar_arrive_expect_tx(&bar, slab_bytes(lof(0), bnd[0], dbd[0]));
         for (int w = 0; w < 4; ++w) issue_part(w, 0);
     }
+    double *xs = reinterpret_cast<double *>(smraw + g.o_xs);
+    const uint32_t sxs = smem_u32(xs);
+    if (CODED == 2)  // slots past a subdomain's intervals are read (times 0) by padding entries
+        for (int t = threadIdx.x; t < p.xs_len; t += blockDim.x) xs[t] = 0.0;
     __syncthreads();
 
     constexpr int NP = WLR / 2;
@@ -1152,6 +1187,15 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
+        if (CODED == 2) {  // a3 staged: the off-block x intervals, as they stand, into shared memory
+            const int32_t *iv = ivs[i & 3];
+#pragma unroll
+            for (int t = 0; t < kMaxIv; ++t) {
+                const int32_t lo = iv[4 * t], len = iv[4 * t + 1], base = iv[4 * t + 2];
+                for (int u = threadIdx.x; u < len; u += blockDim.x) xs[base + u] = ldx<ASYNC>(p.x_in + lo + u);
+            }
+            __syncthreads();
+        }
         mbar_wait(&bar, i & 1);
         double lv[2][WLR];
         uint32_t lc[2][NP];
@@ -1187,8 +1231,11 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             for (int e0 = 0; e0 < wo; e0 += U) {
                 double xv[U];
 #pragma unroll
-                for (int u = 0; u < U; ++u)
-                    if (e0 + u < wo) xv[u] = ldx<ASYNC>(p.x_in + (CODED ? TS + loc : 0) + dcol(e0 + u));
+                for (int u = 0; u < U; ++u) {
+                    if (e0 + u >= wo) continue;
+                    if (CODED == 2) xv[u] = lds_f64(sxs + 8u * (uint32_t)(loc + dcol(e0 + u)));
+                    else xv[u] = ldx<ASYNC>(p.x_in + (CODED ? TS + loc : 0) + dcol(e0 + u));
+                }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (e0 + u < wo) acc -= lds_f64(av + (e0 + u) * kSlice * 8) * xv[u];
@@ -1232,20 +1279,45 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         // before the write-back (the barrier after it guards the buffers' reuse)
         if (p.k > 1) __syncthreads();
         // a4: sweeps 2..k, direct form, off-block part frozen
-        for (int t = 1; t < p.k; ++t) {
-            const double *yi = (t & 1) ? yb : ya;
-            double *yo = (t & 1) ? ya : yb;
+        if (EXT) {
+            for (int t = 1; t < p.k; ++t) {
+                const double *yi = (t & 1) ? yb : ya;
+                double *yo = (t & 1) ? ya : yb;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int loc = row_of(h);
+                    if (warp + h * nw >= nsl || loc >= nrows) continue;
+                    double acc = s[h];
+#pragma unroll
+                    for (int e = 1; e < WLR; ++e) acc -= lv[h][e] * yi[(lc[h][e >> 1] >> (16 * (e & 1))) & 0xffff];
+                    yo[loc] = ext_update(yi[loc], lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
+                }
+                if (t + 1 < p.k) __syncthreads();
+            }
+        } else {
+            // straight-line: row addresses and y indices hoisted out of the sweep loop, rows past
+            // the subdomain's end (partial last subdomain) computed on zeroed entries and not stored
+            const uint32_t ya_s = smem_u32(ya), yb_s = smem_u32(yb);
+            uint32_t yoff[2][WLR], sto[2];
+            bool vh[2];
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-                const int loc = row_of(h);
-                if (warp + h * nw >= nsl || loc >= nrows) continue;
-                double acc = s[h];
+                vh[h] = warp + h * nw < nsl && row_of(h) < nrows;
+                sto[h] = 8u * (uint32_t)row_of(h);
 #pragma unroll
-                for (int e = 1; e < WLR; ++e) acc -= lv[h][e] * yi[(lc[h][e >> 1] >> (16 * (e & 1))) & 0xffff];
-                if (EXT) yo[loc] = ext_update(yi[loc], lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
-                else yo[loc] = lv[h][0] * acc;
+                for (int e = 1; e < WLR; ++e) yoff[h][e] = 8u * ((lc[h][e >> 1] >> (16 * (e & 1))) & 0xffffu);
             }
-            if (t + 1 < p.k) __syncthreads();
+            for (int t = 1; t < p.k; ++t) {
+                const uint32_t yi = (t & 1) ? yb_s : ya_s, yo = (t & 1) ? ya_s : yb_s;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    double acc = s[h];
+#pragma unroll
+                    for (int e = 1; e < WLR; ++e) acc -= lv[h][e] * lds_f64(yi + yoff[h][e]);
+                    if (vh[h]) sts_f64(yo + sto[h], lv[h][0] * acc);
+                }
+                if (t + 1 < p.k) __syncthreads();
+            }
         }
         // ring slot of l_{i+2} complete before the barrier below publishes it
         if (warp == 3 && lane == 0) asm volatile("cp.async.wait_group 1;" ::: "memory");
@@ -2100,9 +2172,10 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
 template <bool ASYNC, int WLR>
 cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
-    const bool coded = p.codes != nullptr;
-    auto kfn = coded ? (ext ? k_block_duo<ASYNC, WLR, true, true> : k_block_duo<ASYNC, WLR, false, true>)
-                     : (ext ? k_block_duo<ASYNC, WLR, true> : k_block_duo<ASYNC, WLR, false>);
+    const int coded = p.codes == nullptr ? 0 : (p.sdict != nullptr ? 2 : 1);
+    auto kfn = coded == 2 ? (ext ? k_block_duo<ASYNC, WLR, true, 2> : k_block_duo<ASYNC, WLR, false, 2>)
+               : coded == 1 ? (ext ? k_block_duo<ASYNC, WLR, true, 1> : k_block_duo<ASYNC, WLR, false, 1>)
+                            : (ext ? k_block_duo<ASYNC, WLR, true, 0> : k_block_duo<ASYNC, WLR, false, 0>);
     const int threads = L.spb / 2 * kSlice;
     std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
     cudaError_t e = ensure_smem(kfn, smem);
@@ -2189,6 +2262,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // the neighbouring lines / planes below a subdomain already hold this iteration's values.
     // (sync modes: the order does not change the iterates; round robin)
     p.claim_chunk = T.async_order == 0 ? (ASYNC ? 1 : 0) : (T.async_order == 1 ? 1 : 0);
+    p.fronts = T.async_order == 3 ? (T.fronts > 0 ? T.fronts : 8) : 0;
     const size_t tma_smem = (size_t)L.spb * slice_buf_bytes(L.max_w) + 2 * (size_t)L.R * sizeof(double);
     const size_t pers_smem = tma_smem + (size_t)L.spb * slice_buf_bytes(L.max_w);
     const size_t stage_smem = 2 * (size_t)stage_geom(L.R, L.spb, L.max_w).bytes + (size_t)L.R * sizeof(double);
@@ -2210,7 +2284,13 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     // vs 2.67 ms per launch); coded columns (Layout::codes, 1 byte per entry instead of 4) when
     // the layout has them
     const bool coded = L.codes != nullptr && T.coded >= 0;
-    const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w, coded).bytes;
+    // staged gathers (CODED = 2, tuning.coded = 2) where every subdomain's off-block columns fit
+    // its x intervals. Not the default: measured on B200 (round 2, tools/kernel_ab.py, async-(5))
+    // C4 0.474 vs 0.335 ms and C5 2.83 vs 2.42 ms per launch against the entry-by-entry relaxed
+    // gathers (one more barrier per subdomain; on C4 the buffer costs a block per SM; on C5 each
+    // ghost value is used once, so staging adds shared-memory traffic and saves no global loads)
+    const bool staged = coded && L.sdict != nullptr && L.xs_len > 0 && T.coded == 2;
+    const size_t duo_smem = duo_geom(L.R, L.spb, L.max_w, coded, staged ? (int)L.xs_len : 0).bytes;
     const bool duo_fits = L.spb % 2 == 0 && L.spb >= 8 && L.max_wl <= 4 && 2 * (duo_smem + 2048) <= 228 * 1024;
     // Async: two blocks per SM whenever they fit (C5 R = 1024: 2.69 vs 2.93 ms per launch with
     // chunked claims; C4 R = 512: 0.40 vs 0.52 ms). With round-robin claims the 2 x 148
@@ -2219,13 +2299,19 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
     const bool duo_on = (T.duo ? T.duo > 0 : ((ASYNC && p.claim_chunk) || pipe_smem > 113 * 1024)) && duo_fits &&
                         (!ASYNC || p.static_claims);
     if (kind == 0 && duo_on && p.w_end == 0 && geom_ok && aligned) {
-        L.last_kernel = coded ? (ASYNC ? "k_block_duo<async,coded>" : "k_block_duo<sync,coded>")
-                              : (ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>");
+        L.last_kernel = staged  ? (ASYNC ? "k_block_duo<async,staged>" : "k_block_duo<sync,staged>")
+                        : coded ? (ASYNC ? "k_block_duo<async,coded>" : "k_block_duo<sync,coded>")
+                                : (ASYNC ? "k_block_duo<async>" : "k_block_duo<sync>");
         KP pc = p;
         if (coded) {
             pc.codes = L.codes;
             pc.dict = L.dict;
             pc.dptr = L.dptr;
+        }
+        if (staged) {
+            pc.sdict = L.sdict;
+            pc.iv = L.iv;
+            pc.xs_len = (int32_t)L.xs_len;
         }
         return launch_duo_t<ASYNC, 4>(pc, L, duo_smem, st);  // two rows per thread: <= 4 local entries
     }

@@ -151,11 +151,11 @@ def test_history_matches_oracle(bar, mode, k):
     np.testing.assert_allclose(h, r.history, rtol=1e-9, atol=1e-15)
 
 
-@pytest.mark.parametrize("coded", ["1", "0"])
+@pytest.mark.parametrize("coded", [0, 2, -1])
 def test_ext_options_on_duo_kernel(bar, coded):
     """N3 tau-scaling and N1 failure windows through the two-blocks-per-SM kernel's EXT
     instantiations (coded and int32 columns): iterates match the oracle to 1e-12."""
-    tune = {"duo": 1, "coded": 0 if coded == "1" else -1}
+    tune = {"duo": 1, "coded": coded}
     A = W.stencil7_3d(128)  # R = two grid lines: <= 4 local entries per row
     R = 256
     b = np.ones(A.n)

@@ -399,7 +399,7 @@ def test_forced_kernel_paths(bar, tune, name, R):
 def test_tuning_validation(bar):
     A = W.trefethen(64)
     M = bar.Matrix.from_csr(A, 16)
-    for bad in ({"kernel": 9}, {"lead": 49}, {"async_order": 3}, {"halo": 2}, {"warps": 33}, {"peer": 1}):
+    for bad in ({"kernel": 9}, {"lead": 49}, {"async_order": 4}, {"halo": 2}, {"warps": 33}, {"peer": 1}):
         with pytest.raises(bar.BarError):
             M.set_tuning(bad)
     with pytest.raises(KeyError):
@@ -410,7 +410,8 @@ def test_tuning_validation(bar):
 
 # ------------------------------------------------------------------ pipelined / two-blocks-per-SM
 @pytest.mark.parametrize("tune", [{"duo": 1}, {"duo": -1}, {"duo": -1, "pipe": -1}, {"duo": 1, "coded": -1},
-                                  {"async_order": "round_robin"}, {"async_order": "chunks"}])
+                                  {"duo": 1, "coded": 2}, {"async_order": "round_robin"}, {"async_order": "chunks"},
+                                  {"async_order": "fronts", "fronts": 4}])
 def test_large_subdomain_kernels(bar, tune):
     """C5's shape at a testable size: 3D 7-point, m = 128, R = 256 = two grid lines (so a row has
     at most 4 local entries, as at 512^3 with R = 1024). The two-blocks-per-SM kernel
@@ -442,14 +443,18 @@ def test_coded_columns(bar):
     b = _dev(np.ones(A.n))
     x0 = _dev(np.random.default_rng(9).uniform(-1, 1, A.n))
     out = {}
-    for coded in ("1", "0"):  # the sync modes pick the duo kernel only for larger slabs: force it
-        M.set_tuning(duo=1, coded=0 if coded == "1" else -1)
+    names = {2: "staged", 1: "coded", 0: "coded", -1: None}
+    for coded in (2, 1, 0, -1):  # the sync modes pick the duo kernel only for larger slabs: force it
+        M.set_tuning(duo=1, coded=coded)
         for mode, k in (("sync-block", 5), ("jacobi", 1)):
             x, info = M.solve(b, x0, k=k, max_global_iters=4, tol=0.0, mode=mode)
             out[coded, mode] = x.cpu().numpy()
-            assert ("coded" in M.info()["last_sweep_kernel"]) == (coded == "1")
-    for mode in ("sync-block", "jacobi"):
-        assert np.array_equal(out["1", mode], out["0", mode])
+            kern = M.info()["last_sweep_kernel"]
+            assert (names[coded] in kern) if names[coded] else ("," not in kern), (coded, kern)
+    for mode in ("sync-block", "jacobi"):  # staged gathers, coded columns, int32 columns: the same bits
+        assert np.array_equal(out[1, mode], out[-1, mode])
+        assert np.array_equal(out[0, mode], out[-1, mode])
+        assert np.array_equal(out[2, mode], out[-1, mode])
     R = W.random_dd(4096, nnz_per_row=7, seed=3)
     MR = bar.Matrix.from_csr(R, 1024)
     assert MR.info()["coded"] == 0
@@ -518,12 +523,12 @@ def test_graph_replay(bar):
     M.close()
 
 
-@pytest.mark.parametrize("coded", ["1", "0"])
+@pytest.mark.parametrize("coded", [0, 2, -1])
 def test_duo_partial_last_subdomain(bar, coded):
     """The two-blocks-per-SM kernel (coded and int32 columns) on a 2D 9-point stencil whose last
     subdomain is partial (n = 10^6 is not a multiple of R = 512, so its last slices are short and
     padded): sync-block-(5) and Jacobi iterates match the oracle to 1e-12, async converges."""
-    tune = {"duo": 1, "coded": 0 if coded == "1" else -1}
+    tune = {"duo": 1, "coded": coded}
     A = W.stencil9_2d(1000)
     R = 512
     b = np.ones(A.n)
@@ -536,3 +541,37 @@ def test_duo_partial_last_subdomain(bar, coded):
         _close(x, ref)
     x, info = _solve(bar, A, b, R, 5, "async", 20000, 1e-10, tuning=tune)
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
+
+
+@pytest.mark.parametrize("name,gen,R", [("s7_m64", lambda: W.stencil7_3d(64), 256),
+                                        ("s9_m300", lambda: W.stencil9_2d(300), 512),
+                                        ("s7_m40", lambda: W.stencil7_3d(40), 320)])
+def test_staged_gathers(bar, name, gen, R):
+    """Staged gathers (k_block_duo<.., staged>: each subdomain's off-block x intervals copied into
+    shared memory once per visit, Layout::iv / sdict): chosen for stencil matrices (3D grid planes
+    and lines, 2D lines, subdomains that straddle grid lines, a partial last subdomain), sync-block
+    and Jacobi iterates match the oracle to 1e-12 in every mode, async converges."""
+    A = gen()
+    b = np.ones(A.n)
+    x0 = np.random.default_rng(21).uniform(-1, 1, A.n)
+    M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "coded": 2})
+    import torch
+
+    for mode, k in (("sync-block", 5), ("jacobi", 1), ("sync-block", 2)):
+        ref = x0
+        for m in range(1, 4):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x = torch.empty(A.n, dtype=torch.float64, device="cuda")
+        M.solve(_dev(b), _dev(x0), x, k=k, max_global_iters=3, tol=0.0, mode=mode)
+        assert "staged" in M.info()["last_sweep_kernel"], M.info()["last_sweep_kernel"]
+        _close(x.cpu().numpy(), ref)
+    x, info = M.solve(_dev(b), None, None, k=5, tol=1e-10, mode="async")
+    assert "staged" in M.info()["last_sweep_kernel"]
+    assert info["converged"] and O.rel_res(A, b, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    M.close()
+    # matrices whose off-block columns are not a few intervals keep the entry-by-entry gathers
+    Rm = W.random_dd(8192, nnz_per_row=5, seed=9, symmetric_pattern=True)
+    MR = bar.Matrix.from_csr(Rm, 512, tuning={"duo": 1, "coded": 2})
+    MR.solve(_dev(np.ones(Rm.n)), None, None, k=5, max_global_iters=2, tol=0.0, mode="sync-block")
+    assert "staged" not in MR.info()["last_sweep_kernel"]
+    MR.close()
