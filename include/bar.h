@@ -230,6 +230,9 @@ typedef struct {
                                1 one ncclAllGather per iteration                                 */
     int32_t peer;           /* multi-GPU async: 0 peer memory when mapped, -1 the collective path */
     int32_t fronts;         /* async_order = 3: number of fronts (0 = 8)                          */
+    int32_t overlap;        /* multi-GPU collective path: 0 sweep the interior subdomains (no ghost
+                               reads) on a second stream while the halo exchange runs, then the
+                               boundary ones; -1 one sweep after the exchange                    */
 } bar_tuning;
 
 /* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a

@@ -243,6 +243,9 @@ struct SweepArgs {
     const uint8_t *frozen = nullptr;  // N1: rows that do not update in this launch (nullable)
     double tau = 1.0;                 // N3: relaxation weight, B = I - tau D^-1 A
     long long m0 = 0;                 // single-launch async: global iteration of the first sweep
+    int64_t l_begin = 0, l_end = 0;   // sweep only subdomains [l_begin, l_end) (l_end = 0: all);
+                                      // cudaErrorNotSupported where the chosen kernel cannot
+    const int *stop = nullptr;        // stop flag polled by the kernels (nullptr: state->stop)
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);

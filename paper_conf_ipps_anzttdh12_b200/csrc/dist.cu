@@ -74,6 +74,14 @@ struct bar_dist_s {
     bool loopback = false;                        // ranks of one process, linked (bar_dist_link_loopback)
     bool has_nccl = false;
     bool owner_handle = false;                    // A was returned by bar_create_csr_dist (A->dist == this)
+    // interior / boundary overlap of the collective path: subdomains [ib, ie) read no ghost, so
+    // they are swept on a second stream while the halo exchange runs; the boundary ones follow it
+    int64_t ib = 0, ie = 0;                       // interior subdomains (ib >= ie: none)
+    cudaStream_t s2 = nullptr;                    // interior stream
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    bar::DevState *state2 = nullptr;              // the interior launches' reduction state
+    double *partials2 = nullptr;                  // and per-block partials
+    double *parts3 = nullptr;                     // device [6]: [lo | interior | hi] partial sums
     std::vector<bar_dist> peers;                  // loopback group (peers[r] is rank r)
 #ifdef BAR_WITH_NCCL
     ncclComm_t comm = nullptr;
@@ -237,6 +245,13 @@ __global__ void k_board_barrier(DevState *S, const double *board, double *const 
 // the estimate above tol until every rank has published once).
 __global__ void k_board_reset(double *board, int P) {
     for (int i = threadIdx.x; i < 2 * P; i += blockDim.x) board[i] = 1e300;
+}
+
+// Overlap: this rank's [sum r^2, sum b^2] from the three launches, in a fixed order.
+__global__ void k_sum_parts(const double *__restrict__ p3, const bar::DevState *S, double *__restrict__ part) {
+    if (S->stop) return;  // queued iterations after the stop: nothing was swept
+    part[0] = (p3[0] + p3[2]) + p3[4];
+    part[1] = (p3[1] + p3[3]) + p3[5];
 }
 
 // ---- planning (host) -----------------------------------------------------------------------
@@ -646,6 +661,68 @@ bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, doub
     return BAR_OK;
 }
 
+// Lazily created resources of the overlapped collective iteration.
+bar_status ensure_overlap(bar_dist D) {
+    if (D->s2) return BAR_OK;
+    BAR_CUDA(cudaStreamCreateWithFlags(&D->s2, cudaStreamNonBlocking));
+    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_fork, cudaEventDisableTiming));
+    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_join, cudaEventDisableTiming));
+    BAR_CUDA(cudaMalloc(&D->state2, sizeof(DevState)));
+    BAR_CUDA(cudaMemset(D->state2, 0, sizeof(DevState)));
+    BAR_CUDA(cudaMalloc(&D->partials2, sizeof(double) * 2 * (size_t)num_blocks_for(D->A->L, BAR_MODE_SYNC_BLOCK)));
+    BAR_CUDA(cudaMalloc(&D->parts3, sizeof(double) * 6));
+    return BAR_OK;
+}
+
+// One global iteration of the collective path with the interior subdomains swept on the second
+// stream while the exchange runs (every rank of `ranks`): fork -> interior sweeps on s2 ||
+// exchange + low and high boundary sweeps on st -> join -> partial sums. Returns
+// cudaErrorNotSupported (nothing enqueued) where the sweep kernel cannot take subdomain ranges.
+bar_status overlapped_iteration(bar_dist *ranks, int nr, double *const *vin, double *const *vout, int32_t k,
+                                bar_mode mode, cudaStream_t st, bool &supported) {
+    bar_status r;
+    supported = true;
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        if ((r = ensure_overlap(D)) != BAR_OK) return r;
+        BAR_CUDA(cudaEventRecord(D->ev_fork, st));
+        BAR_CUDA(cudaStreamWaitEvent(D->s2, D->ev_fork, 0));
+        SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->state2, D->partials2, nullptr,
+                    D->parts3 + 2};
+        a.l_begin = D->ib;
+        a.l_end = D->ie;
+        a.stop = &D->A->W.state->stop;
+        const cudaError_t e = launch_sweep(a, mode, D->s2);
+        if (e == cudaErrorNotSupported) {
+            cudaGetLastError();
+            supported = false;
+            return BAR_OK;
+        }
+        BAR_CUDA(e);
+        BAR_CUDA(cudaEventRecord(D->ev_join, D->s2));
+    }
+    if ((r = exchange(ranks, nr, vin, st)) != BAR_OK) return r;
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        const int64_t q = D->A->L.q;
+        for (int side = 0; side < 2; ++side) {
+            SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state, D->A->W.partials,
+                        nullptr, D->parts3 + (side ? 4 : 0)};
+            a.l_begin = side ? D->ie : 0;
+            a.l_end = side ? q : D->ib;
+            if (a.l_end <= a.l_begin) {  // empty side: a zero partial
+                BAR_CUDA(cudaMemsetAsync(D->parts3 + (side ? 4 : 0), 0, 2 * sizeof(double), st));
+                continue;
+            }
+            BAR_CUDA(launch_sweep(a, mode, st));
+        }
+        BAR_CUDA(cudaStreamWaitEvent(st, D->ev_join, 0));
+        k_sum_parts<<<1, 1, 0, st>>>(D->parts3, D->A->W.state, D->part);
+        BAR_CUDA(cudaGetLastError());
+    }
+    return BAR_OK;
+}
+
 // The solve for the ranks this process drives (1 with NCCL / separate processes, all with
 // loopback). b, x0, x are each rank's owned rows (device or host).
 bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const double *const *x0, double *const *x,
@@ -693,6 +770,10 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
     timer_reset(T);
     int64_t issued = 0, chunk = 8;
     ChunkSizer sizer;  // sized from the agreed state (identical on every rank)
+    // interior / boundary overlap: every rank of this process has an interior, and the tuning
+    // allows it (the kernel's support for subdomain ranges is found at the first iteration)
+    bool overlap = D0->A->L.tune.overlap >= 0 && D0->nranks > 1;
+    for (int i = 0; i < nr; ++i) overlap = overlap && ranks[i]->ib < ranks[i]->ie;
     int64_t iters = 0;
     double rel = 0.0;
     int converged = 0;
@@ -708,17 +789,32 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
                 const bool odd = (m & 1) || mode == BAR_MODE_ASYNC;
                 const std::vector<double *> &vin = odd ? xa : xb;
                 const std::vector<double *> &vout = mode == BAR_MODE_ASYNC ? xa : (odd ? xb : xa);
-                if ((r = exchange(ranks, nr, vin.data(), st)) != BAR_OK) return r;
-                for (int i = 0; i < nr; ++i) {
-                    bar_dist D = ranks[i];
-                    SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state,
-                                D->A->W.partials, nullptr, D->part};
-                    if (i == 0 && (r = timer_begin(T, m, st)) != BAR_OK) return r;
-                    BAR_CUDA(launch_sweep(a, mode, st));
-                    if (i == 0 && (r = timer_end(T, st)) != BAR_OK) return r;
+                bool done = false;
+                if (overlap) {  // interior sweeps on the second stream while the exchange runs
+                    if ((r = timer_begin(T, m, st)) != BAR_OK) return r;
+                    bool supported = true;
+                    if ((r = overlapped_iteration(ranks, nr, vin.data(), vout.data(), k, mode, st, supported)) != BAR_OK)
+                        return r;
+                    if ((r = timer_end(T, st)) != BAR_OK) return r;
+                    done = supported;
+                    if (!supported) {
+                        overlap = false;
+                        T.used = T.used > 0 ? T.used - 1 : 0;
+                    }
+                }
+                if (!done) {
+                    if ((r = exchange(ranks, nr, vin.data(), st)) != BAR_OK) return r;
+                    for (int i = 0; i < nr; ++i) {
+                        bar_dist D = ranks[i];
+                        SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state,
+                                    D->A->W.partials, nullptr, D->part};
+                        if (i == 0 && (r = timer_begin(T, m, st)) != BAR_OK) return r;
+                        BAR_CUDA(launch_sweep(a, mode, st));
+                        if (i == 0 && (r = timer_end(T, st)) != BAR_OK) return r;
+                    }
                 }
                 if ((r = reduce_decide(ranks, nr, false, st)) != BAR_OK) return r;
-                launches += 2 * nr;
+                launches += (done ? 5 : 2) * nr;  // overlapped: three sweeps and the partial sum
             }
             issued += c;
             if ((r = read_state(D0->A, st)) != BAR_OK) return r;
@@ -892,6 +988,26 @@ bar_status create_share(int64_t n_global, int64_t row_begin, int64_t row_end, in
         cudaFree(t_rp);
         cudaFree(t_col);
         cudaFree(t_val);
+    }
+    if (st == BAR_OK) {  // interior subdomains: [ib, ie) with no ghost column in any row
+        std::vector<int32_t> hrp = to_host(rowptr, nl + 1, st);
+        std::vector<int32_t> hcol = to_host(col_local, nnz_local, st);
+        const int64_t R = rows_per_block, q = (nl + R - 1) / R;
+        std::vector<uint8_t> glo(q, 0), ghi(q, 0);
+        for (int64_t i = 0; st == BAR_OK && i < nl; ++i)
+            for (int32_t e = hrp[i]; e < hrp[i + 1]; ++e) {
+                if (hcol[e] < 0) glo[i / R] = 1;
+                else if (hcol[e] >= nl) ghi[i / R] = 1;
+            }
+        int64_t ib = 0, ie = q;
+        for (int64_t l = 0; l < q; ++l)
+            if (glo[l]) ib = l + 1;
+        for (int64_t l = q - 1; l >= 0; --l)
+            if (ghi[l]) ie = l;
+        bool clean = ib < ie;
+        for (int64_t l = ib; clean && l < ie; ++l) clean = !glo[l] && !ghi[l];
+        D->ib = clean ? ib : 0;
+        D->ie = clean ? ie : 0;
     }
     if (st == BAR_OK) {
         std::vector<int32_t> hidx = to_host(send_idx, nsend, st);
@@ -1422,6 +1538,12 @@ void bar_dist_destroy(bar_dist D) {
     cudaFree(D->d_peer_board);
     cudaFree(D->board);
     cudaFreeHost(D->h_exact);
+    if (D->s2) cudaStreamDestroy(D->s2);
+    if (D->ev_fork) cudaEventDestroy(D->ev_fork);
+    if (D->ev_join) cudaEventDestroy(D->ev_join);
+    cudaFree(D->state2);
+    cudaFree(D->partials2);
+    cudaFree(D->parts3);
     if (D->A) {
         D->A->dist = nullptr;
         bar_destroy(D->A);

@@ -59,6 +59,8 @@ struct KP {
     int64_t grid_cap;       // > 0: at most this many persistent blocks (k_block_pipe / k_block_duo)
     int claim_chunk;        // static claims: contiguous chunks of subdomains instead of round robin
     int fronts;             // > 0: F fronts (claims_of), async_order = 3
+    int64_t l_begin, l_end; // subdomains this launch sweeps (l_end = 0: all; k_block_duo / _pipe only)
+    const int *stop;        // the stop flag the kernels poll at start (default &state->stop)
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
@@ -83,15 +85,18 @@ struct Claims {
 // narrow window of G / F subdomains (F = 1 is round robin over the whole matrix, F = G the chunks).
 // A subdomain's far couplings (the plane below on a 3D grid) then lie many rounds back in its
 // front, and the x written meanwhile is F windows of about one plane — small enough for L2.
+// Claims cover the subdomains [l_begin, l_end) (the whole matrix unless a multi-GPU rank sweeps
+// its interior and boundary subdomains in separate launches, dist.cu).
 __device__ __forceinline__ Claims claims_of(const KP &p, int64_t q) {
     const long long G = gridDim.x, c = blockIdx.x;
+    const long long b0 = p.l_begin, Q = (p.l_end > 0 ? p.l_end : (long long)q) - b0;
     if (p.fronts > 0) {
         const long long F = p.fronts, Gf = G / F, f = c / Gf;
         if (f >= F) return {0, 1, 0};  // G not a multiple of F: the remainder blocks idle
-        return {f * (long long)q / F + c % Gf, Gf, (f + 1) * (long long)q / F};
+        return {b0 + f * Q / F + c % Gf, Gf, b0 + (f + 1) * Q / F};
     }
-    if (p.claim_chunk) return {c * (long long)q / G, 1, (c + 1) * (long long)q / G};
-    return {c, G, (long long)q};
+    if (p.claim_chunk) return {b0 + c * Q / G, 1, b0 + (c + 1) * Q / G};
+    return {b0 + c, G, b0 + Q};
 }
 
 
@@ -836,7 +841,7 @@ __host__ __device__ __forceinline__ PipeGeom pipe_geom(int R, int spb, int wmax)
 // l_{i+2}, so no copy completes bytes before its phase expects them.
 template <bool ASYNC, int WLR, bool EXT = false>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_pipe(KP p) {
-    if (*(volatile int *)&p.state->stop) return;
+    if (*(volatile const int *)p.stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bars[3];
     __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
@@ -1062,7 +1067,7 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
 // loads, one coalesced pass) into shared memory, and phase 1 reads x there (Layout::sdict).
 template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
-    if (*(volatile int *)&p.state->stop) return;
+    if (*(volatile const int *)p.stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bar;
     __shared__ __align__(16) int64_t bnd[4][2];                // [j % 4]: E0, E1 of l_j
@@ -2126,7 +2131,8 @@ cudaError_t launch_reg_tma_t(const KP &p, const Layout &L, size_t smem, cudaStre
 int64_t persistent_grid(int per_sm, const KP &p, const Layout &L) {
     int64_t g = (int64_t)(per_sm < 1 ? 1 : per_sm) * L.sms;
     if (p.grid_cap > 0 && g > p.grid_cap) g = p.grid_cap;
-    return g < L.q ? g : L.q;
+    const int64_t nsub = p.l_end > 0 ? p.l_end - p.l_begin : L.q;
+    return g < nsub ? g : nsub;
 }
 
 template <bool ASYNC, int WLR>
@@ -2323,6 +2329,7 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
         if (L.max_wl <= 12) return launch_pipe_t<ASYNC, 12>(p, L, pipe_smem, st);  // <= 512 threads
         return launch_pipe_t<ASYNC, 16>(p, L, pipe_smem, st);
     }
+    if (p.l_end > 0) return cudaErrorNotSupported;  // subdomain ranges: k_block_duo / k_block_pipe only
     if (kind == 0 && geom_ok && aligned && stage_smem <= kSmemMax) {
         L.last_kernel = ASYNC ? "k_block_stage<async>" : "k_block_stage<sync>";
         if (L.max_wl <= 4) return launch_stage_t<ASYNC, 4>(p, L, stage_smem, st);
@@ -2423,6 +2430,9 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
     p.frozen = a.frozen;
     p.tau = a.tau;
     p.w_end = 0;
+    p.l_begin = a.l_begin;
+    p.l_end = a.l_end;
+    p.stop = a.stop ? a.stop : &a.state->stop;
     if (mode == BAR_MODE_JACOBI) {
         // Jacobi (eq. 2) is sync-block-(1) for any R, with the same per-row arithmetic
         // (off-block entries, then local ones, diagonal included): use the staged stream
@@ -2430,6 +2440,7 @@ cudaError_t launch_sweep(const SweepArgs &a, bar_mode mode, cudaStream_t st) {
             p.k = 1;
             return launch_block<false>(p, *a.L, st);
         }
+        if (p.l_end > 0) return cudaErrorNotSupported;
         return launch_rowwise<false>(p, *a.L, st);
     }
     if (mode == BAR_MODE_ASYNC) return launch_block<true>(p, *a.L, st);
@@ -2450,6 +2461,7 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
     p.tau = a.tau;
     p.w_end = w_end > 0 ? w_end : 1;
     p.m0 = a.m0;
+    p.stop = &a.state->stop;
     return launch_block<true>(p, *a.L, st);
 }
 

@@ -543,18 +543,18 @@ def test_duo_partial_last_subdomain(bar, coded):
     assert info["converged"] and O.rel_res(A, b, x) <= 1e-10 * (1 + 1e-6)
 
 
-@pytest.mark.parametrize("name,gen,R", [("s7_m64", lambda: W.stencil7_3d(64), 256),
-                                        ("s9_m300", lambda: W.stencil9_2d(300), 512),
-                                        ("s7_m40", lambda: W.stencil7_3d(40), 320)])
+@pytest.mark.parametrize("name,gen,R", [("s7_m128", lambda: W.stencil7_3d(128), 256),
+                                        ("s9_m600", lambda: W.stencil9_2d(600), 512),
+                                        ("s7_m192", lambda: W.stencil7_3d(192), 384)])
 def test_staged_gathers(bar, name, gen, R):
-    """Staged gathers (k_block_duo<.., staged>: each subdomain's off-block x intervals copied into
-    shared memory once per visit, Layout::iv / sdict): chosen for stencil matrices (3D grid planes
-    and lines, 2D lines, subdomains that straddle grid lines, a partial last subdomain), sync-block
-    and Jacobi iterates match the oracle to 1e-12 in every mode, async converges."""
+    """Staged gathers (k_block_duo<.., staged>, tuning.coded = 2: each subdomain's off-block x
+    intervals copied into shared memory once per visit, Layout::iv / sdict) on stencil matrices
+    (3D grid planes and lines, 2D subdomains that straddle grid lines with a partial last
+    subdomain): sync-block and Jacobi iterates match the oracle to 1e-12, async converges."""
     A = gen()
     b = np.ones(A.n)
     x0 = np.random.default_rng(21).uniform(-1, 1, A.n)
-    M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "coded": 2})
+    M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "coded": 2, "single_launch": -1})
     import torch
 
     for mode, k in (("sync-block", 5), ("jacobi", 1), ("sync-block", 2)):
