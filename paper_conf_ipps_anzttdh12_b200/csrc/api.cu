@@ -147,6 +147,7 @@ bar_status bar_create_csr(int64_t n, int64_t nnz, const int32_t *rowptr, const i
         set_error("rows_per_block out of [1, BAR_MAX_ROWS_PER_BLOCK]");
         return BAR_ERR_INVALID_ARG;
     }
+    NvtxRange nv("bar_create_csr (a1: validate, layout, codes)");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
         cudaGetLastError();
@@ -360,6 +361,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         return BAR_ERR_INVALID_ARG;
     }
     if (mode == BAR_MODE_JACOBI) k = 1;
+    NvtxRange nv(mode == BAR_MODE_ASYNC ? "bar_solve async" : mode == BAR_MODE_SYNC_BLOCK ? "bar_solve sync-block"
+                                                                                          : "bar_solve jacobi");
     if (A->dist) {  // one rank of a row-partitioned solve (collective over its group)
         if (opts && (opts->tau != 1.0 || opts->fail_mask || opts->res_history)) {
             set_error("bar_solve_ex options are not supported on multi-GPU handles");
@@ -440,6 +443,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
     auto next_chunk = [&](int64_t c) -> int64_t { return sizer.next(c, (long long)H.iter, H.last_rel, tol); };
 
     if (mode != BAR_MODE_ASYNC) {
+        NvtxRange nvs("global iterations (per-launch sweeps, fused residual)");
         int64_t issued = 0;  // launches m = 1..issued
         bool stopped = false;
         while (issued < max_global_iters && !stopped) {
@@ -643,6 +647,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                                                                            : (H.stop ? H.work_resume : H.work);
             cta_max = (int64_t)((claimed + L.q - 1) / L.q);
         }
+        NvtxRange nvs(multi ? "async: single-launch solve done; per-launch continuation"
+                            : "async: global iterations (per-launch sweeps)");
         while (!multi && !converged && !bzero && !diverged && H.iter < max_global_iters) {
             const int64_t c = std::min<int64_t>(chunk, max_global_iters - (int64_t)H.iter);
             for (int64_t i = 0; i < c; ++i) {

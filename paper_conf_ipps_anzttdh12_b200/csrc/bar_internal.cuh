@@ -21,9 +21,20 @@
 #include <algorithm>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "bar.h"
 
 namespace bar {
+
+// NVTX range for the phases of a call (SURVEY §5 tracing): visible in nsys / ncu timelines;
+// header-only NVTX3, a no-op unless a tool is attached.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 constexpr int kSlice = 32;  // rows per slice = warp width
 

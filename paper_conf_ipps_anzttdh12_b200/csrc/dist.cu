@@ -532,6 +532,7 @@ bar_status board_barrier(bar_dist *ranks, int nr, bool payload, cudaStream_t st)
 // then sums the board's exact section in rank order on the host (the same bits everywhere).
 bar_status p2p_exact(bar_dist *ranks, int nr, double *const *xv, cudaStream_t st, double &ss, double &bsq,
                      int64_t &it_min, int64_t &it_max) {
+    NvtxRange nv("peer memory: barrier, ghost pull, exact residual, barrier");
     bar_status r;
     if ((r = board_barrier(ranks, nr, false, st)) != BAR_OK) return r;
     for (int i = 0; i < nr; ++i) {
@@ -585,12 +586,20 @@ void fill_info(bar_solve_info *info, bar_dist *ranks, int nr, int64_t iters, int
 bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, double tol, cudaStream_t st,
                      bar_solve_info *info) {
     bar_status r;
+    NvtxRange nv("dist async over peer memory");
     const int P = ranks[0]->nranks;
     for (int i = 0; i < nr; ++i) {
         k_board_reset<<<1, 32, 0, st>>>(ranks[i]->board, P);
         BAR_CUDA(cudaGetLastError());
     }
     if ((r = board_barrier(ranks, nr, false, st)) != BAR_OK) return r;  // boards reset, x set up
+    for (int i = 0; i < nr; ++i) {  // a rank that never arrives: fail now, not after the iterations
+        if ((r = read_state(ranks[i]->A, st)) != BAR_OK) return r;
+        if (ranks[i]->A->W.h_state->aborted == 2) {
+            set_error("peer-memory barrier timed out (a rank did not join the solve)");
+            return BAR_ERR_NCCL;
+        }
+    }
     unsigned long long tag = ranks[0]->epoch;
     bar_dist D0 = ranks[0];
     DevState &H = *D0->A->W.h_state;
@@ -723,6 +732,12 @@ bar_status overlapped_iteration(bar_dist *ranks, int nr, double *const *vin, dou
     return BAR_OK;
 }
 
+const char *overlap_name(bar_dist D, bar_mode mode) {
+    if (mode == BAR_MODE_ASYNC) return "dist async, collective halo exchange";
+    return D->ib < D->ie && D->A->L.tune.overlap >= 0 ? "dist sync, halo exchange overlapped with interior sweeps"
+                                                       : "dist sync, halo exchange then sweep";
+}
+
 // The solve for the ranks this process drives (1 with NCCL / separate processes, all with
 // loopback). b, x0, x are each rank's owned rows (device or host).
 bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const double *const *x0, double *const *x,
@@ -763,6 +778,7 @@ bar_status dist_solve(bar_dist *ranks, int nr, const double *const *b, const dou
         BAR_CUDA(cudaStreamSynchronize(st));
         return r;
     }
+    NvtxRange nv(overlap_name(D0, mode));
     int64_t launches = nr;
     DevState &H = *D0->A->W.h_state;
     // device time of the local sweeps of this process's first rank (bar_solve_info.sweep_kernel_*)
@@ -1294,6 +1310,7 @@ bar_status bar_create_csr_dist(int64_t n_global, int64_t row_begin, int64_t row_
     std::vector<int32_t> lo, hi;
     ghost_lists(row_begin, row_end, nnz_local, h_col.data(), lo, hi);
     // the communicator, then every rank's (row range, ghost count, device) and ghost list
+    NvtxRange nv("bar_create_csr_dist: NCCL planning, layout, IPC mapping");
     ncclComm_t comm = nullptr;
     {
         ncclUniqueId id;

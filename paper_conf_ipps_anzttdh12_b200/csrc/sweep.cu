@@ -612,10 +612,12 @@ __global__ void __launch_bounds__(1024, 1) k_block_pers(KP p) {
     // claimed in increasing order by whichever block is free — a monotone processing front, which
     // is what lets later blocks see this iteration's values of earlier ones (eq. 4's shift
     // s(k+1, j) < 0: the block Gauss-Seidel flavour of P:209).
-    __shared__ long long s_next;
-    if (threadIdx.x == 0) s_next = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)blockIdx.x;
+    // double-buffered: claim i+1 is written to slot (i+1) & 1 while slow threads may still be
+    // reading claim i from the other slot (compute-sanitizer racecheck, round 2)
+    __shared__ long long s_next[2];
+    if (threadIdx.x == 0) s_next[0] = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)blockIdx.x;
     __syncthreads();
-    int64_t l = s_next;
+    int64_t l = s_next[0];
     if (lane == 0) {
         mbar_init(&bars[0][warp], 1);
         mbar_init(&bars[1][warp], 1);
@@ -634,9 +636,10 @@ __global__ void __launch_bounds__(1024, 1) k_block_pers(KP p) {
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
-        if (threadIdx.x == 0) s_next = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)(l + G);
+        if (threadIdx.x == 0)
+            s_next[(i + 1) & 1] = ASYNC ? (long long)atomicAdd(&p.state->work, 1ull) : (long long)(l + G);
         __syncthreads();
-        ln = s_next;
+        ln = s_next[(i + 1) & 1];
         if (lane == 0 && ln < q && warp < nsl_of(ln)) {  // prefetch the next subdomain's slice
             fence_proxy_async_smem();
             const int64_t sl = ln * p.spb + warp;

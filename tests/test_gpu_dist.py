@@ -359,3 +359,68 @@ def test_interior_boundary_overlap(bar, name, gen, args, R, P, mode, k):
     _, c_on = _loop(blocks, n, R, b, k, mode, 20000, 1e-10, np.zeros(n))
     _, c_off = _loop(blocks, n, R, b, k, mode, 20000, 1e-10, np.zeros(n), tuning={"overlap": -1})
     assert c_on["iters"] == c_off["iters"] and c_on["converged"]
+
+
+def _absent_worker(rank, world, store, q):
+    import os
+    import sys
+    import time
+
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch
+    import torch.distributed as dist
+
+    import workloads as W
+    from paper_conf_ipps_anzttdh12_b200 import dist as D
+
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", init_method=f"file://{store}", rank=rank, world_size=world)
+    try:
+        n = W.stencil7_3d(16).n
+        a, c = D.partition(n, 128, world)[rank]
+        A = W.stencil7_3d(16, row_lo=a, row_hi=c)
+
+        def allgather(o):
+            out = [None] * world
+            dist.all_gather_object(out, o)
+            return out
+
+        Pr = D.PeerRank(A, n, 128, 0, rank, world, allgather)
+        if rank == 0:
+            t0 = time.time()
+            b = torch.ones(c - a, dtype=torch.float64, device="cuda")
+            _, info = Pr.solve(b, mode="async", raise_on_error=False)
+            q.put((rank, info["status"], time.time() - t0))
+            dist.barrier()
+        else:  # rank 1 never joins the solve; it keeps its memory mapped until rank 0 is done
+            q.put((rank, "absent", 0.0))
+            dist.barrier()
+        Pr.close()
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e), 0.0))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_peer_timeout_when_a_rank_is_absent(bar):
+    """A rank that never joins a peer-memory solve makes the others fail with BAR_ERR_NCCL after the
+    board barrier's 20 s timeout — no hang, no device fault (the GPU stays usable)."""
+    import multiprocessing as mp
+    import tempfile
+
+    store = tempfile.mktemp(prefix="bar_absent_store_")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_absent_worker, args=(r, 2, store, q), daemon=True) for r in range(2)]
+    for p in ps:
+        p.start()
+    try:
+        res = {r: (st, dt) for r, st, dt in (q.get(timeout=120) for _ in ps)}
+    finally:
+        for p in ps:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    assert res[1][0] == "absent"
+    assert res[0][0] == "BAR_ERR_NCCL", res
+    assert 15 < res[0][1] < 60, res
