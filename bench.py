@@ -312,6 +312,8 @@ def main():
     ap.add_argument("--halo", default="sendrecv", choices=["sendrecv", "allgather"],
                     help="multi-GPU NCCL halo exchange: grouped send/recv (default) or ncclAllGather")
     ap.add_argument("--tune", default="", help="bar_tuning fields, e.g. 'lead=48,duo=1' (A/B runs)")
+    ap.add_argument("--dist-path", action="store_true",
+                    help="use the multi-GPU code path (bar_create_csr_dist) even with one rank")
     args = ap.parse_args()
     if args.R is None:
         args.R = WORKLOADS[args.workload][2]
@@ -326,7 +328,8 @@ def main():
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     dist = None
-    if world > 1:
+    multi = world > 1 or args.dist_path
+    if multi:
         import torch.distributed as dist
 
         dist.init_process_group("nccl", device_id=dev)
@@ -336,7 +339,7 @@ def main():
     for kv in filter(None, args.tune.split(",")):
         key, val = kv.split("=")
         tune[key] = int(val) if val.lstrip("-").isdigit() else val
-    if world > 1:
+    if multi:
         tune["halo"] = args.halo
         if args.no_p2p:
             tune["peer"] = -1
@@ -359,7 +362,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
     A_host = None
     t0 = time.time()
-    if world == 1:
+    if not multi:
         A = make_matrix(args.workload)
         t_gen = time.time() - t0
         t0 = time.time()
@@ -447,7 +450,7 @@ def main():
                           f"launch (graph-replayed single-launch solves: the kernel's %globaltimer stamps)",
                 "kernel_ms_isolated": round(kernel_ms_isolated, 5),
                 "frac_isolated": round(local_bytes / (kernel_ms_isolated * 1e-3) / 1e9 / peak, 4),
-                "peak_source": peak_src, "per": "GPU" if world > 1 else "job"}
+                "peak_source": peak_src, "per": "GPU" if multi else "job"}
     # the layout's own compulsory bytes (coded columns move 1 B per entry instead of the contract's
     # 4) and, from the committed ncu capture of the same kernel AND the same libbar.so build, the
     # DRAM bytes one launch moved (a capture of another build is stale and not used)
@@ -455,7 +458,7 @@ def main():
     roofline["layout_bytes_per_launch"] = lb
     roofline["frac_layout"] = round(lb / (kernel_ms * 1e-3) / 1e9 / peak, 4)
     prof = os.path.join(ROOT, "profiles", f"traffic_{args.workload}_{args.mode}.json")
-    if world == 1 and os.path.exists(prof):
+    if not multi and os.path.exists(prof):
         try:
             tj = json.load(open(prof))
             if tj.get("kernel") == kernel_name and tj.get("libbar_sha256") == lib_hash() and tj.get("R") == args.R:
@@ -493,7 +496,7 @@ def main():
     # N=1: the partitioned path on this one GPU (bar_create_csr_dist, a 1-rank NCCL group; async
     # runs the peer-memory path with its per-iteration publish / estimate kernel): its time to
     # 1e-10 next to bar_solve's, i.e. what the multi-GPU machinery costs before any exchange
-    if world == 1 and not args.no_dist:
+    if not multi and not args.no_dist:
         try:
             from paper_conf_ipps_anzttdh12_b200 import dist as bdist
 
@@ -524,7 +527,7 @@ def main():
     # small systems: the single-launch kernel's bounded lead (3 sweeps, R12) next to the
     # loosest lead the residual slots allow (48), i.e. "no inter-block synchronisation" as close as
     # the design gets
-    if world == 1 and "resident" in kernel_name and args.mode == "async":
+    if not multi and "resident" in kernel_name and args.mode == "async":
         M.set_tuning(dict(tune, lead=48))
         for _ in range(2):
             step()
@@ -540,7 +543,7 @@ def main():
         M.set_tuning(tune or None)
 
     cpu = None
-    if not args.no_cpu_baseline and rank == 0 and world == 1:
+    if not args.no_cpu_baseline and rank == 0 and not multi:
         cores, model = cpu_info()
         full = args.workload not in PROXY or (args.workload == "c4" and not args.cpu_sample)
         meths = oracle_cpu(args.workload, args.k, args.R, args.mode, A=A_host, full=full)
@@ -559,7 +562,7 @@ def main():
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload][0]}", "n": n, "nnz": nnz,
                    "mode": args.mode, "k": args.k, "rows_per_block": args.R, "tol": args.tol, "b": "ones",
-                   "x0": "zeros", "parallelism": f"rows/{world}" if world == 1 else
+                   "x0": "zeros", "parallelism": f"rows/{world}" if not multi else
                    f"rows/{world} ({'NCCL ' + args.halo if args.mode != 'async' or args.no_p2p else 'peer memory'})",
                    "tuning": tune or "defaults",
                    "l2": "inputs > L2 (no flush needed)" if total_bytes / world > 126e6
