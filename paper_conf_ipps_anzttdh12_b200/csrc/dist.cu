@@ -581,6 +581,73 @@ void fill_info(bar_solve_info *info, bar_dist *ranks, int nr, int64_t iters, int
     info->sweep_kernel_iters = T.iters;
 }
 
+// Lazily created resources of the overlapped iteration (collective or peer-memory path).
+bar_status ensure_overlap(bar_dist D) {
+    if (D->s2) return BAR_OK;
+    BAR_CUDA(cudaStreamCreateWithFlags(&D->s2, cudaStreamNonBlocking));
+    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_fork, cudaEventDisableTiming));
+    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_join, cudaEventDisableTiming));
+    BAR_CUDA(cudaMalloc(&D->state2, sizeof(DevState)));
+    BAR_CUDA(cudaMemset(D->state2, 0, sizeof(DevState)));
+    BAR_CUDA(cudaMalloc(&D->partials2, sizeof(double) * 2 * (size_t)num_blocks_for(D->A->L, BAR_MODE_SYNC_BLOCK)));
+    BAR_CUDA(cudaMalloc(&D->parts3, sizeof(double) * 6));
+    return BAR_OK;
+}
+
+// One global iteration with the interior subdomains swept on the second stream while the halo
+// arrives (every rank of `ranks`): fork -> interior sweeps on s2 || exchange (collective) or
+// ghost pull (peer memory) + low and high boundary sweeps on st -> join -> partial sums.
+// supported = false (nothing enqueued) where the sweep kernel cannot take subdomain ranges.
+bar_status overlapped_iteration(bar_dist *ranks, int nr, double *const *vin, double *const *vout, int32_t k,
+                                bar_mode mode, cudaStream_t st, bool &supported, bool p2p = false) {
+    bar_status r;
+    supported = true;
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        if ((r = ensure_overlap(D)) != BAR_OK) return r;
+        BAR_CUDA(cudaEventRecord(D->ev_fork, st));
+        BAR_CUDA(cudaStreamWaitEvent(D->s2, D->ev_fork, 0));
+        SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->state2, D->partials2, nullptr,
+                    D->parts3 + 2};
+        a.l_begin = D->ib;
+        a.l_end = D->ie;
+        a.stop = &D->A->W.state->stop;
+        const cudaError_t e = launch_sweep(a, mode, D->s2);
+        if (e == cudaErrorNotSupported) {
+            cudaGetLastError();
+            supported = false;
+            return BAR_OK;
+        }
+        BAR_CUDA(e);
+        BAR_CUDA(cudaEventRecord(D->ev_join, D->s2));
+    }
+    if (p2p) {  // peer memory: pull the ghosts as they stand while the interior sweeps run
+        for (int i = 0; i < nr; ++i)
+            if ((r = pull_ghosts(ranks[i], st)) != BAR_OK) return r;
+    } else if ((r = exchange(ranks, nr, vin, st)) != BAR_OK) {
+        return r;
+    }
+    for (int i = 0; i < nr; ++i) {
+        bar_dist D = ranks[i];
+        const int64_t q = D->A->L.q;
+        for (int side = 0; side < 2; ++side) {
+            SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state, D->A->W.partials,
+                        nullptr, D->parts3 + (side ? 4 : 0)};
+            a.l_begin = side ? D->ie : 0;
+            a.l_end = side ? q : D->ib;
+            if (a.l_end <= a.l_begin) {  // empty side: a zero partial
+                BAR_CUDA(cudaMemsetAsync(D->parts3 + (side ? 4 : 0), 0, 2 * sizeof(double), st));
+                continue;
+            }
+            BAR_CUDA(launch_sweep(a, mode, st));
+        }
+        BAR_CUDA(cudaStreamWaitEvent(st, D->ev_join, 0));
+        k_sum_parts<<<1, 1, 0, st>>>(D->parts3, D->A->W.state, D->part);
+        BAR_CUDA(cudaGetLastError());
+    }
+    return BAR_OK;
+}
+
 // async-(k) across ranks over peer memory: per global iteration and rank, pull ghosts, sweep,
 // publish + decide — no collective, no barrier; then the confirming residual (board barriers).
 bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, double tol, cudaStream_t st,
@@ -612,25 +679,43 @@ bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, doub
     bool diverged = false, bzero = false;
     std::vector<double *> xs(nr);
     for (int i = 0; i < nr; ++i) xs[i] = ranks[i]->xa;
+    bool overlap = D0->A->L.tune.overlap >= 0 && P > 1;
+    for (int i = 0; i < nr; ++i) overlap = overlap && ranks[i]->ib < ranks[i]->ie;
     for (;;) {
         bool stopped = false;
         while (issued < max_iters && !stopped) {
             const int64_t c = std::min(chunk, max_iters - issued);
             for (int64_t it = 0; it < c; ++it) {
+                bool done = false;
+                if (overlap) {  // interior sweeps on the second stream while the ghosts are pulled
+                    if ((r = timer_begin(T, issued + it + 1, st)) != BAR_OK) return r;
+                    bool supported = true;
+                    if ((r = overlapped_iteration(ranks, nr, xs.data(), xs.data(), k, BAR_MODE_ASYNC, st, supported,
+                                                  true)) != BAR_OK)
+                        return r;
+                    if ((r = timer_end(T, st)) != BAR_OK) return r;
+                    done = supported;
+                    if (!supported) {
+                        overlap = false;
+                        T.used = T.used > 0 ? T.used - 1 : 0;
+                    }
+                }
                 for (int i = 0; i < nr; ++i) {
                     bar_dist D = ranks[i];
-                    if ((r = pull_ghosts(D, st)) != BAR_OK) return r;
-                    SweepArgs a{&D->A->L, D->bbuf, own(D, D->xa), own(D, D->xa), k, D->A->W.state, D->A->W.partials,
-                                nullptr, D->part};
-                    if (i == 0 && (r = timer_begin(T, issued + it + 1, st)) != BAR_OK) return r;
-                    BAR_CUDA(launch_sweep(a, BAR_MODE_ASYNC, st));
-                    if (i == 0 && (r = timer_end(T, st)) != BAR_OK) return r;
+                    if (!done) {
+                        if ((r = pull_ghosts(D, st)) != BAR_OK) return r;
+                        SweepArgs a{&D->A->L, D->bbuf, own(D, D->xa), own(D, D->xa), k, D->A->W.state,
+                                    D->A->W.partials, nullptr, D->part};
+                        if (i == 0 && (r = timer_begin(T, issued + it + 1, st)) != BAR_OK) return r;
+                        BAR_CUDA(launch_sweep(a, BAR_MODE_ASYNC, st));
+                        if (i == 0 && (r = timer_end(T, st)) != BAR_OK) return r;
+                    }
                     k_p2p_publish_decide<<<1, 1, 0, st>>>(D->A->W.state, D->part, D->d_peer_board, D->board, D->rank,
                                                           P, tag);
                     BAR_CUDA(cudaGetLastError());
                 }
+                launches += (done ? 6 : 3) * nr;  // overlapped: pull, three sweeps, sum, publish
             }
-            launches += 3 * nr * c;
             issued += c;
             for (int i = nr - 1; i >= 0; --i) {  // loopback: the last rank's request reaches the others next time
                 if ((r = read_state(ranks[i]->A, st)) != BAR_OK) return r;
@@ -666,68 +751,6 @@ bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, doub
     if (diverged) {
         set_error("relative residual became non-finite or exceeded 1e30");
         return BAR_ERR_DIVERGED;
-    }
-    return BAR_OK;
-}
-
-// Lazily created resources of the overlapped collective iteration.
-bar_status ensure_overlap(bar_dist D) {
-    if (D->s2) return BAR_OK;
-    BAR_CUDA(cudaStreamCreateWithFlags(&D->s2, cudaStreamNonBlocking));
-    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_fork, cudaEventDisableTiming));
-    BAR_CUDA(cudaEventCreateWithFlags(&D->ev_join, cudaEventDisableTiming));
-    BAR_CUDA(cudaMalloc(&D->state2, sizeof(DevState)));
-    BAR_CUDA(cudaMemset(D->state2, 0, sizeof(DevState)));
-    BAR_CUDA(cudaMalloc(&D->partials2, sizeof(double) * 2 * (size_t)num_blocks_for(D->A->L, BAR_MODE_SYNC_BLOCK)));
-    BAR_CUDA(cudaMalloc(&D->parts3, sizeof(double) * 6));
-    return BAR_OK;
-}
-
-// One global iteration of the collective path with the interior subdomains swept on the second
-// stream while the exchange runs (every rank of `ranks`): fork -> interior sweeps on s2 ||
-// exchange + low and high boundary sweeps on st -> join -> partial sums. Returns
-// cudaErrorNotSupported (nothing enqueued) where the sweep kernel cannot take subdomain ranges.
-bar_status overlapped_iteration(bar_dist *ranks, int nr, double *const *vin, double *const *vout, int32_t k,
-                                bar_mode mode, cudaStream_t st, bool &supported) {
-    bar_status r;
-    supported = true;
-    for (int i = 0; i < nr; ++i) {
-        bar_dist D = ranks[i];
-        if ((r = ensure_overlap(D)) != BAR_OK) return r;
-        BAR_CUDA(cudaEventRecord(D->ev_fork, st));
-        BAR_CUDA(cudaStreamWaitEvent(D->s2, D->ev_fork, 0));
-        SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->state2, D->partials2, nullptr,
-                    D->parts3 + 2};
-        a.l_begin = D->ib;
-        a.l_end = D->ie;
-        a.stop = &D->A->W.state->stop;
-        const cudaError_t e = launch_sweep(a, mode, D->s2);
-        if (e == cudaErrorNotSupported) {
-            cudaGetLastError();
-            supported = false;
-            return BAR_OK;
-        }
-        BAR_CUDA(e);
-        BAR_CUDA(cudaEventRecord(D->ev_join, D->s2));
-    }
-    if ((r = exchange(ranks, nr, vin, st)) != BAR_OK) return r;
-    for (int i = 0; i < nr; ++i) {
-        bar_dist D = ranks[i];
-        const int64_t q = D->A->L.q;
-        for (int side = 0; side < 2; ++side) {
-            SweepArgs a{&D->A->L, D->bbuf, own(D, vin[i]), own(D, vout[i]), k, D->A->W.state, D->A->W.partials,
-                        nullptr, D->parts3 + (side ? 4 : 0)};
-            a.l_begin = side ? D->ie : 0;
-            a.l_end = side ? q : D->ib;
-            if (a.l_end <= a.l_begin) {  // empty side: a zero partial
-                BAR_CUDA(cudaMemsetAsync(D->parts3 + (side ? 4 : 0), 0, 2 * sizeof(double), st));
-                continue;
-            }
-            BAR_CUDA(launch_sweep(a, mode, st));
-        }
-        BAR_CUDA(cudaStreamWaitEvent(st, D->ev_join, 0));
-        k_sum_parts<<<1, 1, 0, st>>>(D->parts3, D->A->W.state, D->part);
-        BAR_CUDA(cudaGetLastError());
     }
     return BAR_OK;
 }
