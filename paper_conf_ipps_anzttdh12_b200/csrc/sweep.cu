@@ -61,6 +61,7 @@ struct KP {
     int fronts;             // > 0: F fronts (claims_of), async_order = 3
     int64_t l_begin, l_end; // subdomains this launch sweeps (l_end = 0: all; k_block_duo / _pipe only)
     const int *stop;        // the stop flag the kernels poll at start (default &state->stop)
+    int slab_ahead;         // k_block_duo: L2 bulk prefetch of the slab two subdomains ahead
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
@@ -1127,6 +1128,15 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             const uint32_t nsl = (uint32_t)nsl_of(l);
             bulk_g2s(smraw + g.o_sptr, p.sptr + l * spb, (nsl * 8 + 15) & ~15u, &bar);
             bulk_g2s(smraw + g.o_sw, p.sw + l * spb, (nsl * 4 + 15) & ~15u, &bar);
+            // the slab after this one into L2 already: a second slab buffer, in L2 instead of
+            // shared memory, so HBM keeps streaming while both blocks of the SM sweep locally
+            if (p.slab_ahead && lof(j + 1) < C.lend) {
+                const int64_t *bn = bnd[(j + 1) & 3];
+                const uint32_t nn = (uint32_t)(bn[1] - bn[0]);
+                bulk_prefetch_l2(p.val + bn[0], nn * 8);
+                if (CODED) bulk_prefetch_l2(p.codes + bn[0], (nn + 15) & ~15u);
+                else bulk_prefetch_l2(p.col + bn[0], nn * 4);
+            }
         }
     };
     // warp 3 lane 0: bounds and ghost ranges of l_j into ring slot j % 4 (one cp.async group)
@@ -2047,6 +2057,7 @@ KP make_kp(const Layout &L) {
     const int gp = L.tune.ghost_prefetch;
     p.gr = (gp ? gp > 0 : L.R >= 512) ? L.gr : nullptr;
     p.grid_cap = L.tune.grid_cap > 0 ? L.tune.grid_cap : 0;
+    p.slab_ahead = L.tune.slab_prefetch > 0 ? 1 : 0;
     return p;
 }
 

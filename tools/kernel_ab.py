@@ -43,6 +43,7 @@ def main():
     ap.add_argument("--k", type=int, default=5)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--variants", default="base:")
+    ap.add_argument("--rounds", type=int, default=1, help="repeat the variant list (A B A B ...); medians at the end")
     a = ap.parse_args()
     import torch
 
@@ -77,8 +78,9 @@ def main():
     del src, dst
     clk = os.popen("nvidia-smi --query-gpu=clocks.sm,clocks.mem,power.draw --format=csv,noheader").read().strip()
     print(json.dumps({"box": {"copy_GBs": round(copy_gbs, 1), "clocks": clk}}), flush=True)
-    for mode in a.modes.split(","):
-        for name, tune in parse_variants(a.variants):
+    summary = {}
+    for mode, rnd, (name, tune) in [(m, r, v) for m in a.modes.split(",") for r in range(a.rounds)
+                                     for v in parse_variants(a.variants)]:
             M.set_tuning(tune or None)
             M.sweep(b, x, k=a.k, nsweeps=4, mode=mode)
             lo, hi = 8, 40
@@ -89,12 +91,18 @@ def main():
             solves = [ev_time(lambda: M.solve(b, None, x, k=a.k, mode=mode)) for _ in range(a.reps)]
             ms = statistics.median(s[0] for s in solves)
             iters = [s[1][1]["iters"] for s in solves]
+            summary.setdefault((mode, name), []).append((per_launch, ms))
             print(json.dumps({"workload": a.workload, "R": R, "k": a.k, "mode": mode, "variant": name, "tuning": tune,
                               "launch_ms": round(per_launch, 4),
                               "contract_GBs": round(info["model_bytes_per_iter"] / per_launch / 1e6, 1),
                               "frac_of_copy": round(info["model_bytes_per_iter"] / per_launch / 1e6 / copy_gbs, 3),
                               "kernel": M.info()["last_sweep_kernel"],
                               "solve_ms": round(ms, 3), "iters": iters}), flush=True)
+    if a.rounds > 1:
+        for (mode, name), v in summary.items():
+            print(json.dumps({"median_over_rounds": True, "mode": mode, "variant": name,
+                              "launch_ms": round(statistics.median(t for t, _ in v), 4),
+                              "solve_ms": round(statistics.median(s_ for _, s_ in v), 3), "rounds": len(v)}), flush=True)
     M.close()
 
 
