@@ -38,8 +38,9 @@
 //   [0, 2P)    part:    latest [sum r^2, sum b^2] estimate partial of each rank (async iteration)
 //   [2P, 3P)   stopreq: u64 tag of the latest stop request of each rank (>= the phase tag: stop)
 //   [3P, 4P)   arrive:  u64 latest board-barrier epoch each rank has reached
-//   [4P, 7P)   exact:   [sum r^2, sum b^2, global iterations] of each rank, published with an arrival
-constexpr int kBoardWordsPerRank = 7;
+//   [4P, 8P)   exact:   [sum r^2, sum b^2, global iterations, launches issued] of each rank, published
+//                       with an arrival
+constexpr int kBoardWordsPerRank = 8;
 
 struct bar_dist_s {
     bar_matrix A = nullptr;  // local layout: n_local rows, columns [-n_glo, n_local + n_ghi)
@@ -214,15 +215,16 @@ __global__ void k_p2p_publish_decide(DevState *S, const double *__restrict__ par
 // wait: ACQUIRE every rank's arrival in this rank's board until all reached `epoch`. A wait longer
 // than the timeout sets S->aborted = 2 (a peer is gone) instead of hanging the device.
 __global__ void k_board_barrier(DevState *S, const double *board, double *const *peer_board, int rank, int P,
-                                unsigned long long epoch, const double *payload, int publish, int wait) {
+                                unsigned long long epoch, const double *payload, double issued, int publish, int wait) {
     if (publish) {
         if (payload) {
             const double a = payload[0], b = payload[1], it = (double)S->iter;
             for (int p = 0; p < P; ++p) {
-                double *ex = peer_board[p] + 4 * P + 3 * rank;
+                double *ex = peer_board[p] + 4 * P + 4 * rank;
                 st_relaxed_sys(ex, a);
                 st_relaxed_sys(ex + 1, b);
                 st_relaxed_sys(ex + 2, it);
+                st_relaxed_sys(ex + 3, issued);
             }
         }
         for (int p = 0; p < P; ++p) st_release_sys_u64(peer_board[p] + 3 * P + rank, epoch);
@@ -506,22 +508,22 @@ bar_status pull_ghosts(bar_dist D, cudaStream_t st) {
 }
 
 // Every rank of `ranks` passes the next board-barrier epoch (optionally publishing its payload
-// [sum r^2, sum b^2] from D->part). Separate processes: one publish+wait launch per rank; the
-// loopback group (one stream): all publishes, then all waits.
-bar_status board_barrier(bar_dist *ranks, int nr, bool payload, cudaStream_t st) {
+// [sum r^2, sum b^2] from D->part, its iterations and `issued` launches). Separate processes: one
+// publish+wait launch per rank; the loopback group (one stream): all publishes, then all waits.
+bar_status board_barrier(bar_dist *ranks, int nr, bool payload, cudaStream_t st, int64_t issued = 0) {
     const bool split = ranks[0]->loopback;
     for (int i = 0; i < nr; ++i) {
         bar_dist D = ranks[i];
         ++D->epoch;
         k_board_barrier<<<1, 1, 0, st>>>(D->A->W.state, D->board, D->d_peer_board, D->rank, D->nranks, D->epoch,
-                                          payload ? D->part : nullptr, 1, split ? 0 : 1);
+                                          payload ? D->part : nullptr, (double)issued, 1, split ? 0 : 1);
         BAR_CUDA(cudaGetLastError());
     }
     if (split)
         for (int i = 0; i < nr; ++i) {
             bar_dist D = ranks[i];
             k_board_barrier<<<1, 1, 0, st>>>(D->A->W.state, D->board, D->d_peer_board, D->rank, D->nranks, D->epoch,
-                                              nullptr, 0, 1);
+                                              nullptr, 0.0, 0, 1);
             BAR_CUDA(cudaGetLastError());
         }
     return BAR_OK;
@@ -531,7 +533,7 @@ bar_status board_barrier(bar_dist *ranks, int nr, bool payload, cudaStream_t st)
 // now-frozen ghosts, exact residual partials, publish them with the next barrier; every rank
 // then sums the board's exact section in rank order on the host (the same bits everywhere).
 bar_status p2p_exact(bar_dist *ranks, int nr, double *const *xv, cudaStream_t st, double &ss, double &bsq,
-                     int64_t &it_min, int64_t &it_max) {
+                     int64_t &it_min, int64_t &it_max, int64_t issued, int64_t &issued_min) {
     NvtxRange nv("peer memory: barrier, ghost pull, exact residual, barrier");
     bar_status r;
     if ((r = board_barrier(ranks, nr, false, st)) != BAR_OK) return r;
@@ -540,10 +542,10 @@ bar_status p2p_exact(bar_dist *ranks, int nr, double *const *xv, cudaStream_t st
         if ((r = pull_ghosts(D, st)) != BAR_OK) return r;
         BAR_CUDA(launch_residual(D->A->L, D->bbuf, own(D, xv[i]), D->A->W.state, D->A->W.partials, st, D->part));
     }
-    if ((r = board_barrier(ranks, nr, true, st)) != BAR_OK) return r;
+    if ((r = board_barrier(ranks, nr, true, st, issued)) != BAR_OK) return r;
     bar_dist D0 = ranks[0];
     const int P = D0->nranks;
-    BAR_CUDA(cudaMemcpyAsync(D0->h_exact, D0->board + 4 * P, sizeof(double) * 3 * (size_t)P, cudaMemcpyDeviceToHost,
+    BAR_CUDA(cudaMemcpyAsync(D0->h_exact, D0->board + 4 * P, sizeof(double) * 4 * (size_t)P, cudaMemcpyDeviceToHost,
                              st));
     for (int i = 0; i < nr; ++i)
         if ((r = read_state(ranks[i]->A, st)) != BAR_OK) return r;
@@ -553,14 +555,15 @@ bar_status p2p_exact(bar_dist *ranks, int nr, double *const *xv, cudaStream_t st
             return BAR_ERR_NCCL;
         }
     ss = bsq = 0.0;
-    it_min = INT64_MAX;
+    it_min = issued_min = INT64_MAX;
     it_max = 0;
     for (int p = 0; p < P; ++p) {
-        ss += D0->h_exact[3 * p];
-        bsq += D0->h_exact[3 * p + 1];
-        const int64_t it = (int64_t)D0->h_exact[3 * p + 2];
+        ss += D0->h_exact[4 * p];
+        bsq += D0->h_exact[4 * p + 1];
+        const int64_t it = (int64_t)D0->h_exact[4 * p + 2];
         it_min = std::min(it_min, it);
         it_max = std::max(it_max, it);
+        issued_min = std::min(issued_min, (int64_t)D0->h_exact[4 * p + 3]);
     }
     return BAR_OK;
 }
@@ -725,8 +728,8 @@ bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, doub
             chunk = sizer.next(chunk, (long long)H.iter, H.last_rel, tol);
         }
         double ss = 0.0, bsq = 0.0;
-        int64_t it_min = 0;
-        if ((r = p2p_exact(ranks, nr, xs.data(), st, ss, bsq, it_min, it_max)) != BAR_OK) return r;
+        int64_t it_min = 0, issued_min = 0;
+        if ((r = p2p_exact(ranks, nr, xs.data(), st, ss, bsq, it_min, it_max, issued, issued_min)) != BAR_OK) return r;
         launches += 4 * nr;
         iters = it_min;
         const double bn = std::sqrt(bsq);
@@ -734,10 +737,14 @@ bar_status p2p_solve(bar_dist *ranks, int nr, int32_t k, int64_t max_iters, doub
         if (bn == 0.0) bzero = true;
         else if (!std::isfinite(rel) || rel > 1e30) diverged = true;
         else converged = rel <= tol;
-        if (converged || diverged || bzero || !stopped || issued >= max_iters) break;
-        // the estimate met tol but the exact residual did not: every rank resumes (same bits)
+        // decided from the board's exact section only (the same bits on every rank; a rank's own
+        // `stopped` / `issued` may differ from its peers'): done, or every rank has issued all
+        // max_iters global iterations
+        if (converged || diverged || bzero || issued_min >= max_iters) break;
+        // an estimate met tol but the exact residual did not: every rank resumes
         for (int i = 0; i < nr; ++i) BAR_CUDA(cudaMemsetAsync(&ranks[i]->A->W.state->stop, 0, sizeof(int), st));
         tag = ranks[0]->epoch;  // older stop requests are stale now
+        (void)stopped;
     }
     if (bzero) {
         for (int i = 0; i < nr; ++i)
@@ -933,8 +940,8 @@ bar_status dist_residual(bar_dist D, const double *b, const double *x, cudaStrea
             return BAR_ERR_INVALID_ARG;
         }
         double *xs[1] = {D->xa};
-        int64_t a = 0, c = 0;
-        if ((r = p2p_exact(&D, 1, xs, st, ss, bsq, a, c)) != BAR_OK) return r;
+        int64_t a = 0, c = 0, e = 0;
+        if ((r = p2p_exact(&D, 1, xs, st, ss, bsq, a, c, 0, e)) != BAR_OK) return r;
     } else {
         double *xs[1] = {D->xa};
         if ((r = exchange(&D, 1, xs, st)) != BAR_OK) return r;
@@ -1071,7 +1078,7 @@ bar_status create_share(int64_t n_global, int64_t row_begin, int64_t row_end, in
     if (st == BAR_OK && cudaMemset(D->board, 0, sizeof(double) * kBoardWordsPerRank * (size_t)nranks) != cudaSuccess)
         st = cuda_fail(cudaGetLastError(), "cudaMemset");
     if (st == BAR_OK &&
-        cudaMallocHost((void **)&D->h_exact, sizeof(double) * 3 * (size_t)nranks) != cudaSuccess)
+        cudaMallocHost((void **)&D->h_exact, sizeof(double) * 4 * (size_t)nranks) != cudaSuccess)
         st = cuda_fail(cudaGetLastError(), "cudaMallocHost");
     if (st != BAR_OK) {
         bar_dist_destroy(D);
