@@ -230,6 +230,9 @@ typedef struct {
                                1 one ncclAllGather per iteration                                 */
     int32_t peer;           /* multi-GPU async: 0 peer memory when mapped, -1 the collective path */
     int32_t fronts;         /* async_order = 3: number of fronts (0 = 8)                          */
+    int32_t lazy_publish;   /* k_block_resident: 0 non-blocking residual publication (a ring of
+                               per-block partials, evaluated by block m % q), -1 one blocking
+                               atomic per block and iteration                                    */
     int32_t slab_prefetch;  /* k_block_duo: 1 L2 bulk prefetch of the slab two subdomains ahead
                                (a second slab buffer in L2), 0 off                               */
     int32_t overlap;        /* multi-GPU collective path: 0 sweep the interior subdomains (no ghost

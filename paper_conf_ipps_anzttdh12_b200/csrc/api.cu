@@ -46,6 +46,10 @@ bar_status ensure_workspace(bar_matrix A) {
         BAR_CUDA(cudaMallocHost(&W.h_state, sizeof(DevState)));
         BAR_CUDA(cudaMemset(W.state, 0, sizeof(DevState)));
     }
+    if (!W.ring && L.q <= 8192 && use_async_multi(L)) {  // the single-launch kernel's residual ring
+        BAR_CUDA(cudaMalloc(&W.ring, sizeof(double) * kSlots * (size_t)L.q));
+        BAR_CUDA(cudaMalloc(&W.bsum_arr, sizeof(double) * (size_t)L.q));
+    }
     int64_t need = std::max(num_blocks_for(L, BAR_MODE_SYNC_BLOCK), num_blocks_for(L, BAR_MODE_JACOBI));
     if (W.npartials < need) {
         cudaFree(W.partials);
@@ -221,6 +225,8 @@ void bar_destroy(bar_matrix A) {
     cudaFree(W.stage_x);
     cudaFree(W.partials);
     cudaFree(W.frozen);
+    cudaFree(W.ring);
+    cudaFree(W.bsum_arr);
     cudaFree(W.state);
     cudaFreeHost(W.h_state);
     delete A;
@@ -326,6 +332,8 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
     BAR_CUDA(launch_init_state(A->W.state, -1.0, st));
     if (mode == BAR_MODE_ASYNC && nsweeps > 0) {  // the fully asynchronous kernel when it applies
         SweepArgs a{&A->L, b, x, x, k, A->W.state, A->W.partials, nullptr};
+        a.ring = A->W.ring;
+        a.bsum_arr = A->W.bsum_arr;
         if (use_async_multi(A->L)) {
             cudaError_t e = launch_async_multi(a, (long long)nsweeps * A->L.q, st);
             if (e == cudaSuccess) return BAR_OK;
@@ -563,6 +571,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 if (e != cudaSuccess) return e;
                 if ((e = cudaEventRecord(ev0, s)) != cudaSuccess) return e;
                 SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
+                a.ring = W.ring;
+                a.bsum_arr = W.bsum_arr;
                 if ((e = launch_async_multi(a, w_end, s)) != cudaSuccess) return e;
                 if ((e = cudaEventRecord(ev1, s)) != cudaSuccess) return e;
                 if ((e = launch_residual(L, db, buf0, W.state, W.partials, s)) != cudaSuccess) return e;
@@ -618,6 +628,8 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                     while (resume && !converged && !diverged) {  // rare: estimate met tol, exact did not
                         SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
                         a.m0 = m0;
+                        a.ring = W.ring;
+                        a.bsum_arr = W.bsum_arr;
                         if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;
                         BAR_CUDA(launch_async_multi(a, w_end, st));
                         if ((r = timer_end(T, st)) != BAR_OK) return r;
@@ -643,6 +655,10 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             // x has that many complete global iterations plus the sweeps still in flight when
             // the queue closed, counted in cta_iters_max)
             iters = (converged && H.stop_iter > 0) ? H.stop_iter : H.iters_done;
+            // a resident launch that ran to max_global_iters without a stop: every block swept the
+            // same number of times (its last iterations may not have been evaluated yet with the
+            // lazy residual publication)
+            if (!H.stop && static_multi(L.last_kernel)) iters = std::max<int64_t>(iters, (int64_t)(H.res_sweeps / L.q));
             const unsigned long long claimed = static_multi(L.last_kernel) ? H.res_sweeps
                                                                            : (H.stop ? H.work_resume : H.work);
             cta_max = (int64_t)((claimed + L.q - 1) / L.q);

@@ -171,6 +171,8 @@ struct Workspace {
     double *stage_x = nullptr;  // n: device staging of host x0/x
     double *partials = nullptr; // per-block partial sums of squares
     uint8_t *frozen = nullptr;  // N1 failure mask (device copy, n bytes)
+    double *ring = nullptr;     // [kSlots][q] residual partials of k_block_resident's lazy publication
+    double *bsum_arr = nullptr; // [q]
     int64_t npartials = 0;
     DevState *state = nullptr;  // device
     DevState *h_state = nullptr;// pinned host mirror
@@ -257,6 +259,8 @@ struct SweepArgs {
     int64_t l_begin = 0, l_end = 0;   // sweep only subdomains [l_begin, l_end) (l_end = 0: all);
                                       // cudaErrorNotSupported where the chosen kernel cannot
     const int *stop = nullptr;        // stop flag polled by the kernels (nullptr: state->stop)
+    double *ring = nullptr;           // single-launch resident kernel, lazy publication:
+    double *bsum_arr = nullptr;       //   Workspace::ring / bsum_arr (nullptr: the blocking path)
 };
 int64_t num_blocks_for(const Layout &L, bar_mode mode);
 int64_t rowwise_grid(const Layout &L);

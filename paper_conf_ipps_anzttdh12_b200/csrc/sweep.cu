@@ -62,6 +62,8 @@ struct KP {
     int64_t l_begin, l_end; // subdomains this launch sweeps (l_end = 0: all; k_block_duo / _pipe only)
     const int *stop;        // the stop flag the kernels poll at start (default &state->stop)
     int slab_ahead;         // k_block_duo: L2 bulk prefetch of the slab two subdomains ahead
+    double *ring;           // k_block_resident<LAZY>: [kSlots][q] per-block residual partials
+    double *bsum_arr;       //   and [q] per-block sums of b_i^2
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
     const int32_t *dict;    //   dictionary dict[dptr[l] ..) of column offsets d = col - row
     const int32_t *dptr;
@@ -1745,6 +1747,65 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     if (!MULTI) reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+// k_block_resident<.., LAZY>: warp 0 of block m % q evaluates iteration m once all q partials are
+// in ring[m % kSlots] (thread 0 polls with relaxed loads, then an acquire fence before the CTA
+// barrier that hands the evaluation to the warp): fixed-order sums over the blocks (lane-strided,
+// then the shuffle tree), the stopping rule of iteration_publish, iters_done, and the slot's
+// counter reset for iteration m + kSlots.
+__device__ __noinline__ void lazy_evaluate(const KP &p, long long m, int64_t q, int lane) {
+    DevState *S = p.state;
+    const int slot = (int)(m % kSlots);
+    const double *row = p.ring + (int64_t)slot * q;
+    double ss = 0.0, bsq = 0.0;
+    for (int64_t c = lane; c < q; c += kSlice) {
+        ss += __ldcg(row + c);
+        bsq += __ldcg(p.bsum_arr + c);
+    }
+    ss = warp_sum(ss);
+    bsq = warp_sum(bsq);
+    if (lane != 0) return;
+    S->done[slot] = 0u;
+    const double bn = sqrt(bsq);
+    const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+    atomicMax(&S->iters_done, m + 1);
+    S->bnorm = bn;
+    S->last_rel = rel;
+    if (p.hist) p.hist[m] = rel;
+    bool stop = false;
+    if (bn == 0.0) {
+        S->diverged = 2;
+        stop = true;
+    } else if (!isfinite(rel) || rel > 1e30) {
+        S->diverged = 1;
+        stop = true;
+    } else if (rel <= S->tol) {
+        // evaluations may complete out of order: the first iteration that met tol wins
+        atomicMin(reinterpret_cast<unsigned long long *>(&S->stop_iter), (unsigned long long)(m + 1));
+        stop = true;
+    }
+    if (stop) atomicExch(&S->stop, 1);
+}
+
+// Phase timing of k_block_resident's thread 0 (a profiling build only: -DBAR_PROFILE_RESIDENT):
+// clock64 deltas between the marks, summed over the launch, added per block into g_res_prof.
+#ifdef BAR_PROFILE_RESIDENT
+__device__ unsigned long long g_res_prof[8];
+#define BAR_PROF_DECL long long prof_t[6] = {0, 0, 0, 0, 0, 0}, prof_last = clock64();
+#define BAR_PROF_MARK(i)                            \
+    if (threadIdx.x == 0) {                         \
+        const long long now = clock64();            \
+        prof_t[i] += now - prof_last;               \
+        prof_last = now;                            \
+    }
+#define BAR_PROF_FLUSH                                                                  \
+    if (threadIdx.x == 0)                                                               \
+        for (int i = 0; i < 6; ++i) atomicAdd(&g_res_prof[i], (unsigned long long)prof_t[i]);
+#else
+#define BAR_PROF_DECL
+#define BAR_PROF_MARK(i)
+#define BAR_PROF_FLUSH
+#endif
+
 // k_block_resident: the fully asynchronous solve for systems whose subdomains all fit on the
 // device at once (q <= co-resident blocks; C1-C3). Block c OWNS subdomain c for the whole launch,
 // the paper's picture taken literally: one thread block per subdomain, iterating with no
@@ -1761,11 +1822,12 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // resident at once; if they are not (other work on the device holds SMs), a waiting block
 // times out after ~2 ms, raises state->aborted and the stop flag, every block exits, and the
 // host continues the solve from the current iterate with per-launch kernels (R12).
-template <int WLR>
+template <int WLR, bool LAZY = false>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_resident(KP p) {
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ double sred[2][32];
     __shared__ int go;
+    __shared__ long long eval_m;  // LAZY: iteration warp 0 evaluates in this pass (-1: none)
     if (threadIdx.x == 0) stamp_first(p.state);
     const int R = p.R, spb = p.spb;
     const int64_t q = (p.n + R - 1) / R;
@@ -1823,36 +1885,77 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         bsum = 0.0;
         for (int w = 0; w < W; ++w) bsum += sred[1][w];
     }
+    // LAZY publication: block c stores its partial of iteration m into ring[m % kSlots][c] and
+    // bumps done[m % kSlots] with a release reduction (no returned value, nothing to wait for);
+    // iteration m is evaluated by block m % q once it sees all q contributions (a relaxed load
+    // issued one iteration ahead; acquire fence when complete): fixed-order sum of the ring row
+    // and of the blocks' sum b_i^2, then the stopping rule as in iteration_publish (lazy_evaluate)
+    long long next_eval = p.m0 + (((long long)blockIdx.x - p.m0) % q + q) % q;  // first m >= m0 with m % q == c
+    unsigned int dv_ld = 0;
+    if (LAZY && threadIdx.x == 0)
+        asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.bsum_arr + blockIdx.x), "d"(bsum) : "memory");
     int cur = 0;
     // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
     // it before the launch: x^(0) already meets tol)
     int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
     long long done_ld = p.m0;  // thread 0: iters_done, loaded one iteration ahead of its use
     unsigned long long sweeps = 0;
-    for (long long m = p.m0;; ++m) {
+    BAR_PROF_DECL
+    for (long long m = p.m0;;) {
+        BAR_PROF_MARK(0)
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
+            // LAZY: this block's pending evaluation, if all q partials of that iteration are in
+            // (dv_ld: loaded one iteration ahead); evaluated by warp 0 after the barrier below
+            if (LAZY) {
+                eval_m = -1;
+                if (next_eval < m && dv_ld == (unsigned int)q) {
+                    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+                    eval_m = next_eval;
+                    next_eval += q;
+                    dv_ld = 0;
+                }
+            }
             // bounded lead over the last completed iteration (p.lead sweeps; residual slots are
             // reused mod 64). The lead is checked against iters_done as loaded one iteration ago
             // and only re-read (waited on) when exceeded. The wait is itself bounded (~2 ms of
             // %globaltimer): a lagging block that long behind is not resident, so the launch gives
-            // up (aborted + stop) instead of waiting on work that cannot run
+            // up (aborted + stop) instead of waiting on work that cannot run. LAZY: the iteration
+            // the others wait for may be the one this block evaluates — then stop waiting, let
+            // warp 0 evaluate it, and come back (go = 2) before sweeping
             if (g && m - done_ld > p.lead) {
-                const unsigned long long t0c = globaltimer_ns();
-                while (g && m - *(volatile long long *)&p.state->iters_done > p.lead) {
-                    if (*(volatile int *)&p.state->stop) g = 0;
-                    else if (globaltimer_ns() - t0c > 2000000ull) {
-                        atomicExch(&p.state->aborted, 1);
-                        atomicExch(&p.state->stop, 1);
-                        g = 0;
+                if (LAZY && eval_m >= 0) {
+                    g = 2;
+                } else {
+                    const unsigned long long t0c = globaltimer_ns();
+                    while (g && m - *(volatile long long *)&p.state->iters_done > p.lead) {
+                        if (*(volatile int *)&p.state->stop) g = 0;
+                        else if (globaltimer_ns() - t0c > 2000000ull) {
+                            atomicExch(&p.state->aborted, 1);
+                            atomicExch(&p.state->stop, 1);
+                            g = 0;
+                        } else if (LAZY && next_eval < m &&
+                                   *(volatile unsigned int *)&p.state->done[next_eval % kSlots] == (unsigned int)q) {
+                            asm volatile("fence.acq_rel.gpu;" ::: "memory");
+                            eval_m = next_eval;
+                            next_eval += q;
+                            g = 2;
+                            break;
+                        }
                     }
                 }
             }
             go = g;
         }
         __syncthreads();
+        if (LAZY && warp == 0 && eval_m >= 0) lazy_evaluate(p, eval_m, q, lane);
         if (!go) break;
+        if (LAZY && go == 2) {  // evaluated for the waiting blocks; re-check the lead
+            __syncthreads();
+            continue;
+        }
+        BAR_PROF_MARK(1)
         ++sweeps;
         if (threadIdx.x == 0) {  // issued now, consumed at the next iteration's start
             asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(stop_ld) : "l"(&p.state->stop));
@@ -1880,6 +1983,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             y1[loc] = y0[loc] + dinv * acc;
         }
         __syncthreads();
+        BAR_PROF_MARK(2)
         for (int t = 1; t < p.k; ++t) {  // a4: sweeps 2..k, direct form, off-block part frozen
             const double *yi = ybuf(cur ^ (t & 1));
             double *yo = ybuf(cur ^ ((t + 1) & 1));
@@ -1891,23 +1995,40 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             }
             __syncthreads();
         }
+        BAR_PROF_MARK(3)
         cur ^= p.k & 1;
         if (ok) stx<true>(p.x_out + TS + loc, ybuf(cur)[loc]);  // a6
         const double wr = warp_sum(rr);
         if (lane == 0) sred[0][warp] = wr;
         __syncthreads();
+        BAR_PROF_MARK(4)
         if (threadIdx.x == 0) {
             const int W = blockDim.x >> 5;
             double a0 = 0.0;
             for (int w = 0; w < W; ++w) a0 += sred[0][w];
-            iteration_publish(p, m, 1u, a0, bsum, q);
+            if (LAZY) {
+                const int slot = (int)(m % kSlots);
+                asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.ring + (int64_t)slot * q + blockIdx.x),
+                             "d"(a0)
+                             : "memory");
+                asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&p.state->done[slot]) : "memory");
+                if (next_eval <= m)  // consumed at the next iteration's start
+                    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];"
+                                 : "=r"(dv_ld)
+                                 : "l"(&p.state->done[next_eval % kSlots]));
+            } else {
+                iteration_publish(p, m, 1u, a0, bsum, q);
+            }
             stop_seen = stop_ld;
         }
+        BAR_PROF_MARK(5)
+        ++m;
     }
     if (threadIdx.x == 0) {
         atomicAdd(&p.state->res_sweeps, sweeps);
         stamp_last(p.state);
     }
+    BAR_PROF_FLUSH
 }
 
 // Jacobi (eq. 2) and the standalone residual, persistent warps: warp g handles slices
@@ -2226,7 +2347,15 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     // (0.29 vs 0.33 ms), C3 0.205 vs 0.217 ms; blocks racing far ahead sweep on stale ghosts
     KP pp = p;
     pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 3;
-    k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(pp);
+    if (p.ring && L.tune.lazy_publish >= 0) {
+        if (ensure_smem(k_block_resident<WLR, true>, smem) != cudaSuccess) {
+            cudaGetLastError();
+            return false;
+        }
+        k_block_resident<WLR, true><<<(unsigned)L.q, threads, smem, st>>>(pp);
+    } else {
+        k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(pp);
+    }
     err = cudaGetLastError();
     return true;
 }
@@ -2476,6 +2605,8 @@ cudaError_t launch_async_multi(const SweepArgs &a, long long w_end, cudaStream_t
     p.w_end = w_end > 0 ? w_end : 1;
     p.m0 = a.m0;
     p.stop = &a.state->stop;
+    p.ring = a.ring;
+    p.bsum_arr = a.bsum_arr;
     return launch_block<true>(p, *a.L, st);
 }
 
@@ -2588,3 +2719,14 @@ cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st) {
 }
 
 }  // namespace bar
+
+#ifdef BAR_PROFILE_RESIDENT
+extern "C" int bar_debug_resident_profile(unsigned long long *out8, int reset) {
+    cudaMemcpyFromSymbol(out8, bar::g_res_prof, sizeof(unsigned long long) * 8);
+    if (reset) {
+        unsigned long long z[8] = {};
+        cudaMemcpyToSymbol(bar::g_res_prof, z, sizeof(z));
+    }
+    return (int)cudaGetLastError();
+}
+#endif
