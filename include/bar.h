@@ -230,6 +230,8 @@ typedef struct {
                                1 one ncclAllGather per iteration                                 */
     int32_t peer;           /* multi-GPU async: 0 peer memory when mapped, -1 the collective path */
     int32_t fronts;         /* async_order = 3: number of fronts (0 = 8)                          */
+    int32_t stage_bx;       /* k_block_duo: 0 stage b_J and x_J with the slab (bulk copies) where
+                               that keeps the blocks per SM, -1 per-row loads                    */
     int32_t lazy_publish;   /* k_block_resident: 0 non-blocking residual publication (a ring of
                                per-block partials, evaluated by block m % q), -1 one blocking
                                atomic per block and iteration                                    */

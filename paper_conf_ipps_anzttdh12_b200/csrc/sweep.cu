@@ -1047,13 +1047,14 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
 // Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
 struct DuoGeom {
-    uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, o_xs, bytes;
+    uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, o_xs, o_bj, o_xj, bytes;
 };
 
 // coded: the column block holds 1-byte codes and is followed by the subdomain's dictionary
 // (<= kDictMax int32 offsets); otherwise int32 columns. xs_len > 0 (staged gathers): a buffer
 // of xs_len doubles for the subdomain's off-block x intervals.
-__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, bool coded = false, int xs_len = 0) {
+__host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, bool coded = false, int xs_len = 0,
+                                                     bool bx = false) {
     DuoGeom g;
     g.vcap = (uint32_t)spb * kSlice * (uint32_t)wmax;
     g.o_col = g.vcap * 8;
@@ -1063,7 +1064,9 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
     g.o_ya = (g.o_sw + (((uint32_t)spb * 4 + 15) & ~15u) + 127) & ~127u;
     g.o_yb = g.o_ya + (uint32_t)R * 8;
     g.o_xs = g.o_yb + (uint32_t)R * 8;
-    g.bytes = g.o_xs + (uint32_t)xs_len * 8;
+    g.o_bj = g.o_xs + (uint32_t)xs_len * 8;  // bx: b_J and x_J staged with the slab
+    g.o_xj = g.o_bj + (bx ? (uint32_t)R * 8 : 0u);
+    g.bytes = g.o_xj + (bx ? (uint32_t)R * 8 : 0u);
     return g;
 }
 
@@ -1071,7 +1074,11 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
 // memory (relaxed loads); 2 coded columns with STAGED gathers: at the start of each subdomain the
 // block copies its off-block x intervals (Layout::iv, at most kMaxIv, x "as it stands", relaxed
 // loads, one coalesced pass) into shared memory, and phase 1 reads x there (Layout::sdict).
-template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0>
+// BX: b_J and x_J ride with the slab (two more bulk copies on the slab's mbarrier) instead of
+// per-row global loads in phase 1. x_J of l_{j+1} is read when its slab is issued, during l_j's
+// sweeps: only the block that sweeps l_{j+1} writes those rows in this launch (static claims), so
+// the bulk read races with no write. Requires even n (16-byte copies end inside b and x).
+template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0, bool BX = false>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     if (*(volatile const int *)p.stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
@@ -1081,7 +1088,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     __shared__ __align__(16) int32_t dbd[4][2];                 // [j % 4]: dictionary D0, D1 (CODED)
     __shared__ __align__(16) int32_t ivs[CODED == 2 ? 4 : 1][4 * kMaxIv];  // [j % 4]: x intervals of l_j
     const int R = p.R, spb = p.spb;
-    const DuoGeom g = duo_geom(R, spb, p.wmax, CODED != 0, CODED == 2 ? p.xs_len : 0);
+    const DuoGeom g = duo_geom(R, spb, p.wmax, CODED != 0, CODED == 2 ? p.xs_len : 0, BX);
     const int64_t q = (p.n + R - 1) / R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;  // = spb / 2
@@ -1094,7 +1101,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         const uint32_t nsl = (uint32_t)nsl_of(l);
         const uint32_t colb = CODED ? (uint32_t)(bd[1] - bd[0]) + (uint32_t)(db[1] - db[0]) * 4
                                     : (uint32_t)(bd[1] - bd[0]) * 4;
-        return (uint32_t)(bd[1] - bd[0]) * 8 + colb + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u);
+        const uint32_t bx = BX ? 2u * 8u * (uint32_t)min((int64_t)R, p.n - (int64_t)l * R) : 0u;
+        return (uint32_t)(bd[1] - bd[0]) * 8 + colb + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u) + bx;
     };
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
     auto issue_part = [&](int w, long long j) {
@@ -1104,6 +1112,13 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         if (w == 3) {  // what l_j's first phase reads directly: b_J, x_J and its ghost x ranges
             const int64_t TS = l * (int64_t)R;
             const uint32_t nrows = (uint32_t)min((int64_t)R, p.n - TS);
+            if (BX) {  // b_J, x_J with the slab; only the ghost ranges are prefetched into L2
+                fence_proxy_async_smem();
+                bulk_g2s_hint(smraw + g.o_bj, p.b + TS, nrows * 8, &bar, policy_evict_first());
+                bulk_g2s(smraw + g.o_xj, p.x_in + TS, nrows * 8, &bar);
+                if (p.gr) prefetch_ghost_x(p.x_in, gsm[j & 3], kGhostRanges);
+                return;
+            }
             const uintptr_t b0 = reinterpret_cast<uintptr_t>(p.b + TS) & ~(uintptr_t)15;
             const uintptr_t b1 = (reinterpret_cast<uintptr_t>(p.b + TS + nrows) + 15) & ~(uintptr_t)15;
             bulk_prefetch_l2_hint(reinterpret_cast<const void *>(b0), (uint32_t)(b1 - b0), policy_evict_first());
@@ -1245,8 +1260,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             auto dcol = [&](int e) -> int32_t {
                 return CODED ? lds_s32(ad + 4 * lds_u8(ac + e * kSlice)) : lds_s32(ac + e * kSlice * 4);
             };
-            const double bi = p.b[TS + loc];
-            ya[loc] = ldx<ASYNC>(p.x_in + TS + loc);
+            const double bi = BX ? lds_f64(sb + g.o_bj + 8u * loc) : p.b[TS + loc];
+            ya[loc] = BX ? lds_f64(sb + g.o_xj + 8u * loc) : ldx<ASYNC>(p.x_in + TS + loc);
             double acc = bi;
             for (int e0 = 0; e0 < wo; e0 += U) {
                 double xv[U];
@@ -2311,7 +2326,7 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
 }
 
 template <bool ASYNC, int WLR>
-cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st) {
+cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st, size_t smem_bx = 0) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
     const int coded = p.codes == nullptr ? 0 : (p.sdict != nullptr ? 2 : 1);
     auto kfn = coded == 2 ? (ext ? k_block_duo<ASYNC, WLR, true, 2> : k_block_duo<ASYNC, WLR, false, 2>)
@@ -2321,7 +2336,19 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
     cudaError_t e = ensure_smem(kfn, smem);
     if (e != cudaSuccess) return e;
-    const int64_t g = persistent_grid(occupancy(kfn, threads, smem), p, L);
+    const int occ = occupancy(kfn, threads, smem);
+    // b_J / x_J staged with the slab (coded layout, no EXT) where that keeps the blocks per SM
+    if (smem_bx > 0 && coded == 1 && !ext) {
+        auto kbx = k_block_duo<ASYNC, WLR, false, 1, true>;
+        if (ensure_smem(kbx, smem_bx) == cudaSuccess && occupancy(kbx, threads, smem_bx) >= occ) {
+            L.last_kernel = ASYNC ? "k_block_duo<async,coded,bx>" : "k_block_duo<sync,coded,bx>";
+            const int64_t g = persistent_grid(occ, p, L);
+            kbx<<<(unsigned)g, threads, smem_bx, st>>>(p);
+            return cudaGetLastError();
+        }
+        cudaGetLastError();
+    }
+    const int64_t g = persistent_grid(occ, p, L);
     kfn<<<(unsigned)g, threads, smem, st>>>(p);
     return cudaGetLastError();
 }
@@ -2462,7 +2489,11 @@ cudaError_t launch_block(KP p, const Layout &L, cudaStream_t st) {
             pc.iv = L.iv;
             pc.xs_len = (int32_t)L.xs_len;
         }
-        return launch_duo_t<ASYNC, 4>(pc, L, duo_smem, st);  // two rows per thread: <= 4 local entries
+        // b_J / x_J with the slab: n even (every subdomain's rows then end on a 16-byte boundary)
+        const size_t bx_smem = (coded && !staged && L.n % 2 == 0 && T.stage_bx >= 0)
+                                   ? duo_geom(L.R, L.spb, L.max_w, true, 0, true).bytes
+                                   : 0;
+        return launch_duo_t<ASYNC, 4>(pc, L, duo_smem, st, bx_smem);  // two rows per thread: <= 4 local entries
     }
     if (kind == 0 && pipe_on && p.w_end == 0 && geom_ok && aligned && pipe_smem <= kSmemMax) {
         L.last_kernel = ASYNC ? "k_block_pipe<async>" : "k_block_pipe<sync>";
