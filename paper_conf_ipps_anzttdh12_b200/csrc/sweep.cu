@@ -1294,7 +1294,12 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         __syncthreads();
         if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
             issue_part(warp, i + 1);
-            if (warp == 3) fetch_ring(i + 3);  // into slot (i + 3) % 4 (l_{i-1}'s, no longer read)
+            if (warp == 3) {
+                fetch_ring(i + 3);  // into slot (i + 3) % 4 (l_{i-1}'s, no longer read)
+                // ring slot of l_{i+2} complete; the next barrier publishes it (thread 0 reads it
+                // before the first barrier of the next subdomain)
+                asm volatile("cp.async.wait_group 1;" ::: "memory");
+            }
         }
         // first local sweep in the correction form; its numerator is the residual (a5)
 #pragma unroll
@@ -1354,12 +1359,19 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 if (t + 1 < p.k) __syncthreads();
             }
         }
-        // ring slot of l_{i+2} complete before the barrier below publishes it
-        if (warp == 3 && lane == 0) asm volatile("cp.async.wait_group 1;" ::: "memory");
-        // a6: write back
-        const double *yk = (p.k & 1) ? yb : ya;
+        // a6: write back (the thread's own two rows)
+        double *yk = (p.k & 1) ? yb : ya;
         for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
-        __syncthreads();
+        if (p.k == 1) {
+            __syncthreads();  // publishes the ring slot; guards ya against the next phase 1
+        } else if (p.k & 1) {
+            // no barrier: the next subdomain's y^0 goes into this one's final buffer yk, of which
+            // each thread writes only its own rows (already written back above), while threads
+            // still in the last sweep read only the other buffer; the barrier after sweep 1
+            // published the ring slot
+            yb = ya;
+            ya = yk;
+        }
     }
     if (warp == 3 && lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);

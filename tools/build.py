@@ -61,12 +61,14 @@ def nccl_paths() -> tuple[str, str] | None:
     return None
 
 
-def build_bar(force: bool = False) -> str:
-    """libbar.so: the C-ABI library (include/bar.h) with every kernel, for sm_100a only."""
+def build_bar(force: bool = False, out_name: str = "libbar.so", defines: tuple = ()) -> str:
+    """libbar.so: the C-ABI library (include/bar.h) with every kernel, for sm_100a only.
+    `defines` builds an instrumented copy under another name (e.g. BAR_PROFILE_RESIDENT=1 ->
+    libbar_prof.so for tools/resident_phase_probe.py); the product library never has them."""
     csrc = os.path.join(PKG, "csrc")
     srcs = sorted(glob.glob(os.path.join(csrc, "*.cu")))
     deps = srcs + sorted(glob.glob(os.path.join(csrc, "*.cuh"))) + [os.path.join(ROOT, "include", "bar.h")]
-    out = os.path.join(PKG, "libbar.so")
+    out = os.path.join(PKG, out_name)
     if not (force or _stale(out, deps)):
         return out
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-shared",
@@ -76,6 +78,7 @@ def build_bar(force: bool = False) -> str:
     if nccl is not None:
         inc, lib = nccl
         cmd += ["-DBAR_WITH_NCCL=1", "-I", inc, "-L", lib, "-Xlinker", "-rpath=" + lib]
+    cmd += ["-D" + d for d in defines]
     cmd += ["-o", out, *srcs]
     if nccl is not None:
         cmd += ["-l:libnccl.so.2"]
@@ -83,8 +86,9 @@ def build_bar(force: bool = False) -> str:
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc build of libbar.so failed")
-    with open(os.path.join(PKG, "ptxas_info.txt"), "w") as f:
-        f.write(r.stderr)
+    if not defines:
+        with open(os.path.join(PKG, "ptxas_info.txt"), "w") as f:
+            f.write(r.stderr)
     return out
 
 
@@ -106,4 +110,7 @@ def build_all(force: bool = False) -> None:
 
 
 if __name__ == "__main__":
-    build_all(force="--force" in sys.argv)
+    if "--profile-resident" in sys.argv:
+        build_bar(True, "libbar_prof.so", ("BAR_PROFILE_RESIDENT=1",))
+    else:
+        build_all(force="--force" in sys.argv)

@@ -1,3 +1,5 @@
+"""Per-phase cycle counts of k_block_resident (R17): build the instrumented library
+first with `python tools/build.py --profile-resident` (-> libbar_prof.so), then run on a GPU box."""
 import ctypes, os, sys
 sys.path.insert(0, os.getcwd())
 os.environ["BAR_LIB"] = "paper_conf_ipps_anzttdh12_b200/libbar_prof.so"
