@@ -575,3 +575,42 @@ def test_staged_gathers(bar, name, gen, R):
     MR.solve(_dev(np.ones(Rm.n)), None, None, k=5, max_global_iters=2, tol=0.0, mode="sync-block")
     assert "staged" not in MR.info()["last_sweep_kernel"]
     MR.close()
+
+
+@pytest.mark.parametrize("name,gen,R", [("s9_m600", lambda: W.stencil9_2d(600), 512),
+                                        ("s7_m64", lambda: W.stencil7_3d(64), 1024)])
+@pytest.mark.parametrize("stage_bx", [0, -1])
+@pytest.mark.parametrize("grid_cap", [0, 5])
+def test_duo_slab_staging_and_buffer_rotation(bar, name, gen, R, stage_bx, grid_cap):
+    """k_block_duo with b_J / x_J bulk-copied with the slab (tuning.stage_bx = 0, the default
+    where the blocks per SM stay the same) and with per-row loads (-1); grid_cap = 5
+    makes every block sweep dozens of subdomains in a row, which exercises the y-buffer rotation
+    that replaces the end-of-subdomain barrier (k odd: buffers swap, k even: no swap, k = 1:
+    barrier). Sync-block-(k) for k = 2, 3, 5 and Jacobi match the oracle to 1e-12 after 3
+    iterations; async-(5) converges."""
+    import torch
+
+    A = gen()
+    b = np.random.default_rng(5).uniform(0.5, 1.5, A.n)
+    x0 = np.random.default_rng(6).uniform(-1, 1, A.n)
+    M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "single_launch": -1, "stage_bx": stage_bx,
+                                          "grid_cap": grid_cap})
+    kernels = set()
+    for mode, k in (("sync-block", 5), ("sync-block", 2), ("sync-block", 3), ("jacobi", 1)):
+        ref = x0
+        for _ in range(3):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x = torch.empty(A.n, dtype=torch.float64, device="cuda")
+        M.solve(_dev(b), _dev(x0), x, k=k, max_global_iters=3, tol=0.0, mode=mode)
+        kernels.add(M.info()["last_sweep_kernel"])
+        _close(x.cpu().numpy(), ref)
+    x, info = M.solve(_dev(b), None, None, k=5, tol=1e-10, mode="async")
+    kernels.add(M.info()["last_sweep_kernel"])
+    assert info["converged"] and O.rel_res(A, b, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    M.close()
+    assert all(kn.startswith("k_block_duo<") and ",coded" in kn for kn in kernels), kernels
+    staged = {kn for kn in kernels if kn.endswith(",bx>")}
+    if stage_bx < 0:
+        assert not staged, kernels
+    elif name == "s7_m64":  # C5's geometry: the staged variant keeps two blocks per SM
+        assert staged, kernels

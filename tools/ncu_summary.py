@@ -5,6 +5,7 @@
     python tools/ncu_summary.py launches gpurun_out/launches.csv profiles/r01_c5_launches.txt
 """
 import csv
+import re
 import io
 import json
 import subprocess
@@ -55,7 +56,7 @@ def full(rep, out, traffic_json=None):
 
         kern = d.get("Kernel Name", "?")
         json.dump({"dram_bytes_per_launch": sum(dram) / len(dram), "source": rep, "libbar_sha256": bench.lib_hash(),
-                   "kernel": KERNEL_NAMES.get(kern.split("(")[0].split("::")[-1], kern), "R": R_ARG},
+                   "kernel": libbar_name(kern), "R": R_ARG},
                   open(traffic_json, "w"))
     print("\n".join(lines))
 
@@ -84,9 +85,16 @@ def launches(csv_path, out):
     print("\n".join(lines))
 
 
-# ncu kernel names -> the names libbar reports (bar_matrix_info.last_sweep_kernel)
-KERNEL_NAMES = {"k_block_duo<1, 4, 0, 1>": "k_block_duo<async,coded>", "k_block_duo<0, 4, 0, 1>": "k_block_duo<sync,coded>",
-                "k_block_duo<1, 4, 0, 0>": "k_block_duo<async>", "k_block_duo<0, 4, 0, 0>": "k_block_duo<sync>"}
+def libbar_name(ncu_name):
+    """ncu's demangled k_block_duo<ASYNC, WLR, EXT, CODED, BX> -> the name libbar reports
+    (bar_matrix_info.last_sweep_kernel); other kernels keep their ncu name."""
+    m = re.search(r"k_block_duo<([^>]*)>", ncu_name)
+    if not m:
+        return ncu_name
+    a = [int(re.sub(r"\(\w+\)", "", t).strip()) for t in m.group(1).split(",")]
+    a += [0] * (5 - len(a))
+    return ("k_block_duo<" + ("async" if a[0] else "sync") + {0: "", 1: ",coded", 2: ",staged"}[a[3]]
+            + {0: "", 1: ",bx", 2: ",x"}[a[4]] + ">")
 R_ARG = None
 
 if __name__ == "__main__":
