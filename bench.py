@@ -23,7 +23,6 @@ subdomain size in grid lines); such values carry "extrapolated": true and say ho
 from __future__ import annotations
 
 import argparse
-import hashlib
 import json
 import os
 import statistics
@@ -83,8 +82,11 @@ def load_peaks():
 
 
 def lib_hash() -> str:
-    p = os.path.join(ROOT, "paper_conf_ipps_anzttdh12_b200", "libbar.so")
-    return hashlib.sha256(open(p, "rb").read()).hexdigest()[:16] if os.path.exists(p) else "missing"
+    """The loaded libbar's build id (bar_build_id: a hash of its sources and flags, the same for
+    every rebuild of the same sources)."""
+    from paper_conf_ipps_anzttdh12_b200 import bar
+
+    return bar.bar_build_id()
 
 
 class ClockSampler:
@@ -461,7 +463,7 @@ def main():
     if not multi and os.path.exists(prof):
         try:
             tj = json.load(open(prof))
-            if tj.get("kernel") == kernel_name and tj.get("libbar_sha256") == lib_hash() and tj.get("R") == args.R:
+            if tj.get("kernel") == kernel_name and tj.get("libbar_build_id") == lib_hash() and tj.get("R") == args.R:
                 roofline["traffic"] = tj["dram_bytes_per_launch"]
                 roofline["frac_dram"] = round(tj["dram_bytes_per_launch"] / (kernel_ms * 1e-3) / 1e9 / peak, 4)
                 roofline["traffic_source"] = tj.get("source", prof)
@@ -572,7 +574,7 @@ def main():
         "oracle_iters": (cpu or {}).get(f"sync_block_{args.k}" if args.mode != "jacobi" else "jacobi", {}).get("iters"),
         "gpu_launches": launches, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
         "clocks": clk.summary(), "setup_s": {"generate": round(t_gen, 2), "create": round(t_setup, 2)},
-        "layout": minfo, "libbar_sha256": lib_hash(),
+        "layout": minfo, "libbar_build_id": lib_hash(),
     }
     line.update(extra)
     if rank == 0:

@@ -401,6 +401,13 @@ void bar_dist_destroy(bar_dist D);
 /* bar_last_error — text of the last failure on the calling thread ("" if none). */
 const char *bar_last_error(void);
 
+/* bar_build_id — identity of this build: "src:<16 hex> sm_100a", the hex being a SHA-256 over the
+ * library's sources (csrc/*.cu, *.cuh, include/bar.h) and its nvcc flags, fixed at build time
+ * (tools/build.py). Unlike a hash of the .so (nvcc output is not byte-reproducible) it is the same
+ * for every build of the same sources; measurements stamped with it (profiles/traffic_*.json) are
+ * used only by a library with the same id. Static string, never NULL. */
+const char *bar_build_id(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -35,7 +35,7 @@ EXPORTS = ("bar_create_csr", "bar_solve", "bar_solve_ex", "bar_sweep", "bar_resi
            "bar_set_tuning", "bar_destroy", "bar_last_error", "bar_create_csr_dist", "bar_nccl_unique_id",
            "bar_dist_ghosts", "bar_dist_localize", "bar_dist_plan", "bar_dist_create", "bar_dist_link_loopback",
            "bar_dist_solve", "bar_dist_solve_loopback", "bar_dist_sweep", "bar_dist_p2p_handles",
-           "bar_dist_enable_p2p", "bar_dist_set_tuning", "bar_dist_destroy")
+           "bar_dist_enable_p2p", "bar_dist_set_tuning", "bar_dist_destroy", "bar_build_id")
 
 
 class SolveInfo(ctypes.Structure):
@@ -119,6 +119,8 @@ _lib.bar_destroy.restype = None
 _lib.bar_destroy.argtypes = [_vp]
 _lib.bar_last_error.restype = ctypes.c_char_p
 _lib.bar_last_error.argtypes = []
+_lib.bar_build_id.restype = ctypes.c_char_p
+_lib.bar_build_id.argtypes = []
 
 
 class BarError(RuntimeError):
@@ -150,6 +152,10 @@ def _check(st: int):
 
 def bar_last_error() -> str:
     return _lib.bar_last_error().decode()
+
+
+def bar_build_id() -> str:
+    return _lib.bar_build_id().decode()
 
 
 def bar_create_csr(n, nnz, rowptr, col, val, rows_per_block, device=0):

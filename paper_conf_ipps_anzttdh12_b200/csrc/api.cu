@@ -135,6 +135,11 @@ extern "C" {
 
 const char *bar_last_error(void) { return g_err.c_str(); }
 
+#ifndef BAR_SOURCE_ID
+#define BAR_SOURCE_ID "unknown"
+#endif
+const char *bar_build_id(void) { return "src:" BAR_SOURCE_ID " sm_100a"; }
+
 bar_status bar_create_csr(int64_t n, int64_t nnz, const int32_t *rowptr, const int32_t *col, const double *val,
                           int32_t rows_per_block, int device, bar_matrix *out) {
     g_err.clear();

@@ -6,6 +6,7 @@ snapshot. ``build_all()`` is what ``__graft_entry__.build()`` calls.
 from __future__ import annotations
 
 import glob
+import hashlib
 import os
 import subprocess
 import sys
@@ -61,6 +62,16 @@ def nccl_paths() -> tuple[str, str] | None:
     return None
 
 
+def source_id(deps: list[str], flags: list[str]) -> str:
+    """SHA-256 (16 hex) over the library's sources (paths relative to the repo) and nvcc flags:
+    the build identity libbar reports through bar_build_id()."""
+    h = hashlib.sha256()
+    for d in sorted(deps):
+        h.update(os.path.relpath(d, ROOT).encode() + b"\0" + open(d, "rb").read() + b"\0")
+    h.update(" ".join(flags).encode())
+    return h.hexdigest()[:16]
+
+
 def build_bar(force: bool = False, out_name: str = "libbar.so", defines: tuple = ()) -> str:
     """libbar.so: the C-ABI library (include/bar.h) with every kernel, for sm_100a only.
     `defines` builds an instrumented copy under another name (e.g. BAR_PROFILE_RESIDENT=1 ->
@@ -71,14 +82,14 @@ def build_bar(force: bool = False, out_name: str = "libbar.so", defines: tuple =
     out = os.path.join(PKG, out_name)
     if not (force or _stale(out, deps)):
         return out
-    cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-shared",
-           "-Xptxas", "-v", "--expt-relaxed-constexpr",
+    flags = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-v",
+             "--expt-relaxed-constexpr", *["-D" + d for d in defines]]
+    cmd = [NVCC, *flags, "-DBAR_SOURCE_ID=\"" + source_id(deps, flags) + "\"",
            "-I", os.path.join(ROOT, "include"), "-I", csrc]
     nccl = nccl_paths()
     if nccl is not None:
         inc, lib = nccl
         cmd += ["-DBAR_WITH_NCCL=1", "-I", inc, "-L", lib, "-Xlinker", "-rpath=" + lib]
-    cmd += ["-D" + d for d in defines]
     cmd += ["-o", out, *srcs]
     if nccl is not None:
         cmd += ["-l:libnccl.so.2"]

@@ -55,7 +55,7 @@ def full(rep, out, traffic_json=None):
         import bench
 
         kern = d.get("Kernel Name", "?")
-        json.dump({"dram_bytes_per_launch": sum(dram) / len(dram), "source": rep, "libbar_sha256": bench.lib_hash(),
+        json.dump({"dram_bytes_per_launch": sum(dram) / len(dram), "source": rep, "libbar_build_id": bench.lib_hash(),
                    "kernel": libbar_name(kern), "R": R_ARG},
                   open(traffic_json, "w"))
     print("\n".join(lines))
