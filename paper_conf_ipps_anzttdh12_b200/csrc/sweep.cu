@@ -1046,6 +1046,29 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // that also frees the slab. The slab of the next subdomain is issued right after that barrier,
 // split over four warps as in k_block_pipe; its mbarrier byte count is posted before it.
 // Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
+// Phase timing of k_block_duo (a profiling build only: -DBAR_PROFILE_DUO, tools/duo_phase_probe.py):
+// lane 0 of warps 0 (slab issuer), 3 (b/x, ring and prefetch issuer) and nw - 1 (rows only) sums
+// clock64 deltas between the marks over the launch; added into g_duo_prof[3][8] at the end.
+#ifdef BAR_PROFILE_DUO
+__device__ unsigned long long g_duo_prof[3][8];
+#define DUO_PROF_DECL                                                                         \
+    const int prof_w = warp == 0 ? 0 : warp == 3 ? 1 : warp == nw - 1 ? 2 : -1;              \
+    long long prof_t[8] = {0, 0, 0, 0, 0, 0, 0, 0}, prof_last = clock64();
+#define DUO_PROF_MARK(i)                         \
+    if (prof_w >= 0 && lane == 0) {              \
+        const long long now = clock64();         \
+        prof_t[i] += now - prof_last;            \
+        prof_last = now;                         \
+    }
+#define DUO_PROF_FLUSH                                                                          \
+    if (prof_w >= 0 && lane == 0)                                                               \
+        for (int i = 0; i < 8; ++i) atomicAdd(&g_duo_prof[prof_w][i], (unsigned long long)prof_t[i]);
+#else
+#define DUO_PROF_DECL
+#define DUO_PROF_MARK(i)
+#define DUO_PROF_FLUSH
+#endif
+
 struct DuoGeom {
     uint32_t vcap, o_col, o_dict, o_sptr, o_sw, o_ya, o_yb, o_xs, o_bj, o_xj, bytes;
 };
@@ -1078,7 +1101,11 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
 // per-row global loads in phase 1. x_J of l_{j+1} is read when its slab is issued, during l_j's
 // sweeps: only the block that sweeps l_{j+1} writes those rows in this launch (static claims), so
 // the bulk read races with no write. Requires even n (16-byte copies end inside b and x).
-template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0, bool BX = false>
+// WOR > 0 (coded columns, <= WOR off-block entries per row): phase 1 fully unrolled over the
+// off-block entries in three stages — (A) a row's codes, offsets and all its gathers issued,
+// (B) its local entries into registers, (C) its off-block sum — with one 64-bit row base per
+// row and 32-bit offsets (the generic loop re-derived a 64-bit address per entry).
+template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0, bool BX = false, int WOR = 0>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     if (*(volatile const int *)p.stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
@@ -1105,6 +1132,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         return (uint32_t)(bd[1] - bd[0]) * 8 + colb + ((nsl * 8 + 15) & ~15u) + ((nsl * 4 + 15) & ~15u) + bx;
     };
     // part w of the issue for l_j (slab) and the L2 prefetches of what l_j / l_{j+1} read directly
+    // (w = 3: b_J and x_J; the ghost ranges are prefetched separately, ghost_prefetch)
     auto issue_part = [&](int w, long long j) {
         const long long l = lof(j);
         if (l >= C.lend) return;
@@ -1116,7 +1144,6 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 fence_proxy_async_smem();
                 bulk_g2s_hint(smraw + g.o_bj, p.b + TS, nrows * 8, &bar, policy_evict_first());
                 bulk_g2s(smraw + g.o_xj, p.x_in + TS, nrows * 8, &bar);
-                if (p.gr) prefetch_ghost_x(p.x_in, gsm[j & 3], kGhostRanges);
                 return;
             }
             const uintptr_t b0 = reinterpret_cast<uintptr_t>(p.b + TS) & ~(uintptr_t)15;
@@ -1125,7 +1152,6 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             const uintptr_t x0 = reinterpret_cast<uintptr_t>(p.x_in + TS) & ~(uintptr_t)15;
             const uintptr_t x1 = (reinterpret_cast<uintptr_t>(p.x_in + TS + nrows) + 15) & ~(uintptr_t)15;
             bulk_prefetch_l2(reinterpret_cast<const void *>(x0), (uint32_t)(x1 - x0));
-            if (p.gr) prefetch_ghost_x(p.x_in, gsm[j & 3], kGhostRanges);
             return;
         }
         fence_proxy_async_smem();
@@ -1207,7 +1233,13 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         }
         mbar_arrive_expect_tx(&bar, slab_bytes(lof(0), bnd[0], dbd[0]));
         for (int w = 0; w < 4; ++w) issue_part(w, 0);
+        if (p.gr && lof(0) < C.lend) prefetch_ghost_x(p.x_in, gsm[0], kGhostRanges);
     }
+    // the issue after the slab is freed, split over warps so that no warp's share holds up the
+    // barrier after the first sweep: roles 0..3 the slab parts (issue_part), 4 the ghost-range L2
+    // prefetch, 5 the ring of bounds (cp.async, always the same thread: its groups are per thread)
+    constexpr int kRoles = 6;
+    const int ring_warp = (kRoles - 1) % nw;
     double *xs = reinterpret_cast<double *>(smraw + g.o_xs);
     const uint32_t sxs = smem_u32(xs);
     if (CODED == 2)  // slots past a subdomain's intervals are read (times 0) by padding entries
@@ -1216,12 +1248,14 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
 
     constexpr int NP = WLR / 2;
     double rr = 0.0, bb = 0.0;
+    DUO_PROF_DECL
     for (int i = 0;; ++i) {
         const long long l = lof(i);
         if (l >= C.lend) break;
         const int64_t TS = l * (int64_t)R;
         const int nrows = (int)min((int64_t)R, p.n - TS);
         const int nsl = (nrows + kSlice - 1) / kSlice;
+        DUO_PROF_MARK(7)
         if (CODED == 2) {  // a3 staged: the off-block x intervals, as they stand, into shared memory
             const int32_t *iv = ivs[i & 3];
 #pragma unroll
@@ -1232,6 +1266,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             __syncthreads();
         }
         mbar_wait(&bar, i & 1);
+        DUO_PROF_MARK(0)
         double lv[2][WLR];
         uint32_t lc[2][NP];
         double s[2] = {0.0, 0.0};
@@ -1247,6 +1282,72 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
         // it stands, the local entries into registers
         const int64_t *ssp = reinterpret_cast<const int64_t *>(smraw + g.o_sptr);
         const uint32_t sb = smem_u32(smraw);
+        if constexpr (WOR > 0) {
+            static_assert(CODED == 1, "the unrolled phase 1 reads coded columns");
+            const uint32_t ad = sb + g.o_dict;
+            uint32_t av[2], ac[2];
+            int wl[2], wo[2];
+            double xv[2][WOR], bi[2], xj[2];
+            // (A) offsets and gathers of row h (x as it stands)
+            auto stage_a = [&](int h) {
+                const int sl = warp + h * nw, loc = row_of(h);
+                const bool v = sl < nsl && loc < nrows;
+                const int sw = v ? lds_s32(sb + g.o_sw + 4 * sl) : 0;
+                wl[h] = sw & 0xffff;
+                wo[h] = sw >> 16;
+                const uint32_t off = v ? (uint32_t)(ssp[sl] - ssp[0]) + lane : 0u;
+                av[h] = sb + off * 8;
+                ac[h] = sb + g.o_col + off;
+                const double *xr = p.x_in + (TS + loc);
+#pragma unroll
+                for (int e = 0; e < WOR; ++e)
+                    xv[h][e] = e < wo[h] ? ldx<ASYNC>(xr + lds_s32(ad + 4 * lds_u8(ac[h] + e * kSlice))) : 0.0;
+                bi[h] = !v ? 0.0 : BX ? lds_f64(sb + g.o_bj + 8u * loc) : p.b[TS + loc];
+                xj[h] = !v ? 0.0 : BX ? lds_f64(sb + g.o_xj + 8u * loc) : ldx<ASYNC>(xr);
+            };
+            // (B) local entries of row h into registers, branch-free (slots past wl read in-bounds
+            // shared memory, zeroed)
+            auto stage_b = [&](int h) {
+                const int loc = row_of(h);
+#pragma unroll
+                for (int e = 0; e < WLR; ++e) {
+                    const bool ok = e < wl[h];
+                    const double v = lds_f64(av[h] + (wo[h] + e) * kSlice * 8);
+                    const uint32_t c = (uint32_t)(loc + lds_s32(ad + 4 * lds_u8(ac[h] + (wo[h] + e) * kSlice))) & 0xffffu;
+                    lv[h][e] = ok ? v : 0.0;
+                    lc[h][e >> 1] |= (ok ? c : 0u) << (16 * (e & 1));
+                }
+            };
+            // (C) s_i = b_i - sum_{j not in J} a_ij x_j; y^0 = x_J
+            auto stage_c = [&](int h) {
+                const int sl = warp + h * nw, loc = row_of(h);
+                double acc = bi[h];
+#pragma unroll
+                for (int e = 0; e < WOR; ++e)
+                    if (e < wo[h]) acc -= lds_f64(av[h] + e * kSlice * 8) * xv[h][e];
+                s[h] = acc;
+                if (sl < nsl && loc < nrows) ya[loc] = xj[h];
+                bb += bi[h] * bi[h];
+            };
+            if constexpr (WOR <= 4) {
+                // both rows' gathers in flight together (one gather latency per subdomain instead
+                // of two); the local entries after the sums, so the gathered values and the
+                // local entries are never live at once (64 registers)
+                stage_a(0);
+                stage_a(1);
+                stage_c(0);
+                stage_c(1);
+                stage_b(0);
+                stage_b(1);
+            } else {  // one row at a time, its local entries loaded while its gathers fly
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    stage_a(h);
+                    stage_b(h);
+                    stage_c(h);
+                }
+            }
+        } else
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
             const int sl = warp + h * nw, loc = row_of(h);
@@ -1288,19 +1389,27 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             }
             bb += bi * bi;
         }
+        DUO_PROF_MARK(1)
         // post the byte count of l_{i+1}'s slab before the barrier that frees the buffer
         if (threadIdx.x == 0 && lof(i + 1) < C.lend)
             mbar_arrive_expect_tx(&bar, slab_bytes(lof(i + 1), bnd[(i + 1) & 3], dbd[(i + 1) & 3]));
         __syncthreads();
-        if (warp < 4 && lane == 0) {  // the slab is free: stream l_{i+1} into it
-            issue_part(warp, i + 1);
-            if (warp == 3) {
-                fetch_ring(i + 3);  // into slot (i + 3) % 4 (l_{i-1}'s, no longer read)
-                // ring slot of l_{i+2} complete; the next barrier publishes it (thread 0 reads it
-                // before the first barrier of the next subdomain)
-                asm volatile("cp.async.wait_group 1;" ::: "memory");
+        DUO_PROF_MARK(2)
+        if (lane == 0) {  // the slab is free: stream l_{i+1} into it
+            for (int r = warp; r < kRoles; r += nw) {
+                if (r < 4) {
+                    issue_part(r, i + 1);
+                } else if (r == 4) {
+                    if (p.gr && lof(i + 1) < C.lend) prefetch_ghost_x(p.x_in, gsm[(i + 1) & 3], kGhostRanges);
+                } else {
+                    fetch_ring(i + 3);  // into slot (i + 3) % 4 (l_{i-1}'s, no longer read)
+                    // ring slot of l_{i+2} complete; the next barrier publishes it (thread 0 reads
+                    // it before the first barrier of the next subdomain)
+                    asm volatile("cp.async.wait_group 1;" ::: "memory");
+                }
             }
         }
+        DUO_PROF_MARK(3)
         // first local sweep in the correction form; its numerator is the residual (a5)
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
@@ -1315,9 +1424,11 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             if (EXT) yb[loc] = ext_update(xo, xo + lv[h][0] * acc, p.frozen && p.frozen[TS + loc], p.tau);
             else yb[loc] = xo + lv[h][0] * acc;
         }
+        DUO_PROF_MARK(4)
         // every thread writes back exactly its own two rows, so the last sweep needs no barrier
         // before the write-back (the barrier after it guards the buffers' reuse)
         if (p.k > 1) __syncthreads();
+        DUO_PROF_MARK(5)
         // a4: sweeps 2..k, direct form, off-block part frozen
         if (EXT) {
             for (int t = 1; t < p.k; ++t) {
@@ -1359,6 +1470,7 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 if (t + 1 < p.k) __syncthreads();
             }
         }
+        DUO_PROF_MARK(6)
         // a6: write back (the thread's own two rows)
         double *yk = (p.k & 1) ? yb : ya;
         for (int r = threadIdx.x; r < nrows; r += blockDim.x) stx<ASYNC>(p.x_out + TS + r, yk[r]);
@@ -1373,7 +1485,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
             ya = yk;
         }
     }
-    if (warp == 3 && lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
+    DUO_PROF_FLUSH
+    if (warp == ring_warp && lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
     reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
@@ -2337,12 +2450,28 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
     return cudaGetLastError();
 }
 
+// Name of the coded k_block_duo variant (Layout::last_kernel, bench roofline.kernel): wo4 / wo8 =
+// the unrolled phase 1, bx = b_J, x_J with the slab.
+const char *duo_coded_name(bool async, bool bx, int wor) {
+    static const char *names[2][2][3] = {
+        {{"k_block_duo<sync,coded>", "k_block_duo<sync,coded,wo4>", "k_block_duo<sync,coded,wo8>"},
+         {"k_block_duo<sync,coded,bx>", "k_block_duo<sync,coded,wo4,bx>", "k_block_duo<sync,coded,wo8,bx>"}},
+        {{"k_block_duo<async,coded>", "k_block_duo<async,coded,wo4>", "k_block_duo<async,coded,wo8>"},
+         {"k_block_duo<async,coded,bx>", "k_block_duo<async,coded,wo4,bx>", "k_block_duo<async,coded,wo8,bx>"}}};
+    return names[async][bx][wor == 0 ? 0 : wor == 4 ? 1 : 2];
+}
+
 template <bool ASYNC, int WLR>
 cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st, size_t smem_bx = 0) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
     const int coded = p.codes == nullptr ? 0 : (p.sdict != nullptr ? 2 : 1);
+    // unrolled phase 1 (WOR) for the coded layouts with <= 4 / <= 8 off-block entries per row
+    const int wor = coded == 1 && !ext && L.tune.unroll_off >= 0 ? (L.max_wo <= 4 ? 4 : (L.max_wo <= 8 ? 8 : 0)) : 0;
     auto kfn = coded == 2 ? (ext ? k_block_duo<ASYNC, WLR, true, 2> : k_block_duo<ASYNC, WLR, false, 2>)
-               : coded == 1 ? (ext ? k_block_duo<ASYNC, WLR, true, 1> : k_block_duo<ASYNC, WLR, false, 1>)
+               : coded == 1 ? (ext ? k_block_duo<ASYNC, WLR, true, 1>
+                               : wor == 4 ? k_block_duo<ASYNC, WLR, false, 1, false, 4>
+                               : wor == 8 ? k_block_duo<ASYNC, WLR, false, 1, false, 8>
+                                          : k_block_duo<ASYNC, WLR, false, 1>)
                             : (ext ? k_block_duo<ASYNC, WLR, true, 0> : k_block_duo<ASYNC, WLR, false, 0>);
     const int threads = L.spb / 2 * kSlice;
     std::lock_guard<std::recursive_mutex> lk(g_launch_mu);
@@ -2351,15 +2480,17 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     const int occ = occupancy(kfn, threads, smem);
     // b_J / x_J staged with the slab (coded layout, no EXT) where that keeps the blocks per SM
     if (smem_bx > 0 && coded == 1 && !ext) {
-        auto kbx = k_block_duo<ASYNC, WLR, false, 1, true>;
+        auto kbx = wor == 4 ? k_block_duo<ASYNC, WLR, false, 1, true, 4>
+                   : wor == 8 ? k_block_duo<ASYNC, WLR, false, 1, true, 8> : k_block_duo<ASYNC, WLR, false, 1, true>;
         if (ensure_smem(kbx, smem_bx) == cudaSuccess && occupancy(kbx, threads, smem_bx) >= occ) {
-            L.last_kernel = ASYNC ? "k_block_duo<async,coded,bx>" : "k_block_duo<sync,coded,bx>";
+            L.last_kernel = duo_coded_name(ASYNC, true, wor);
             const int64_t g = persistent_grid(occ, p, L);
             kbx<<<(unsigned)g, threads, smem_bx, st>>>(p);
             return cudaGetLastError();
         }
         cudaGetLastError();
     }
+    if (coded == 1 && !ext) L.last_kernel = duo_coded_name(ASYNC, false, wor);
     const int64_t g = persistent_grid(occ, p, L);
     kfn<<<(unsigned)g, threads, smem, st>>>(p);
     return cudaGetLastError();
@@ -2762,6 +2893,17 @@ cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st) {
 }
 
 }  // namespace bar
+
+#ifdef BAR_PROFILE_DUO
+extern "C" int bar_debug_duo_profile(unsigned long long *out24, int reset) {
+    cudaMemcpyFromSymbol(out24, bar::g_duo_prof, sizeof(unsigned long long) * 24);
+    if (reset) {
+        unsigned long long z[24] = {};
+        cudaMemcpyToSymbol(bar::g_duo_prof, z, sizeof(z));
+    }
+    return (int)cudaGetLastError();
+}
+#endif
 
 #ifdef BAR_PROFILE_RESIDENT
 extern "C" int bar_debug_resident_profile(unsigned long long *out8, int reset) {

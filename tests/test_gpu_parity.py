@@ -578,23 +578,25 @@ def test_staged_gathers(bar, name, gen, R):
 
 
 @pytest.mark.parametrize("name,gen,R", [("s9_m600", lambda: W.stencil9_2d(600), 512),
-                                        ("s7_m64", lambda: W.stencil7_3d(64), 1024)])
+                                        ("s7_m128", lambda: W.stencil7_3d(128), 256)])
 @pytest.mark.parametrize("stage_bx", [0, -1])
 @pytest.mark.parametrize("grid_cap", [0, 5])
-def test_duo_slab_staging_and_buffer_rotation(bar, name, gen, R, stage_bx, grid_cap):
+@pytest.mark.parametrize("unroll_off", [0, -1])
+def test_duo_slab_staging_and_buffer_rotation(bar, name, gen, R, stage_bx, grid_cap, unroll_off):
     """k_block_duo with b_J / x_J bulk-copied with the slab (tuning.stage_bx = 0, the default
     where the blocks per SM stay the same) and with per-row loads (-1); grid_cap = 5
     makes every block sweep dozens of subdomains in a row, which exercises the y-buffer rotation
     that replaces the end-of-subdomain barrier (k odd: buffers swap, k even: no swap, k = 1:
-    barrier). Sync-block-(k) for k = 2, 3, 5 and Jacobi match the oracle to 1e-12 after 3
-    iterations; async-(5) converges."""
+    barrier). unroll_off: the unrolled phase 1 (0; wo4 on the 3D stencil's <= 4 off-block entries
+    per row, wo8 on the 2D stencil's <= 7) and the generic loop (-1). Sync-block-(k) for k = 2, 3, 5 and Jacobi match the oracle to
+    1e-12 after 3 iterations; async-(5) converges."""
     import torch
 
     A = gen()
     b = np.random.default_rng(5).uniform(0.5, 1.5, A.n)
     x0 = np.random.default_rng(6).uniform(-1, 1, A.n)
     M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "single_launch": -1, "stage_bx": stage_bx,
-                                          "grid_cap": grid_cap})
+                                          "grid_cap": grid_cap, "unroll_off": unroll_off})
     kernels = set()
     for mode, k in (("sync-block", 5), ("sync-block", 2), ("sync-block", 3), ("jacobi", 1)):
         ref = x0
@@ -609,8 +611,10 @@ def test_duo_slab_staging_and_buffer_rotation(bar, name, gen, R, stage_bx, grid_
     assert info["converged"] and O.rel_res(A, b, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
     M.close()
     assert all(kn.startswith("k_block_duo<") and ",coded" in kn for kn in kernels), kernels
+    want = {-1: None, 0: ",wo4" if name == "s7_m128" else ",wo8"}[unroll_off]
+    assert all((",wo" not in kn) if want is None else (want + "," in kn or want + ">" in kn) for kn in kernels), kernels
     staged = {kn for kn in kernels if kn.endswith(",bx>")}
     if stage_bx < 0:
         assert not staged, kernels
-    elif name == "s7_m64":  # C5's geometry: the staged variant keeps two blocks per SM
+    elif name == "s7_m128":  # C5's geometry (R = two grid lines): the staged variant keeps two blocks per SM
         assert staged, kernels

@@ -123,5 +123,7 @@ def build_all(force: bool = False) -> None:
 if __name__ == "__main__":
     if "--profile-resident" in sys.argv:
         build_bar(True, "libbar_prof.so", ("BAR_PROFILE_RESIDENT=1",))
+    elif "--profile-duo" in sys.argv:
+        build_bar(True, "libbar_duoprof.so", ("BAR_PROFILE_DUO=1",))
     else:
         build_all(force="--force" in sys.argv)

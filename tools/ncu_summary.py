@@ -86,15 +86,19 @@ def launches(csv_path, out):
 
 
 def libbar_name(ncu_name):
-    """ncu's demangled k_block_duo<ASYNC, WLR, EXT, CODED, BX> -> the name libbar reports
-    (bar_matrix_info.last_sweep_kernel); other kernels keep their ncu name."""
+    """ncu's demangled k_block_duo<ASYNC, WLR, EXT, CODED, BX, WOR> -> the name libbar
+    reports (bar_matrix_info.last_sweep_kernel, sweep.cu duo_coded_name); other kernels keep their
+    ncu name."""
     m = re.search(r"k_block_duo<([^>]*)>", ncu_name)
     if not m:
         return ncu_name
     a = [int(re.sub(r"\(\w+\)", "", t).strip()) for t in m.group(1).split(",")]
-    a += [0] * (5 - len(a))
+    a += [0] * (6 - len(a))
+    wo = "" if a[5] == 0 else f",wo{a[5]}"
     return ("k_block_duo<" + ("async" if a[0] else "sync") + {0: "", 1: ",coded", 2: ",staged"}[a[3]]
-            + {0: "", 1: ",bx", 2: ",x"}[a[4]] + ">")
+            + wo + {0: "", 1: ",bx", 2: ",x"}[a[4]] + ">")
+
+
 R_ARG = None
 
 if __name__ == "__main__":
