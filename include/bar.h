@@ -240,8 +240,9 @@ typedef struct {
     int32_t overlap;        /* multi-GPU collective path: 0 sweep the interior subdomains (no ghost
                                reads) on a second stream while the halo exchange runs, then the
                                boundary ones; -1 one sweep after the exchange                    */
-    int32_t unroll_off;     /* k_block_duo, coded columns: 0 phase 1 unrolled over <= 4 / <= 8
-                               off-block entries per row, -1 the generic loop                    */
+    int32_t unroll_off;     /* k_block_duo, coded columns: 0 phase 1 unrolled where a row has <= 4
+                               off-block entries (both rows' gathers in flight), -1 the generic
+                               loop                                                              */
 } bar_tuning;
 
 /* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a

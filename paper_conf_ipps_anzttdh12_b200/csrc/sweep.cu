@@ -1102,9 +1102,14 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
 // sweeps: only the block that sweeps l_{j+1} writes those rows in this launch (static claims), so
 // the bulk read races with no write. Requires even n (16-byte copies end inside b and x).
 // WOR > 0 (coded columns, <= WOR off-block entries per row): phase 1 fully unrolled over the
-// off-block entries in three stages — (A) a row's codes, offsets and all its gathers issued,
-// (B) its local entries into registers, (C) its off-block sum — with one 64-bit row base per
-// row and 32-bit offsets (the generic loop re-derived a 64-bit address per entry).
+// off-block entries in three stages — (A) both rows' codes, offsets and all their gathers issued,
+// (C) the off-block sums, (B) the local entries into registers — with one 64-bit row base per row
+// and 32-bit offsets (the generic loop re-derived a 64-bit address per entry and exposed one
+// gather latency per row). WOR = 4 (3D stencils at R = two grid lines); measured on B200 (round
+// 2, tools/kernel_ab.py, same box): C5 async 2.35 vs 2.50 ms, sync-block 2.32 vs 2.39 ms per
+// launch. With up to 8 off-block entries (2D 9-point, C4) the 16 gathered values of two rows
+// spill at 64 registers and one row at a time is no faster than the generic loop (0.359 / 0.378
+// vs 0.346 ms), so WOR = 8 is not built.
 template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0, bool BX = false, int WOR = 0>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
     if (*(volatile const int *)p.stop) return;
@@ -1329,24 +1334,14 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 if (sl < nsl && loc < nrows) ya[loc] = xj[h];
                 bb += bi[h] * bi[h];
             };
-            if constexpr (WOR <= 4) {
-                // both rows' gathers in flight together (one gather latency per subdomain instead
-                // of two); the local entries after the sums, so the gathered values and the
-                // local entries are never live at once (64 registers)
-                stage_a(0);
-                stage_a(1);
-                stage_c(0);
-                stage_c(1);
-                stage_b(0);
-                stage_b(1);
-            } else {  // one row at a time, its local entries loaded while its gathers fly
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    stage_a(h);
-                    stage_b(h);
-                    stage_c(h);
-                }
-            }
+            // both rows' gathers in flight together; the local entries after the sums, so the
+            // gathered values and the local entries are never live at once (64 registers)
+            stage_a(0);
+            stage_a(1);
+            stage_c(0);
+            stage_c(1);
+            stage_b(0);
+            stage_b(1);
         } else
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
@@ -2450,27 +2445,26 @@ cudaError_t launch_pipe_t(const KP &p, const Layout &L, size_t smem, cudaStream_
     return cudaGetLastError();
 }
 
-// Name of the coded k_block_duo variant (Layout::last_kernel, bench roofline.kernel): wo4 / wo8 =
-// the unrolled phase 1, bx = b_J, x_J with the slab.
+// Name of the coded k_block_duo variant (Layout::last_kernel, bench roofline.kernel): wo4 = the
+// unrolled phase 1, bx = b_J, x_J with the slab.
 const char *duo_coded_name(bool async, bool bx, int wor) {
-    static const char *names[2][2][3] = {
-        {{"k_block_duo<sync,coded>", "k_block_duo<sync,coded,wo4>", "k_block_duo<sync,coded,wo8>"},
-         {"k_block_duo<sync,coded,bx>", "k_block_duo<sync,coded,wo4,bx>", "k_block_duo<sync,coded,wo8,bx>"}},
-        {{"k_block_duo<async,coded>", "k_block_duo<async,coded,wo4>", "k_block_duo<async,coded,wo8>"},
-         {"k_block_duo<async,coded,bx>", "k_block_duo<async,coded,wo4,bx>", "k_block_duo<async,coded,wo8,bx>"}}};
-    return names[async][bx][wor == 0 ? 0 : wor == 4 ? 1 : 2];
+    static const char *names[2][2][2] = {
+        {{"k_block_duo<sync,coded>", "k_block_duo<sync,coded,wo4>"},
+         {"k_block_duo<sync,coded,bx>", "k_block_duo<sync,coded,wo4,bx>"}},
+        {{"k_block_duo<async,coded>", "k_block_duo<async,coded,wo4>"},
+         {"k_block_duo<async,coded,bx>", "k_block_duo<async,coded,wo4,bx>"}}};
+    return names[async][bx][wor == 4 ? 1 : 0];
 }
 
 template <bool ASYNC, int WLR>
 cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t st, size_t smem_bx = 0) {
     const bool ext = p.frozen != nullptr || p.tau != 1.0;
     const int coded = p.codes == nullptr ? 0 : (p.sdict != nullptr ? 2 : 1);
-    // unrolled phase 1 (WOR) for the coded layouts with <= 4 / <= 8 off-block entries per row
-    const int wor = coded == 1 && !ext && L.tune.unroll_off >= 0 ? (L.max_wo <= 4 ? 4 : (L.max_wo <= 8 ? 8 : 0)) : 0;
+    // unrolled phase 1 (WOR) for the coded layouts with <= 4 off-block entries per row
+    const int wor = coded == 1 && !ext && L.tune.unroll_off >= 0 && L.max_wo <= 4 ? 4 : 0;
     auto kfn = coded == 2 ? (ext ? k_block_duo<ASYNC, WLR, true, 2> : k_block_duo<ASYNC, WLR, false, 2>)
                : coded == 1 ? (ext ? k_block_duo<ASYNC, WLR, true, 1>
                                : wor == 4 ? k_block_duo<ASYNC, WLR, false, 1, false, 4>
-                               : wor == 8 ? k_block_duo<ASYNC, WLR, false, 1, false, 8>
                                           : k_block_duo<ASYNC, WLR, false, 1>)
                             : (ext ? k_block_duo<ASYNC, WLR, true, 0> : k_block_duo<ASYNC, WLR, false, 0>);
     const int threads = L.spb / 2 * kSlice;
@@ -2481,7 +2475,7 @@ cudaError_t launch_duo_t(const KP &p, const Layout &L, size_t smem, cudaStream_t
     // b_J / x_J staged with the slab (coded layout, no EXT) where that keeps the blocks per SM
     if (smem_bx > 0 && coded == 1 && !ext) {
         auto kbx = wor == 4 ? k_block_duo<ASYNC, WLR, false, 1, true, 4>
-                   : wor == 8 ? k_block_duo<ASYNC, WLR, false, 1, true, 8> : k_block_duo<ASYNC, WLR, false, 1, true>;
+                   : k_block_duo<ASYNC, WLR, false, 1, true>;
         if (ensure_smem(kbx, smem_bx) == cudaSuccess && occupancy(kbx, threads, smem_bx) >= occ) {
             L.last_kernel = duo_coded_name(ASYNC, true, wor);
             const int64_t g = persistent_grid(occ, p, L);

@@ -94,7 +94,7 @@ def libbar_name(ncu_name):
         return ncu_name
     a = [int(re.sub(r"\(\w+\)", "", t).strip()) for t in m.group(1).split(",")]
     a += [0] * (6 - len(a))
-    wo = "" if a[5] == 0 else f",wo{a[5]}"
+    wo = "" if a[5] == 0 else f",wo{a[5]}"  # WOR
     return ("k_block_duo<" + ("async" if a[0] else "sync") + {0: "", 1: ",coded", 2: ",staged"}[a[3]]
             + wo + {0: "", 1: ",bx", 2: ",x"}[a[4]] + ">")
 
