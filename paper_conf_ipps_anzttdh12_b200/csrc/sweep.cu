@@ -1048,12 +1048,18 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // Subdomains are claimed statically (claims_of: round robin or contiguous chunks).
 // Phase timing of k_block_duo (a profiling build only: -DBAR_PROFILE_DUO, tools/duo_phase_probe.py):
 // lane 0 of warps 0 (slab issuer), 3 (b/x, ring and prefetch issuer) and nw - 1 (rows only) sums
-// clock64 deltas between the marks over the launch; added into g_duo_prof[3][8] at the end.
+// clock64 deltas between the marks over the launch; added into g_duo_prof[0..2][8] at the end.
+// Row 3 (thread 0): [0] sum and [1] max over blocks of the block's %globaltimer span (ns) from
+// kernel entry to the end of its last subdomain, [2] the latest end, [3] the earliest entry
+// (ns, against ~0 initial values: min via atomicMin on ~end), [4] blocks.
 #ifdef BAR_PROFILE_DUO
-__device__ unsigned long long g_duo_prof[3][8];
+__device__ unsigned long long g_duo_prof[4][8];
 #define DUO_PROF_DECL                                                                         \
     const int prof_w = warp == 0 ? 0 : warp == 3 ? 1 : warp == nw - 1 ? 2 : -1;              \
     long long prof_t[8] = {0, 0, 0, 0, 0, 0, 0, 0}, prof_last = clock64();
+#define DUO_PROF_ENTRY                \
+    unsigned long long prof_t0;       \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
 #define DUO_PROF_MARK(i)                         \
     if (prof_w >= 0 && lane == 0) {              \
         const long long now = clock64();         \
@@ -1062,8 +1068,18 @@ __device__ unsigned long long g_duo_prof[3][8];
     }
 #define DUO_PROF_FLUSH                                                                          \
     if (prof_w >= 0 && lane == 0)                                                               \
-        for (int i = 0; i < 8; ++i) atomicAdd(&g_duo_prof[prof_w][i], (unsigned long long)prof_t[i]);
+        for (int i = 0; i < 8; ++i) atomicAdd(&g_duo_prof[prof_w][i], (unsigned long long)prof_t[i]); \
+    if (threadIdx.x == 0) {                                                                     \
+        unsigned long long t_end;                                                               \
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));                               \
+        atomicAdd(&g_duo_prof[3][0], t_end - prof_t0);                                          \
+        atomicMax(&g_duo_prof[3][1], t_end - prof_t0);                                          \
+        atomicMax(&g_duo_prof[3][2], t_end);                                                    \
+        atomicMax(&g_duo_prof[3][3], ~prof_t0);                                                 \
+        atomicAdd(&g_duo_prof[3][4], 1ull);                                                     \
+    }
 #else
+#define DUO_PROF_ENTRY
 #define DUO_PROF_DECL
 #define DUO_PROF_MARK(i)
 #define DUO_PROF_FLUSH
@@ -1112,6 +1128,7 @@ __host__ __device__ __forceinline__ DuoGeom duo_geom(int R, int spb, int wmax, b
 // vs 0.346 ms), so WOR = 8 is not built.
 template <bool ASYNC, int WLR, bool EXT = false, int CODED = 0, bool BX = false, int WOR = 0>
 __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
+    DUO_PROF_ENTRY
     if (*(volatile const int *)p.stop) return;
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ __align__(8) uint64_t bar;
@@ -2889,10 +2906,10 @@ cudaError_t launch_init_state(DevState *state, double tol, cudaStream_t st) {
 }  // namespace bar
 
 #ifdef BAR_PROFILE_DUO
-extern "C" int bar_debug_duo_profile(unsigned long long *out24, int reset) {
-    cudaMemcpyFromSymbol(out24, bar::g_duo_prof, sizeof(unsigned long long) * 24);
+extern "C" int bar_debug_duo_profile(unsigned long long *out32, int reset) {
+    cudaMemcpyFromSymbol(out32, bar::g_duo_prof, sizeof(unsigned long long) * 32);
     if (reset) {
-        unsigned long long z[24] = {};
+        unsigned long long z[32] = {};
         cudaMemcpyToSymbol(bar::g_duo_prof, z, sizeof(z));
     }
     return (int)cudaGetLastError();

@@ -125,5 +125,6 @@ if __name__ == "__main__":
         build_bar(True, "libbar_prof.so", ("BAR_PROFILE_RESIDENT=1",))
     elif "--profile-duo" in sys.argv:
         build_bar(True, "libbar_duoprof.so", ("BAR_PROFILE_DUO=1",))
+
     else:
         build_all(force="--force" in sys.argv)

@@ -42,11 +42,19 @@ def main():
     x = torch.zeros(M.n, dtype=torch.float64, device="cuda")
     M.sweep(b, x, k=a.k, nsweeps=3, mode=a.mode)
     torch.cuda.synchronize()
-    out = (ctypes.c_ulonglong * 24)()
+    out = (ctypes.c_ulonglong * 32)()
     bar._lib.bar_debug_duo_profile(out, 1)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
     M.sweep(b, x, k=a.k, nsweeps=a.sweeps, mode=a.mode)
+    e1.record()
     torch.cuda.synchronize()
     bar._lib.bar_debug_duo_profile(out, 1)
+    ms = e0.elapsed_time(e1) / a.sweeps
+    nb = out[28]
+    span_avg = out[24] / max(nb, 1) / 1e3  # us per block per launch (summed over launches)
+    print(f"  launch {ms * 1e3:.1f} us (events); blocks {nb // a.sweeps} per launch; block span avg "
+          f"{span_avg / a.sweeps * a.sweeps:.1f} us (entry to exit, per launch), max {out[25] / 1e3:.1f} us")
     q = M.info()["num_subdomains"]
     print(f"{a.workload} {a.mode} k={a.k} kernel={M.info()['last_sweep_kernel']} tune={tune}: cycles per subdomain")
     for w, name in enumerate(["warp 0", "warp 3", "last warp"]):
