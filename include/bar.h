@@ -218,7 +218,7 @@ typedef struct {
     int32_t async_queue;    /* 0 static claims, 1 device work-queue claims (k_block_stage)       */
     int32_t resident;       /* 0 auto, -1 never use the block-owns-subdomain single-launch kernel */
     int32_t lead;           /* k_block_resident: max sweeps a block may lead the last completed
-                               global iteration (0 = default 3; 1..48)                           */
+                               global iteration (0 = default 48, the residual ring's bound; 1..48) */
     int32_t ghost_prefetch; /* L2 bulk prefetch of the gather ranges: 0 auto (R >= 512), 1, -1   */
     int32_t graph;          /* single-launch async: 0 capture + replay as a CUDA graph, -1 never  */
     int32_t single_launch;  /* async: 0 auto (one launch for all iterations when one iteration

@@ -2524,10 +2524,14 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     // resident, the kernel aborts and the host continues with per-launch kernels: DESIGN.md R12)
     if ((int64_t)occupancy(k_block_resident<WLR>, threads, smem) * L.sms < L.q) return false;
     L.last_kernel = "k_block_resident<async>";
-    // lead 3 (B200, round 1, tools/kernel_ab.py): C2 51 vs 56-59 global iterations with lead 40
-    // (0.29 vs 0.33 ms), C3 0.205 vs 0.217 ms; blocks racing far ahead sweep on stale ghosts
+    // lead: 48 by default, the loosest bound the residual ring allows (kSlots = 64 slots), i.e. as
+    // close to "no inter-block synchronisation" as the bookkeeping gets. Round 1 measured lead 3
+    // ahead (C2 51 vs 56-59 iterations with lead 40); with the lazy publication of round 2 the
+    // bound no longer matters (B200, tools/kernel_ab.py, medians of 3 x 41 solves, lead 3 / 8 /
+    // 16 / 48: C1 0.157 / 0.157 / 0.157 / 0.157 ms with 29 / 28 / 28 / 28 iterations, C2 0.220 /
+    // 0.219 / 0.219 / 0.221 ms with 52 / 53 / 53 / 53, C3 0.182 / 0.182 / 0.181 / 0.181 ms, 27)
     KP pp = p;
-    pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 3;
+    pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 48;
     if (p.ring && L.tune.lazy_publish >= 0) {
         if (ensure_smem(k_block_resident<WLR, true>, smem) != cudaSuccess) {
             cudaGetLastError();

@@ -47,7 +47,7 @@ def test_our_arm_line(bar):
     assert c["kind"] == "oracle" and c["cores"] == 1 and c["value"] > 0 and c["sample"]
     assert c["jacobi"]["iters"] == 137 and c["gauss_seidel"]["iters"] == 14  # SURVEY P12 counts
     assert c["sync_block_5"]["iters"] == 28 and d["oracle_iters"] == 28 and not c["extrapolated"]
-    assert d["partitioned_1rank"]["converged"] and d["lead_48"]["global_iters"] > 0
+    assert d["partitioned_1rank"]["converged"] and d["lead_3"]["global_iters"] > 0
     e = d["e2e"]
     assert e["h2d_bytes_per_step"] == 8 * 2000 and e["d2h_bytes_per_step"] == 8 * 2000 and e["value"] > 0
     assert d["clocks"]["sm_max_mhz"]

@@ -377,7 +377,7 @@ def test_siam_constant_async(bar, golden):
 @pytest.mark.parametrize("tune", [{"kernel": "block"}, {"kernel": "reg"}, {"kernel": "reg_tma"}, {"kernel": "pers"},
                                   {"pipe": 1}, {"pipe": -1}, {"jacobi_rowwise": 1}, {"single_launch": 1},
                                   {"single_launch": -1}, {"ghost_prefetch": -1}, {"ghost_prefetch": 1},
-                                  {"async_queue": "queue"}, {"resident": -1}, {"lead": 48}, {"graph": -1}])
+                                  {"async_queue": "queue"}, {"resident": -1}, {"lead": 3}, {"graph": -1}])
 @pytest.mark.parametrize("name,R", [("fv1", 128), ("s7_m12", 288), ("tref2000", 128), ("s7_m12", 512),
                                     ("rand", 1024)])
 def test_forced_kernel_paths(bar, tune, name, R):

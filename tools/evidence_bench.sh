@@ -11,7 +11,7 @@ for m in sync-block jacobi; do
   timeout 600 python bench.py --mode $m --no-dist > $OUT/bench_c5_$m.json 2> $OUT/bench_c5_$m.err
 done
 for wl in c4 c3 c2 c1; do
-  timeout 600 python bench.py --workload $wl > $OUT/bench_${wl}_async.json 2> $OUT/bench_${wl}_async.err
+  timeout 600 python bench.py --workload $wl $( [ $wl = c4 ] || echo "--steps 50 --warmup 5" ) > $OUT/bench_${wl}_async.json 2> $OUT/bench_${wl}_async.err
 done
 timeout 900 python bench.py --impl reference > $OUT/bench_reference_c5.json 2> $OUT/bench_reference_c5.err
 for f in $OUT/bench_*.json; do echo "$f: $(tail -c 300 $f | head -c 300)"; done | cut -c1-200

@@ -26,6 +26,6 @@ timeout 900 python tools/local_iters.py --workload c5 > $OUT/n4_c5.txt 2>&1
 timeout 900 python tools/local_iters.py --workload c4 > $OUT/n4_c4.txt 2>&1
 timeout 900 python tools/local_iters.py --workload c2 > $OUT/n4_c2.txt 2>&1
 timeout 900 python tools/nondeterminism.py --workload c1 --runs 200 > $OUT/n2_c1.txt 2>&1
-timeout 900 python tools/nondeterminism.py --workload c1 --runs 200 --lead 48 > $OUT/n2_c1_lead48.txt 2>&1
+timeout 900 python tools/nondeterminism.py --workload c1 --runs 200 --lead 3 > $OUT/n2_c1_lead3.txt 2>&1
 timeout 900 python tools/nondeterminism.py --workload c2 --runs 100 > $OUT/n2_c2.txt 2>&1
 ls -la $OUT | tail -30

@@ -48,7 +48,7 @@ def main():
     ap.add_argument("--k", type=int, default=5)
     ap.add_argument("--R", type=int, default=128)
     ap.add_argument("--single-launch", type=int, default=-1, help="-1 auto, 0 per-launch, 1 single launch")
-    ap.add_argument("--lead", type=int, default=0, help="single-launch kernel's lead bound (0 = default 3)")
+    ap.add_argument("--lead", type=int, default=0, help="single-launch kernel's lead bound (0 = default 48)")
     a = ap.parse_args()
     from conftest import load_golden
 
@@ -57,7 +57,7 @@ def main():
     name, rows = table(a.workload, a.runs, a.k, a.R, a.single_launch, tuning={"lead": a.lead} if a.lead else None)
     clk = os.popen("nvidia-smi --query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active --format=csv,noheader")
     print(f"# N2: async-({a.k}), R={a.R}, {name}, b=1, x0=0, {a.runs} runs per checkpoint, exact residuals;"
-          f" lead {a.lead or 3}; clocks after the run: {clk.read().strip()}")
+          f" lead {a.lead or 48}; clocks after the run: {clk.read().strip()}")
     print(f"# paper column: the 1000-run average of {tab} (C2070; fv1 there is the real fv1, here the "
           f"pattern-exact synthetic)")
     print(f"{'iters':>5} {'avg':>11} {'max':>11} {'min':>11} {'abs.var':>10} {'rel.var':>10} {'variance':>10} "
