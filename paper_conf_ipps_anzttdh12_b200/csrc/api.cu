@@ -432,8 +432,13 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         if ((r = ensure_buf(&W.stage_x, n)) != BAR_OK) return r;
         buf0 = W.stage_x;
     }
+    // the single-launch async path enqueues the zero start and the state reset with its first
+    // pass (inside the replayed graph: two API launches fewer per solve)
+    bool async_multi = mode == BAR_MODE_ASYNC && use_async_multi(L);
+    if (opts && opts->async_single_launch >= 0) async_multi = mode == BAR_MODE_ASYNC && opts->async_single_launch == 1;
+    async_multi = async_multi && !ext_opts && max_global_iters > 0;
     if (x0 == nullptr) {
-        BAR_CUDA(cudaMemsetAsync(buf0, 0, bytes, st));
+        if (!async_multi) BAR_CUDA(cudaMemsetAsync(buf0, 0, bytes, st));
     } else if (x0 != x || !x_dev) {
         BAR_CUDA(cudaMemcpyAsync(buf0, x0, bytes, cudaMemcpyDefault, st));
     }
@@ -442,7 +447,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         if ((r = ensure_buf(&W.xbuf, n)) != BAR_OK) return r;
         buf1 = W.xbuf;
     }
-    BAR_CUDA(launch_init_state(W.state, tol, st));
+    if (!async_multi) BAR_CUDA(launch_init_state(W.state, tol, st));
     ++launches;
 
     DevState &H = *W.h_state;
@@ -501,10 +506,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
         }
     } else {
         // async-(k): in place on buf0. Check x^(0) first (exact), then iterate.
-        bool multi = use_async_multi(L);
-        if (opts && opts->async_single_launch >= 0) multi = opts->async_single_launch == 1;
-        if (ext_opts) multi = false;
-        multi = multi && max_global_iters > 0;
+        bool multi = async_multi;
         // the single-launch path decides the x^(0) check on the device (k_init_check), so the
         // x^(0) residual, the solve and the confirming residual need ONE host round trip
         auto apply_init = [&](double r0) {
@@ -570,9 +572,12 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             T.used = 0;
             cudaEvent_t ev0 = T.ev[0], ev1 = T.ev[1];
             auto enqueue_first = [&](cudaStream_t s) -> cudaError_t {
+                cudaError_t e = cudaSuccess;
+                if (x0 == nullptr && (e = cudaMemsetAsync(buf0, 0, bytes, s)) != cudaSuccess) return e;
+                if ((e = launch_init_state(W.state, tol, s)) != cudaSuccess) return e;
                 // the residual kernel's last block applies the x^(0) check (k_init_check's rule)
-                cudaError_t e = x0 == nullptr ? launch_zero_start_residual(L, db, W.state, W.partials, s, true)
-                                              : launch_residual(L, db, buf0, W.state, W.partials, s, nullptr, true);
+                e = x0 == nullptr ? launch_zero_start_residual(L, db, W.state, W.partials, s, true)
+                                  : launch_residual(L, db, buf0, W.state, W.partials, s, nullptr, true);
                 if (e != cudaSuccess) return e;
                 if ((e = cudaEventRecord(ev0, s)) != cudaSuccess) return e;
                 SweepArgs a{&L, db, buf0, buf0, k, W.state, W.partials, nullptr};
