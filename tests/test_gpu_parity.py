@@ -618,3 +618,63 @@ def test_duo_slab_staging_and_buffer_rotation(bar, name, gen, R, stage_bx, grid_
         assert not staged, kernels
     elif name == "s7_m128":  # C5's geometry (R = two grid lines): the staged variant keeps two blocks per SM
         assert staged, kernels
+
+
+def _banded_random(n, band, per_row, seed):
+    """Seeded banded random matrix: per row the diagonal plus `per_row` distinct offsets in
+    [-band, band] (clipped at the matrix edges), off-diagonals uniform in [-1, -0.1], diagonal
+    1.5 x the row's absolute off-diagonal sum (rho(|B|) <= 2/3). Few distinct column offsets per
+    subdomain (coded columns) with random values and a ragged pattern near the subdomain edges."""
+    rng = np.random.default_rng(seed)
+    offs = np.array([d for d in range(-band, band + 1) if d != 0])
+    pick = np.argsort(rng.random((n, offs.size)), axis=1)[:, :per_row]
+    d = np.sort(offs[pick], axis=1)
+    rows = np.arange(n)[:, None]
+    c = rows + d
+    ok = (c >= 0) & (c < n)
+    v = -rng.uniform(0.1, 1.0, size=d.shape)
+    v[~ok] = 0.0
+    diag = 1.5 * np.abs(v).sum(axis=1) + 1.0
+    cols = np.concatenate([np.where(ok, c, -1), rows], axis=1)
+    vals = np.concatenate([v, diag[:, None]], axis=1)
+    order = np.argsort(cols, axis=1, kind="stable")
+    cols = np.take_along_axis(cols, order, axis=1)
+    vals = np.take_along_axis(vals, order, axis=1)
+    keep = cols >= 0
+    counts = keep.sum(axis=1)
+    rowptr = np.zeros(n + 1, dtype=np.int32)
+    rowptr[1:] = np.cumsum(counts)
+    return W.CSR(n, rowptr, cols[keep].astype(np.int32), vals[keep].astype(np.float64), name=f"banded_{n}_{seed}")
+
+
+@pytest.mark.parametrize("n,R,seed", [(1_000_123, 256, 1), (1_000_123, 512, 2), (700_001, 1024, 3)])
+@pytest.mark.parametrize("unroll_off", [0, -1])
+def test_duo_unrolled_random_banded(bar, n, R, seed, unroll_off):
+    """The two-blocks-per-SM kernel's unrolled phase 1 (<= 4 off-block entries per row, coded
+    columns; `wo4` in the kernel name) against the generic loop (-1) on random banded matrices:
+    random values (not a stencil's constant coefficients), rows with 0-3 off-block entries in any
+    position, a partial last subdomain and partial last slice (n not a multiple of R or 32).
+    Sync-block-(k) for k = 1, 3, 5 and Jacobi match the oracle to 1e-12 after 2 iterations;
+    async-(5) meets the exact residual."""
+    import torch
+
+    A = _banded_random(n, 60, 3, seed)  # <= 4 local entries (the duo kernel), <= 3 off-block
+    b = np.random.default_rng(seed + 100).uniform(0.5, 1.5, n)
+    x0 = np.random.default_rng(seed + 200).uniform(-1, 1, n)
+    M = bar.Matrix.from_csr(A, R, tuning={"duo": 1, "single_launch": -1, "unroll_off": unroll_off})
+    assert M.info()["coded"] == 1
+    kernels = set()
+    for mode, k in (("sync-block", 5), ("sync-block", 3), ("sync-block", 1), ("jacobi", 1)):
+        ref = x0
+        for _ in range(2):
+            ref = O.jacobi_step(A, b, ref) if mode == "jacobi" else O.block_jacobi_step(A, b, ref, R, k)
+        x = torch.empty(n, dtype=torch.float64, device="cuda")
+        M.solve(_dev(b), _dev(x0), x, k=k, max_global_iters=2, tol=0.0, mode=mode)
+        kernels.add(M.info()["last_sweep_kernel"])
+        _close(x.cpu().numpy(), ref)
+    x, info = M.solve(_dev(b), None, None, k=5, tol=1e-10, mode="async")
+    kernels.add(M.info()["last_sweep_kernel"])
+    assert info["converged"] and O.rel_res(A, b, x.cpu().numpy()) <= 1e-10 * (1 + 1e-6)
+    M.close()
+    assert all(kn.startswith("k_block_duo<") for kn in kernels), kernels
+    assert all((",wo4" in kn) == (unroll_off == 0) for kn in kernels), kernels
