@@ -334,6 +334,14 @@ def main():
     if multi:
         import torch.distributed as dist
 
+        if "RANK" not in os.environ:  # --dist-path without torchrun: a 1-rank group on 127.0.0.1
+            import socket
+
+            with socket.socket() as so:
+                so.bind(("127.0.0.1", 0))
+                port = so.getsockname()[1]
+            os.environ.update(RANK="0", WORLD_SIZE="1", LOCAL_RANK="0", MASTER_ADDR="127.0.0.1",
+                              MASTER_PORT=str(port))
         dist.init_process_group("nccl", device_id=dev)
     from paper_conf_ipps_anzttdh12_b200 import bar
 

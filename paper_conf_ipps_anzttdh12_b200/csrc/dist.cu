@@ -1428,7 +1428,9 @@ bar_status bar_create_csr_dist(int64_t n_global, int64_t row_begin, int64_t row_
             // IPC handles of every rank's iterate and board, and owned-block offsets
             std::vector<unsigned char> mine(136, 0);
             int64_t off = 0;
-            st = bar_dist_p2p_handles(D, mine.data(), &off);
+            // (an export failure only disables peer memory: every rank still joins the gather)
+            const bool exported = bar_dist_p2p_handles(D, mine.data(), &off) == BAR_OK;
+            cudaGetLastError();
             std::memcpy(mine.data() + 128, &off, 8);
             unsigned char *dh = nullptr;
             if (st == BAR_OK && cudaMalloc(&dh, 136 * (size_t)(P + 1)) != cudaSuccess)
@@ -1449,7 +1451,27 @@ bar_status bar_create_csr_dist(int64_t n_global, int64_t row_begin, int64_t row_
                     std::memcpy(handles.data() + 128 * (size_t)p, all.data() + 136 * (size_t)p, 128);
                     std::memcpy(&offs[p], all.data() + 136 * (size_t)p + 128, 8);
                 }
-                st = enable_p2p(D, gsrc.data(), handles.data(), offs.data());
+                // a rank that cannot map its peers (IPC refused) is not an error of the solve: all
+                // ranks agree (min all-reduce) and, if any failed, unmap and keep the collective
+                // NCCL path for async as well
+                int mapped = exported && enable_p2p(D, gsrc.data(), handles.data(), offs.data()) == BAR_OK ? 1 : 0;
+                cudaGetLastError();
+                int *dm = nullptr;
+                if (cudaMalloc(&dm, sizeof(int)) != cudaSuccess) st = cuda_fail(cudaGetLastError(), "cudaMalloc");
+                if (st == BAR_OK) {
+                    cudaMemcpy(dm, &mapped, sizeof(int), cudaMemcpyHostToDevice);
+                    ncclResult_t rr = ncclAllReduce(dm, dm, 1, ncclInt32, ncclMin, comm, s);
+                    if (rr != ncclSuccess) st = nccl_fail((int)rr, "ncclAllReduce");
+                    else if (cudaMemcpy(&mapped, dm, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess)
+                        st = cuda_fail(cudaGetLastError(), "cudaMemcpy");
+                }
+                cudaFree(dm);
+                if (st == BAR_OK && !mapped) {
+                    for (void *q : D->opened) cudaIpcCloseMemHandle(q);
+                    D->opened.clear();
+                    D->p2p = false;
+                    cudaGetLastError();
+                }
             }
         }
     }
