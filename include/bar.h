@@ -243,6 +243,8 @@ typedef struct {
     int32_t unroll_off;     /* k_block_duo, coded columns: 0 phase 1 unrolled where a row has <= 4
                                off-block entries (both rows' gathers in flight), -1 the generic
                                loop                                                              */
+    int32_t fuse_residual;  /* k_block_resident: 0 the confirming residual computed at the end of
+                               the single launch (grid barrier), -1 a separate residual kernel    */
 } bar_tuning;
 
 /* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a

@@ -247,7 +247,8 @@ bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning) {
     if (tuning) t = *tuning;
     if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 3 || t.fronts < 0 || t.async_queue < 0 ||
         t.async_queue > 1 || t.lead < 0 || t.lead > 48 || t.grid_cap < 0 || t.warps < 0 || t.warps > 32 ||
-        t.halo < 0 || t.halo > 1 || t.peer > 0 || t.coded > 2 || t.overlap > 0 || t.unroll_off > 0) {
+        t.halo < 0 || t.halo > 1 || t.peer > 0 || t.coded > 2 || t.overlap > 0 || t.unroll_off > 0 ||
+        t.fuse_residual > 0) {
         set_error("bar_tuning field out of range");
         return BAR_ERR_INVALID_ARG;
     }
@@ -571,6 +572,11 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             if ((r = timer_begin(T, 1, st)) != BAR_OK) return r;  // creates the events
             T.used = 0;
             cudaEvent_t ev0 = T.ev[0], ev1 = T.ev[1];
+            // k_block_resident with the lazy publication computes the confirming residual itself
+            // (sweep.cu, KP::fuse_residual): no residual kernel in the first pass
+            auto fused_now = [&]() {
+                return static_multi(L.last_kernel) && W.ring && L.tune.lazy_publish >= 0 && L.tune.fuse_residual >= 0;
+            };
             auto enqueue_first = [&](cudaStream_t s) -> cudaError_t {
                 cudaError_t e = cudaSuccess;
                 if (x0 == nullptr && (e = cudaMemsetAsync(buf0, 0, bytes, s)) != cudaSuccess) return e;
@@ -585,7 +591,7 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
                 a.bsum_arr = W.bsum_arr;
                 if ((e = launch_async_multi(a, w_end, s)) != cudaSuccess) return e;
                 if ((e = cudaEventRecord(ev1, s)) != cudaSuccess) return e;
-                if ((e = launch_residual(L, db, buf0, W.state, W.partials, s)) != cudaSuccess) return e;
+                if (!fused_now() && (e = launch_residual(L, db, buf0, W.state, W.partials, s)) != cudaSuccess) return e;
                 return cudaMemcpyAsync(W.h_state, W.state, sizeof(DevState), cudaMemcpyDeviceToHost, s);
             };
             SolveGraph &Gr = W.graph;
@@ -624,6 +630,14 @@ bar_status bar_solve_ex(bar_matrix A, const double *b, const double *x0, double 
             } else {
                 BAR_CUDA(e);
                 BAR_CUDA(cudaStreamSynchronize(st));
+                if (fused_now()) {
+                    --launches;
+                    if (!H.exact_fused) {  // the fused pass gave up (blocks not co-resident): the kernel
+                        BAR_CUDA(launch_residual(L, db, buf0, W.state, W.partials, st));
+                        ++launches;
+                        if ((r = read_state(A, st)) != BAR_OK) return r;
+                    }
+                }
                 // kernel time from the events, or (graph replay) from the kernel's own timestamps
                 T.m[0] = 1;
                 T.used = use_graph ? 0 : 1;

@@ -67,6 +67,10 @@ struct DevState {
     unsigned long long t_first, t_last;  // single-launch kernels: %globaltimer (ns) of the first
                                          // block start and the last block exit (graph replays
                                          // cannot time their kernel with host-visible events)
+    // k_block_resident's fused exact residual of the returned iterate (KP::fuse_residual): blocks
+    // arrived at the final grid barrier, reduction ticket, and whether exact_rel was produced
+    unsigned int fuse_arrive, fuse_ticket;
+    int exact_fused;
 };
 constexpr int kSlots = 64;
 

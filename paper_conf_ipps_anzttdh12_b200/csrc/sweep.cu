@@ -62,6 +62,7 @@ struct KP {
     int64_t l_begin, l_end; // subdomains this launch sweeps (l_end = 0: all; k_block_duo / _pipe only)
     const int *stop;        // the stop flag the kernels poll at start (default &state->stop)
     int slab_ahead;         // k_block_duo: L2 bulk prefetch of the slab two subdomains ahead
+    int fuse_residual;      // k_block_resident<LAZY>: exact residual of the final x at the end of the launch
     double *ring;           // k_block_resident<LAZY>: [kSlots][q] per-block residual partials
     double *bsum_arr;       //   and [q] per-block sums of b_i^2
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
@@ -2176,10 +2177,95 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         BAR_PROF_MARK(5)
         ++m;
     }
-    if (threadIdx.x == 0) {
-        atomicAdd(&p.state->res_sweeps, sweeps);
-        stamp_last(p.state);
+    if (threadIdx.x == 0) atomicAdd(&p.state->res_sweeps, sweeps);
+    // The exact residual ||b - A x||_2 of the iterate the solve returns (a5, the confirming
+    // residual of a7), fused: once every block has stopped sweeping (a grid barrier — all q blocks
+    // are co-resident; bounded by ~2 ms of %globaltimer like the lead wait, after which the host
+    // runs the residual kernel instead), each block forms r_i = b_i - sum_j a_ij x_j for its rows
+    // from the matrix entries it already holds (off-block x as written, x_J from shared memory),
+    // and the last block sums the q partials in block order (own ticket and ring row 0, so a
+    // partial pass leaves the residual kernel's state untouched).
+    if (LAZY && p.fuse_residual) {
+        __shared__ int fuse_go;
+        if (threadIdx.x == 0) {
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&p.state->fuse_arrive) : "memory");
+            const unsigned long long t0c = globaltimer_ns();
+            int okb = 1;
+            for (;;) {
+                unsigned int a;
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(a) : "l"(&p.state->fuse_arrive) : "memory");
+                if (a >= (unsigned int)q) break;
+                if (globaltimer_ns() - t0c > 2000000ull) {
+                    okb = 0;
+                    break;
+                }
+            }
+            fuse_go = okb && !*(volatile int *)&p.state->aborted;
+        }
+        __syncthreads();
+        if (fuse_go) {
+            double r2 = 0.0;
+            if (ok) {
+                double s = bi;
+                for (int e0 = 0; e0 < wo; e0 += 2 * U) {
+                    double xv[2 * U];
+#pragma unroll
+                    for (int u = 0; u < 2 * U; ++u)
+                        if (e0 + u < wo) xv[u] = ldx<true>(p.x_in + oc[ooff + (e0 + u) * kSlice]);
+#pragma unroll
+                    for (int u = 0; u < 2 * U; ++u)
+                        if (e0 + u < wo) s -= ov[ooff + (e0 + u) * kSlice] * xv[u];
+                }
+                const double *yf = ybuf(cur);
+#pragma unroll
+                for (int e = 0; e < WLR; ++e) s -= lv[e] * yf[(lc[e >> 1] >> (16 * (e & 1))) & 0xffff];
+                r2 = s * s;
+            }
+            const double wr = warp_sum(r2);
+            if (lane == 0) sred[0][warp] = wr;
+            __syncthreads();
+            __shared__ bool fuse_last;
+            if (threadIdx.x == 0) {
+                const int W = blockDim.x >> 5;
+                double a0 = 0.0;
+                for (int w = 0; w < W; ++w) a0 += sred[0][w];
+                asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.ring + blockIdx.x), "d"(a0) : "memory");
+                unsigned int tk;
+                asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(tk) : "l"(&p.state->fuse_ticket) : "memory");
+                fuse_last = tk == (unsigned int)q - 1;
+            }
+            __syncthreads();
+            if (fuse_last) {
+                double s0 = 0.0, s1 = 0.0;
+                for (int64_t i = threadIdx.x; i < q; i += blockDim.x) {
+                    double v0, v1;
+                    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v0) : "l"(p.ring + i) : "memory");
+                    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v1) : "l"(p.bsum_arr + i) : "memory");
+                    s0 += v0;
+                    s1 += v1;
+                }
+                s0 = warp_sum(s0);
+                s1 = warp_sum(s1);
+                __syncthreads();
+                if (lane == 0) {
+                    sred[0][warp] = s0;
+                    sred[1][warp] = s1;
+                }
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    const int W = blockDim.x >> 5;
+                    double ss = 0.0, bsq = 0.0;
+                    for (int w = 0; w < W; ++w) {
+                        ss += sred[0][w];
+                        bsq += sred[1][w];
+                    }
+                    apply_stop_rule(p.state, ss, bsq, true, nullptr);
+                    p.state->exact_fused = 1;
+                }
+            }
+        }
     }
+    if (threadIdx.x == 0) stamp_last(p.state);
     BAR_PROF_FLUSH
 }
 
@@ -2305,6 +2391,9 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->res_sweeps = 0;
     S->t_first = ~0ull;
     S->t_last = 0;
+    S->fuse_arrive = 0;
+    S->fuse_ticket = 0;
+    S->exact_fused = 0;
     for (int i = 0; i < kSlots; ++i) {
         S->done[i] = 0;
         S->ss[i] = 0.0;
@@ -2532,6 +2621,7 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     // 0.219 / 0.219 / 0.221 ms with 52 / 53 / 53 / 53, C3 0.182 / 0.182 / 0.181 / 0.181 ms, 27)
     KP pp = p;
     pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 48;
+    pp.fuse_residual = p.ring && L.tune.lazy_publish >= 0 && L.tune.fuse_residual >= 0;
     if (p.ring && L.tune.lazy_publish >= 0) {
         if (ensure_smem(k_block_resident<WLR, true>, smem) != cudaSuccess) {
             cudaGetLastError();
@@ -2852,6 +2942,9 @@ __global__ void k_resume_queue(DevState *S, int clear_slots) {
     if (threadIdx.x == 0) {
         S->stop = 0;
         S->work = S->work_resume;
+        S->fuse_arrive = 0;
+        S->fuse_ticket = 0;
+        S->exact_fused = 0;
     }
 }
 
