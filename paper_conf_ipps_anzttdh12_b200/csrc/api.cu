@@ -47,7 +47,8 @@ bar_status ensure_workspace(bar_matrix A) {
         BAR_CUDA(cudaMemset(W.state, 0, sizeof(DevState)));
     }
     if (!W.ring && L.q <= 8192 && use_async_multi(L)) {  // the single-launch kernel's residual ring
-        BAR_CUDA(cudaMalloc(&W.ring, sizeof(double) * kSlots * (size_t)L.q));
+        BAR_CUDA(cudaMalloc(&W.ring, sizeof(double) * (kSlots + 1) * (size_t)L.q));  // + the fused residual's row
+        BAR_CUDA(cudaMemset(W.ring, 0xFF, sizeof(double) * (kSlots + 1) * (size_t)L.q));  // no tag matches
         BAR_CUDA(cudaMalloc(&W.bsum_arr, sizeof(double) * (size_t)L.q));
     }
     int64_t need = std::max(num_blocks_for(L, BAR_MODE_SYNC_BLOCK), num_blocks_for(L, BAR_MODE_JACOBI));
@@ -248,7 +249,7 @@ bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning) {
     if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 3 || t.fronts < 0 || t.async_queue < 0 ||
         t.async_queue > 1 || t.lead < 0 || t.lead > 48 || t.grid_cap < 0 || t.warps < 0 || t.warps > 32 ||
         t.halo < 0 || t.halo > 1 || t.peer > 0 || t.coded > 2 || t.overlap > 0 || t.unroll_off > 0 ||
-        t.fuse_residual > 0) {
+        t.fuse_residual > 0 || t.lazy_publish > 1) {
         set_error("bar_tuning field out of range");
         return BAR_ERR_INVALID_ARG;
     }

@@ -71,6 +71,8 @@ struct DevState {
     // arrived at the final grid barrier, reduction ticket, and whether exact_rel was produced
     unsigned int fuse_arrive, fuse_ticket;
     int exact_fused;
+    unsigned int epoch;     // bumped by every state reset / resume: tags k_block_resident's tagged
+                            // residual publication (stale ring words of earlier launches never match)
 };
 constexpr int kSlots = 64;
 

@@ -1905,20 +1905,30 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 // barrier that hands the evaluation to the warp): fixed-order sums over the blocks (lane-strided,
 // then the shuffle tree), the stopping rule of iteration_publish, iters_done, and the slot's
 // counter reset for iteration m + kSlots.
-__device__ __noinline__ void lazy_evaluate(const KP &p, long long m, int64_t q, int lane) {
+// TAGGED (q <= 256): the ring words carry the iteration and launch epoch in their 12 low mantissa
+// bits (the partial keeps 40 bits of mantissa, a relative 1e-12 of the estimate); they are summed
+// with the tag cleared, and ||b|| is the one the x^(0) residual stored before the launch.
+template <bool TAGGED>
+__device__ __noinline__ void lazy_evaluate(const KP &p, long long m, int64_t q, int lane, double bnorm0) {
     DevState *S = p.state;
     const int slot = (int)(m % kSlots);
     const double *row = p.ring + (int64_t)slot * q;
     double ss = 0.0, bsq = 0.0;
     for (int64_t c = lane; c < q; c += kSlice) {
-        ss += __ldcg(row + c);
-        bsq += __ldcg(p.bsum_arr + c);
+        if (TAGGED) {
+            unsigned long long w;
+            asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w) : "l"(row + c) : "memory");
+            ss += __longlong_as_double((long long)(w & ~0xFFFull));
+        } else {
+            ss += __ldcg(row + c);
+            bsq += __ldcg(p.bsum_arr + c);
+        }
     }
     ss = warp_sum(ss);
-    bsq = warp_sum(bsq);
+    if (!TAGGED) bsq = warp_sum(bsq);
     if (lane != 0) return;
-    S->done[slot] = 0u;
-    const double bn = sqrt(bsq);
+    if (!TAGGED) S->done[slot] = 0u;
+    const double bn = TAGGED ? bnorm0 : sqrt(bsq);
     const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
     atomicMax(&S->iters_done, m + 1);
     S->bnorm = bn;
@@ -1975,7 +1985,16 @@ __device__ unsigned long long g_res_prof[8];
 // resident at once; if they are not (other work on the device holds SMs), a waiting block
 // times out after ~2 ms, raises state->aborted and the stop flag, every block exits, and the
 // host continues the solve from the current iterate with per-launch kernels (R12).
-template <int WLR, bool LAZY = false>
+// Words of a tagged ring row each lane of warp 0 holds (k_block_resident<.., 2>): 8 (q <= 256) in
+// the 256 / 512-thread variants, 2 (q <= 64) in the 1024-thread ones (64 registers).
+__host__ __device__ constexpr int resident_pend(int wlr) { return wlr > 8 ? 8 : 2; }
+
+// LAZY: 0 blocking publication (iteration_publish), 1 ring + counter (release reduction),
+// 2 tagged ring words (q <= 32 resident_pend): a block's partial and its iteration tag in ONE relaxed 64-bit
+// store, so publishing needs no release fence (which waited for every write of the block,
+// x included, to reach L2: ~1 K cycles per iteration); warp 0 of the evaluating block loads the
+// q words one iteration ahead (<= 8 per lane) and votes on their tags.
+template <int WLR, int LAZY = 0>
 __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_block_resident(KP p) {
     extern __shared__ __align__(128) unsigned char smraw[];
     __shared__ double sred[2][32];
@@ -2047,6 +2066,26 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     unsigned int dv_ld = 0;
     if (LAZY && threadIdx.x == 0)
         asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.bsum_arr + blockIdx.x), "d"(bsum) : "memory");
+    // LAZY == 2: the launch's epoch, ||b|| from the x^(0) residual, the words of slot next_eval
+    const unsigned int ep = LAZY == 2 ? *(volatile unsigned int *)&p.state->epoch : 0u;
+    const double bnorm0 = LAZY == 2 ? *(volatile double *)&p.state->bnorm : 0.0;
+    auto tag_of = [&](long long mm) -> unsigned long long {
+        return ((unsigned long long)(ep & 0xFu) << 8) | ((unsigned long long)mm & 0xFFull);
+    };
+    constexpr int PEND = resident_pend(WLR);  // words per lane: q <= 32 PEND (registers)
+    unsigned long long pend[PEND];
+#pragma unroll
+    for (int j = 0; j < PEND; ++j) pend[j] = ~0ull;  // no tag matches
+    // thread 0's slow path (lead wait): are all q words of iteration mm's slot tagged mm?
+    auto tags_ready = [&](long long mm) -> bool {
+        const unsigned long long *row = reinterpret_cast<const unsigned long long *>(p.ring) + (mm % kSlots) * q;
+        for (int64_t c = 0; c < q; ++c) {
+            unsigned long long w;
+            asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w) : "l"(row + c) : "memory");
+            if ((w & 0xFFFull) != tag_of(mm)) return false;
+        }
+        return true;
+    };
     int cur = 0;
     // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
     // it before the launch: x^(0) already meets tol)
@@ -2056,17 +2095,25 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     BAR_PROF_DECL
     for (long long m = p.m0;;) {
         BAR_PROF_MARK(0)
+        bool tag_rdy = false;  // LAZY == 2: warp 0's vote on the words loaded one iteration ahead
+        if (LAZY == 2 && warp == 0) {
+            bool r = next_eval < m;
+#pragma unroll
+            for (int j = 0; j < PEND; ++j)
+                if (lane + 32 * j < q) r = r && (pend[j] & 0xFFFull) == tag_of(next_eval);
+            tag_rdy = __all_sync(0xffffffffu, r);
+        }
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
             // LAZY: this block's pending evaluation, if all q partials of that iteration are in
-            // (dv_ld: loaded one iteration ahead); evaluated by warp 0 after the barrier below
+            // (dv_ld / the tagged words: loaded one iteration ahead); evaluated by warp 0 after the
+            // barrier below
             if (LAZY) {
                 eval_m = -1;
-                if (next_eval < m && dv_ld == (unsigned int)q) {
-                    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+                if (next_eval < m && (LAZY == 2 ? tag_rdy : dv_ld == (unsigned int)q)) {
+                    if (LAZY == 1) asm volatile("fence.acq_rel.gpu;" ::: "memory");
                     eval_m = next_eval;
-                    next_eval += q;
                     dv_ld = 0;
                 }
             }
@@ -2089,10 +2136,11 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                             atomicExch(&p.state->stop, 1);
                             g = 0;
                         } else if (LAZY && next_eval < m &&
-                                   *(volatile unsigned int *)&p.state->done[next_eval % kSlots] == (unsigned int)q) {
-                            asm volatile("fence.acq_rel.gpu;" ::: "memory");
+                                   (LAZY == 2 ? tags_ready(next_eval)
+                                              : *(volatile unsigned int *)&p.state->done[next_eval % kSlots] ==
+                                                    (unsigned int)q)) {
+                            if (LAZY == 1) asm volatile("fence.acq_rel.gpu;" ::: "memory");
                             eval_m = next_eval;
-                            next_eval += q;
                             g = 2;
                             break;
                         }
@@ -2102,7 +2150,10 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             go = g;
         }
         __syncthreads();
-        if (LAZY && warp == 0 && eval_m >= 0) lazy_evaluate(p, eval_m, q, lane);
+        if (LAZY && eval_m >= 0) {  // every thread advances next_eval (warp 0 votes with it)
+            if (warp == 0) lazy_evaluate<LAZY == 2>(p, eval_m, q, lane, bnorm0);
+            next_eval = eval_m + q;
+        }
         if (!go) break;
         if (LAZY && go == 2) {  // evaluated for the waiting blocks; re-check the lead
             __syncthreads();
@@ -2159,7 +2210,13 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             const int W = blockDim.x >> 5;
             double a0 = 0.0;
             for (int w = 0; w < W; ++w) a0 += sred[0][w];
-            if (LAZY) {
+            if (LAZY == 2) {
+                const int slot = (int)(m % kSlots);
+                const unsigned long long w = ((unsigned long long)__double_as_longlong(a0) & ~0xFFFull) | tag_of(m);
+                asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p.ring + (int64_t)slot * q + blockIdx.x),
+                             "l"(w)
+                             : "memory");
+            } else if (LAZY) {
                 const int slot = (int)(m % kSlots);
                 asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.ring + (int64_t)slot * q + blockIdx.x),
                              "d"(a0)
@@ -2174,6 +2231,15 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             }
             stop_seen = stop_ld;
         }
+        if (LAZY == 2 && warp == 0 && next_eval <= m) {  // consumed at the next iteration's start
+            __syncwarp();  // thread 0's own word (just stored) is visible to the lane that loads it
+            const unsigned long long *row =
+                reinterpret_cast<const unsigned long long *>(p.ring) + (next_eval % kSlots) * q;
+#pragma unroll
+            for (int j = 0; j < PEND; ++j)
+                if (lane + 32 * j < q)
+                    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(pend[j]) : "l"(row + lane + 32 * j) : "memory");
+        }
         BAR_PROF_MARK(5)
         ++m;
     }
@@ -2184,7 +2250,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // runs the residual kernel instead), each block forms r_i = b_i - sum_j a_ij x_j for its rows
     // from the matrix entries it already holds (off-block x as written, x_J from shared memory),
     // and the last block sums the q partials in block order (own ticket and ring row 0, so a
-    // partial pass leaves the residual kernel's state untouched).
+    // partial pass leaves the residual kernel's state untouched; ring row kSlots).
     if (LAZY && p.fuse_residual) {
         __shared__ int fuse_go;
         if (threadIdx.x == 0) {
@@ -2229,7 +2295,8 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                 const int W = blockDim.x >> 5;
                 double a0 = 0.0;
                 for (int w = 0; w < W; ++w) a0 += sred[0][w];
-                asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.ring + blockIdx.x), "d"(a0) : "memory");
+                asm volatile("st.relaxed.gpu.global.f64 [%0], %1;" ::"l"(p.ring + kSlots * q + blockIdx.x), "d"(a0)
+                             : "memory");
                 unsigned int tk;
                 asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(tk) : "l"(&p.state->fuse_ticket) : "memory");
                 fuse_last = tk == (unsigned int)q - 1;
@@ -2239,7 +2306,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                 double s0 = 0.0, s1 = 0.0;
                 for (int64_t i = threadIdx.x; i < q; i += blockDim.x) {
                     double v0, v1;
-                    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v0) : "l"(p.ring + i) : "memory");
+                    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v0) : "l"(p.ring + kSlots * q + i) : "memory");
                     asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v1) : "l"(p.bsum_arr + i) : "memory");
                     s0 += v0;
                     s1 += v1;
@@ -2394,6 +2461,7 @@ __global__ void k_init_state(DevState *S, double tol) {
     S->fuse_arrive = 0;
     S->fuse_ticket = 0;
     S->exact_fused = 0;
+    S->epoch += 1;
     for (int i = 0; i < kSlots; ++i) {
         S->done[i] = 0;
         S->ss[i] = 0.0;
@@ -2622,12 +2690,15 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     KP pp = p;
     pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 48;
     pp.fuse_residual = p.ring && L.tune.lazy_publish >= 0 && L.tune.fuse_residual >= 0;
+    // tagged publication (LAZY = 2) while warp 0 can hold the q words, else the counter
     if (p.ring && L.tune.lazy_publish >= 0) {
-        if (ensure_smem(k_block_resident<WLR, true>, smem) != cudaSuccess) {
+        const bool tagged = L.q <= 32 * resident_pend(WLR) && L.tune.lazy_publish == 0;
+        auto kfn = tagged ? k_block_resident<WLR, 2> : k_block_resident<WLR, 1>;
+        if (ensure_smem(kfn, smem) != cudaSuccess) {
             cudaGetLastError();
             return false;
         }
-        k_block_resident<WLR, true><<<(unsigned)L.q, threads, smem, st>>>(pp);
+        kfn<<<(unsigned)L.q, threads, smem, st>>>(pp);
     } else {
         k_block_resident<WLR><<<(unsigned)L.q, threads, smem, st>>>(pp);
     }
@@ -2945,6 +3016,7 @@ __global__ void k_resume_queue(DevState *S, int clear_slots) {
         S->fuse_arrive = 0;
         S->fuse_ticket = 0;
         S->exact_fused = 0;
+        S->epoch += 1;
     }
 }
 
