@@ -1900,14 +1900,37 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     if (!MULTI) reduce_finalize<ASYNC ? kAsync : kSync>(rr, bb, p);
 }
 
+// The stopping rule of iteration m from its sum of r_i^2 (lazy / tagged publication).
+__device__ __forceinline__ void lazy_rule(DevState *S, long long m, double ss, double bn, double *hist) {
+    const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
+    atomicMax(&S->iters_done, m + 1);
+    S->bnorm = bn;
+    S->last_rel = rel;
+    if (hist) hist[m] = rel;
+    bool stop = false;
+    if (bn == 0.0) {
+        S->diverged = 2;
+        stop = true;
+    } else if (!isfinite(rel) || rel > 1e30) {
+        S->diverged = 1;
+        stop = true;
+    } else if (rel <= S->tol) {
+        // evaluations may complete out of order: the first iteration that met tol wins
+        atomicMin(reinterpret_cast<unsigned long long *>(&S->stop_iter), (unsigned long long)(m + 1));
+        stop = true;
+    }
+    if (stop) atomicExch(&S->stop, 1);
+}
+
 // k_block_resident<.., LAZY>: warp 0 of block m % q evaluates iteration m once all q partials are
-// in ring[m % kSlots] (thread 0 polls with relaxed loads, then an acquire fence before the CTA
-// barrier that hands the evaluation to the warp): fixed-order sums over the blocks (lane-strided,
-// then the shuffle tree), the stopping rule of iteration_publish, iters_done, and the slot's
-// counter reset for iteration m + kSlots.
-// TAGGED (q <= 256): the ring words carry the iteration and launch epoch in their 12 low mantissa
-// bits (the partial keeps 40 bits of mantissa, a relative 1e-12 of the estimate); they are summed
-// with the tag cleared, and ||b|| is the one the x^(0) residual stored before the launch.
+// in ring[m % kSlots] (LAZY = 1: thread 0 polls the slot's counter with relaxed loads, then an
+// acquire fence before the CTA barrier that hands the evaluation to the warp): fixed-order sums
+// over the blocks (lane-strided, then the shuffle tree), the stopping rule, iters_done, and the
+// slot's counter reset for iteration m + kSlots. TAGGED (LAZY = 2; this function only on the
+// lead-wait path, the regular evaluation sums the words warp 0 already holds): the ring words
+// carry the iteration and launch epoch in their 12 low mantissa bits (the partial keeps 40 bits of
+// mantissa, a relative 1e-12 of the estimate); they are summed with the tag cleared, and ||b|| is
+// the one the x^(0) residual stored before the launch.
 template <bool TAGGED>
 __device__ __noinline__ void lazy_evaluate(const KP &p, long long m, int64_t q, int lane, double bnorm0) {
     DevState *S = p.state;
@@ -1928,25 +1951,7 @@ __device__ __noinline__ void lazy_evaluate(const KP &p, long long m, int64_t q, 
     if (!TAGGED) bsq = warp_sum(bsq);
     if (lane != 0) return;
     if (!TAGGED) S->done[slot] = 0u;
-    const double bn = TAGGED ? bnorm0 : sqrt(bsq);
-    const double rel = bn != 0.0 ? sqrt(ss) / bn : 0.0;
-    atomicMax(&S->iters_done, m + 1);
-    S->bnorm = bn;
-    S->last_rel = rel;
-    if (p.hist) p.hist[m] = rel;
-    bool stop = false;
-    if (bn == 0.0) {
-        S->diverged = 2;
-        stop = true;
-    } else if (!isfinite(rel) || rel > 1e30) {
-        S->diverged = 1;
-        stop = true;
-    } else if (rel <= S->tol) {
-        // evaluations may complete out of order: the first iteration that met tol wins
-        atomicMin(reinterpret_cast<unsigned long long *>(&S->stop_iter), (unsigned long long)(m + 1));
-        stop = true;
-    }
-    if (stop) atomicExch(&S->stop, 1);
+    lazy_rule(S, m, ss, TAGGED ? bnorm0 : sqrt(bsq), p.hist);
 }
 
 // Phase timing of k_block_resident's thread 0 (a profiling build only: -DBAR_PROFILE_RESIDENT):
@@ -2095,14 +2100,6 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     BAR_PROF_DECL
     for (long long m = p.m0;;) {
         BAR_PROF_MARK(0)
-        bool tag_rdy = false;  // LAZY == 2: warp 0's vote on the words loaded one iteration ahead
-        if (LAZY == 2 && warp == 0) {
-            bool r = next_eval < m;
-#pragma unroll
-            for (int j = 0; j < PEND; ++j)
-                if (lane + 32 * j < q) r = r && (pend[j] & 0xFFFull) == tag_of(next_eval);
-            tag_rdy = __all_sync(0xffffffffu, r);
-        }
         if (threadIdx.x == 0) {
             // every block sweeps exactly max_global_iters = w_end / q times unless the solve stops
             int g = m < p.w_end / q && !stop_seen;
@@ -2111,7 +2108,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             // barrier below
             if (LAZY) {
                 eval_m = -1;
-                if (next_eval < m && (LAZY == 2 ? tag_rdy : dv_ld == (unsigned int)q)) {
+                if (LAZY == 1 && next_eval < m && dv_ld == (unsigned int)q) {
                     if (LAZY == 1) asm volatile("fence.acq_rel.gpu;" ::: "memory");
                     eval_m = next_eval;
                     dv_ld = 0;
@@ -2155,6 +2152,18 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
             next_eval = eval_m + q;
         }
         if (!go) break;
+        // LAZY == 2: warp 0 loads the words of iteration next_eval (already swept and published
+        // by this block) now and votes on them at the end of this iteration, so the other blocks
+        // have had this whole iteration to publish theirs
+        const bool pend_issued = LAZY == 2 && go == 1 && next_eval < m;
+        if (LAZY == 2 && warp == 0 && pend_issued) {
+            const unsigned long long *row =
+                reinterpret_cast<const unsigned long long *>(p.ring) + (next_eval % kSlots) * q;
+#pragma unroll
+            for (int j = 0; j < PEND; ++j)
+                if (lane + 32 * j < q)
+                    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(pend[j]) : "l"(row + lane + 32 * j) : "memory");
+        }
         if (LAZY && go == 2) {  // evaluated for the waiting blocks; re-check the lead
             __syncthreads();
             continue;
@@ -2206,6 +2215,21 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         if (lane == 0) sred[0][warp] = wr;
         __syncthreads();
         BAR_PROF_MARK(4)
+        if (LAZY == 2 && warp == 0 && pend_issued) {  // evaluate iteration next_eval if all q words are in
+            bool r = true;
+#pragma unroll
+            for (int j = 0; j < PEND; ++j)
+                if (lane + 32 * j < q) r = r && (pend[j] & 0xFFFull) == tag_of(next_eval);
+            if (__all_sync(0xffffffffu, r)) {
+                double ss = 0.0;
+#pragma unroll
+                for (int j = 0; j < PEND; ++j)
+                    if (lane + 32 * j < q) ss += __longlong_as_double((long long)(pend[j] & ~0xFFFull));
+                ss = warp_sum(ss);
+                if (lane == 0) lazy_rule(p.state, next_eval, ss, bnorm0, p.hist);
+                next_eval += q;  // warp 0 only: the other warps never read it in this variant
+            }
+        }
         if (threadIdx.x == 0) {
             const int W = blockDim.x >> 5;
             double a0 = 0.0;
@@ -2230,15 +2254,6 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                 iteration_publish(p, m, 1u, a0, bsum, q);
             }
             stop_seen = stop_ld;
-        }
-        if (LAZY == 2 && warp == 0 && next_eval <= m) {  // consumed at the next iteration's start
-            __syncwarp();  // thread 0's own word (just stored) is visible to the lane that loads it
-            const unsigned long long *row =
-                reinterpret_cast<const unsigned long long *>(p.ring) + (next_eval % kSlots) * q;
-#pragma unroll
-            for (int j = 0; j < PEND; ++j)
-                if (lane + 32 * j < q)
-                    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(pend[j]) : "l"(row + lane + 32 * j) : "memory");
         }
         BAR_PROF_MARK(5)
         ++m;
