@@ -752,6 +752,11 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 
 // Thread 0: the state reset leaves t_first = ~0, t_last = 0; every block of a single-launch
 // kernel lowers t_first at its start and raises t_last at its exit.
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *a) {
+    unsigned long long w;
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w) : "l"(a) : "memory");
+    return w;
+}
 __device__ __forceinline__ void stamp_first(DevState *S) { atomicMin(&S->t_first, globaltimer_ns()); }
 __device__ __forceinline__ void stamp_last(DevState *S) { atomicMax(&S->t_last, globaltimer_ns()); }
 
@@ -2082,14 +2087,18 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
 #pragma unroll
     for (int j = 0; j < PEND; ++j) pend[j] = ~0ull;  // no tag matches
     // thread 0's slow path (lead wait): are all q words of iteration mm's slot tagged mm?
-    auto tags_ready = [&](long long mm) -> bool {
+    auto tags_ready = [&](long long mm) -> bool {  // (batches of 8 loads in flight)
         const unsigned long long *row = reinterpret_cast<const unsigned long long *>(p.ring) + (mm % kSlots) * q;
-        for (int64_t c = 0; c < q; ++c) {
-            unsigned long long w;
-            asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w) : "l"(row + c) : "memory");
-            if ((w & 0xFFFull) != tag_of(mm)) return false;
+        bool all = true;
+        for (int64_t c0 = 0; c0 < q && all; c0 += 8) {
+            unsigned long long w[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                w[u] = c0 + u < q ? ld_relaxed_u64(row + c0 + u) : tag_of(mm);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) all = all && (w[u] & 0xFFFull) == tag_of(mm);
         }
-        return true;
+        return all;
     };
     int cur = 0;
     // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
