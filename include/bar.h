@@ -246,6 +246,9 @@ typedef struct {
                                loop                                                              */
     int32_t fuse_residual;  /* k_block_resident: 0 the confirming residual computed at the end of
                                the single launch (grid barrier), -1 a separate residual kernel    */
+    int32_t gather_ahead;   /* k_block_resident (rows of > 12 local entries, 256 threads): 0 the
+                               next iteration's off-block x loaded right after the write-back,
+                               -1 at the start of the sweep                                      */
 } bar_tuning;
 
 /* bar_set_tuning — replace the handle's tuning (NULL = defaults). Not thread-safe with a

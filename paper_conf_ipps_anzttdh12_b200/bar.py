@@ -73,7 +73,7 @@ class Tuning(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int32) for f in (
         "kernel", "duo", "pipe", "coded", "async_order", "async_queue", "resident", "lead", "ghost_prefetch", "graph",
         "single_launch", "jacobi_rowwise", "grid_cap", "warps", "halo", "peer", "fronts",
-        "stage_bx", "lazy_publish", "slab_prefetch", "overlap", "unroll_off", "fuse_residual")]
+        "stage_bx", "lazy_publish", "slab_prefetch", "overlap", "unroll_off", "fuse_residual", "gather_ahead")]
 
     KERNELS = {"auto": 0, "block": 1, "reg": 2, "reg_tma": 3, "pers": 4}
     ORDERS = {"auto": 0, "chunks": 1, "round_robin": 2, "fronts": 3}

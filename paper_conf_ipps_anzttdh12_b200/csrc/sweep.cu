@@ -63,6 +63,7 @@ struct KP {
     const int *stop;        // the stop flag the kernels poll at start (default &state->stop)
     int slab_ahead;         // k_block_duo: L2 bulk prefetch of the slab two subdomains ahead
     int fuse_residual;      // k_block_resident<LAZY>: exact residual of the final x at the end of the launch
+    int gather_ahead;       // k_block_resident (256-thread variants): next iteration's gathers issued after the write-back
     double *ring;           // k_block_resident<LAZY>: [kSlots][q] per-block residual partials
     double *bsum_arr;       //   and [q] per-block sums of b_i^2
     const uint8_t *codes;   // coded layout (Layout::codes): per entry, index into its subdomain's
@@ -2101,6 +2102,20 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         return all;
     };
     int cur = 0;
+    // Gathers one iteration ahead (the 256-thread variants have the registers): a row's off-block
+    // x values for iteration m + 1 are loaded right after its write-back of iteration m — x "as
+    // it stands" a few hundred cycles earlier than at the next sweep, which eq. 3 allows — so their
+    // L2 latency overlaps the residual publication and the next iteration's start instead of
+    // opening the sweep
+    constexpr int GPRE = WLR > 12 ? 16 : 0;
+    const bool pre = GPRE > 0 && p.gather_ahead && wo <= GPRE;
+    double xg[GPRE > 0 ? GPRE : 1];
+    auto issue_gathers = [&]() {
+#pragma unroll
+        for (int e = 0; e < GPRE; ++e)
+            if (e < wo) xg[e] = ldx<true>(p.x_in + oc[ooff + e * kSlice]);
+    };
+    if (pre && ok) issue_gathers();
     // thread 0: the stop flag, loaded one iteration ahead of its use (k_init_check may have raised
     // it before the launch: x^(0) already meets tol)
     int stop_seen = threadIdx.x == 0 ? *(volatile int *)&p.state->stop : 0, stop_ld = 0;
@@ -2186,7 +2201,11 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         const double *y0 = ybuf(cur);
         double *y1 = ybuf(cur ^ 1);
         double s = bi, rr = 0.0;
-        if (ok) {
+        if (ok && pre) {  // a3 from the values gathered one iteration ahead
+#pragma unroll
+            for (int e = 0; e < GPRE; ++e)
+                if (e < wo) s -= ov[ooff + e * kSlice] * xg[e];
+        } else if (ok) {
             // a3: off-block part, x as it stands
             for (int e0 = 0; e0 < wo; e0 += 2 * U) {
                 double xv[2 * U];
@@ -2197,6 +2216,8 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
                 for (int u = 0; u < 2 * U; ++u)
                     if (e0 + u < wo) s -= ov[ooff + (e0 + u) * kSlice] * xv[u];
             }
+        }
+        if (ok) {
             // first local sweep in the correction form: its numerator is r_i (a5)
             double acc = s;
 #pragma unroll
@@ -2220,6 +2241,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         BAR_PROF_MARK(3)
         cur ^= p.k & 1;
         if (ok) stx<true>(p.x_out + TS + loc, ybuf(cur)[loc]);  // a6
+        if (pre && ok) issue_gathers();  // for the next iteration
         const double wr = warp_sum(rr);
         if (lane == 0) sred[0][warp] = wr;
         __syncthreads();
@@ -2714,6 +2736,7 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     KP pp = p;
     pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 48;
     pp.fuse_residual = p.ring && L.tune.lazy_publish >= 0 && L.tune.fuse_residual >= 0;
+    pp.gather_ahead = L.tune.gather_ahead >= 0;
     // tagged publication (LAZY = 2) while warp 0 can hold the q words, else the counter
     if (p.ring && L.tune.lazy_publish >= 0) {
         const bool tagged = L.q <= 32 * resident_pend(WLR) && L.tune.lazy_publish == 0;
