@@ -342,6 +342,9 @@ bar_status bar_sweep(bar_matrix A, const double *b, double *x, int32_t k, int64_
         a.ring = A->W.ring;
         a.bsum_arr = A->W.bsum_arr;
         if (use_async_multi(A->L)) {
+            // ||b|| for the single launch's residual estimates (the tagged publication reads the
+            // one the x^(0) residual stores; bar_sweep has none otherwise)
+            BAR_CUDA(launch_zero_start_residual(A->L, b, A->W.state, A->W.partials, st));
             cudaError_t e = launch_async_multi(a, (long long)nsweeps * A->L.q, st);
             if (e == cudaSuccess) return BAR_OK;
             if (e != cudaErrorNotSupported) return cuda_fail(e, "launch_async_multi");

@@ -356,8 +356,8 @@ def test_bar_sweep_async_does_the_work(bar, name, R, single):
         rr = O.rel_res(A, b, xd.cpu().numpy())
         ref = O.solve(A, b, method=O.BLOCK_JACOBI, R=R, k=5, tol=0.0, max_iters=nsw).rel_res
         assert rr <= 30 * ref, (nsw, rr, ref)
-        if prev is not None:
-            assert rr < prev
+        if prev is not None:  # 8 more global iterations (each contracts by well under 0.75 here)
+            assert rr < 0.1 * prev, (rr, prev)
         prev = rr
     M.close()
 
