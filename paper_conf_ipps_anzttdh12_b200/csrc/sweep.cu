@@ -18,6 +18,7 @@
 // Every kernel is HBM-bound (about 0.17 flop/byte): no tensor cores. Matrix entries are read
 // with coalesced warp-wide loads from the sliced layout (bar_internal.cuh).
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <map>
 #include <mutex>
@@ -122,6 +123,31 @@ __device__ __forceinline__ double ext_update(double xold, double v, bool frozen,
     if (frozen) return xold;
     return tau == 1.0 ? v : xold + tau * (v - xold);
 }
+
+// Bounds checks of a checking build only (-DBAR_CHECK_BOUNDS -> libbar_check.so, tools/build.py
+// --check-bounds): shared-memory reads against the launch's dynamic allocation and the ring /
+// tag indices of the single-launch kernel; a failed check prints the site and traps. (The pool's
+// compute-sanitizer was closed during round 2; this build stands in for its memcheck on the
+// kernel paths added since the last sanitizer run.)
+#ifdef BAR_CHECK_BOUNDS
+__device__ __forceinline__ uint32_t dyn_smem_bytes() {
+    uint32_t v;
+    asm volatile("mov.u32 %0, %%dynamic_smem_size;" : "=r"(v));
+    return v;
+}
+#define BAR_CHECK(cond, what)                                                                          \
+    do {                                                                                               \
+        if (!(cond)) {                                                                                 \
+            printf("BAR_CHECK failed: %s (block %d thread %d, line %d)\n", what, (int)blockIdx.x,     \
+                   (int)threadIdx.x, __LINE__);                                                        \
+            __trap();                                                                                  \
+        }                                                                                              \
+    } while (0)
+#else
+#define BAR_CHECK(cond, what) \
+    do {                      \
+    } while (0)
+#endif
 
 enum Kind { kSync = 0, kAsync = 1, kResidual = 2 };
 
@@ -1327,6 +1353,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
                 const uint32_t off = v ? (uint32_t)(ssp[sl] - ssp[0]) + lane : 0u;
                 av[h] = sb + off * 8;
                 ac[h] = sb + g.o_col + off;
+                BAR_CHECK(!v || (off + (uint32_t)(wo[h] + wl[h] - 1) * kSlice + 1) * 8 <= g.o_col, "duo slab values");
+                BAR_CHECK(!v || off + (uint32_t)(wo[h] + wl[h] - 1) * kSlice + 1 <= g.o_dict - g.o_col, "duo slab codes");
                 const double *xr = p.x_in + (TS + loc);
 #pragma unroll
                 for (int e = 0; e < WOR; ++e)
@@ -1341,6 +1369,8 @@ __global__ void __launch_bounds__(512, 2) k_block_duo(KP p) {
 #pragma unroll
                 for (int e = 0; e < WLR; ++e) {
                     const bool ok = e < wl[h];
+                    BAR_CHECK(av[h] + (uint32_t)(wo[h] + e) * kSlice * 8 + 8 - sb <= dyn_smem_bytes(), "duo local value read");
+                    BAR_CHECK(ac[h] + (uint32_t)(wo[h] + e) * kSlice + 1 - sb <= dyn_smem_bytes(), "duo local code read");
                     const double v = lds_f64(av[h] + (wo[h] + e) * kSlice * 8);
                     const uint32_t c = (uint32_t)(loc + lds_s32(ad + 4 * lds_u8(ac[h] + (wo[h] + e) * kSlice))) & 0xffffu;
                     lv[h][e] = ok ? v : 0.0;
@@ -2090,6 +2120,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
     // thread 0's slow path (lead wait): are all q words of iteration mm's slot tagged mm?
     auto tags_ready = [&](long long mm) -> bool {  // (batches of 8 loads in flight)
         const unsigned long long *row = reinterpret_cast<const unsigned long long *>(p.ring) + (mm % kSlots) * q;
+        BAR_CHECK(mm >= 0, "tags_ready iteration");
         bool all = true;
         for (int64_t c0 = 0; c0 < q && all; c0 += 8) {
             unsigned long long w[8];
@@ -2180,6 +2211,7 @@ __global__ void __launch_bounds__(WLR > 12 ? 256 : (WLR > 8 ? 512 : 1024), 1) k_
         // by this block) now and votes on them at the end of this iteration, so the other blocks
         // have had this whole iteration to publish theirs
         const bool pend_issued = LAZY == 2 && go == 1 && next_eval < m;
+        BAR_CHECK(!pend_issued || (next_eval >= 0 && q <= 32 * PEND), "tagged pending words");
         if (LAZY == 2 && warp == 0 && pend_issued) {
             const unsigned long long *row =
                 reinterpret_cast<const unsigned long long *>(p.ring) + (next_eval % kSlots) * q;

@@ -125,6 +125,8 @@ if __name__ == "__main__":
         build_bar(True, "libbar_prof.so", ("BAR_PROFILE_RESIDENT=1",))
     elif "--profile-duo" in sys.argv:
         build_bar(True, "libbar_duoprof.so", ("BAR_PROFILE_DUO=1",))
+    elif "--check-bounds" in sys.argv:
+        build_bar(True, "libbar_check.so", ("BAR_CHECK_BOUNDS=1",))
 
     else:
         build_all(force="--force" in sys.argv)
