@@ -51,3 +51,24 @@ def test_our_arm_line(bar):
     e = d["e2e"]
     assert e["h2d_bytes_per_step"] == 8 * 2000 and e["d2h_bytes_per_step"] == 8 * 2000 and e["value"] > 0
     assert d["clocks"]["sm_max_mhz"]
+
+
+def test_ncu_kernel_names_map_to_libbar_names():
+    """tools/ncu_summary.libbar_name: ncu's demangled k_block_duo template arguments -> the name
+    libbar reports (bar_matrix_info.last_sweep_kernel), which bench.py matches against the kernel
+    stamped into profiles/traffic_*.json (a capture of another kernel variant is never used)."""
+    import sys
+
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    from ncu_summary import libbar_name
+
+    base = "void bar::<unnamed>::k_block_duo<{}>(bar::<unnamed>::KP)"
+    assert libbar_name(base.format("(bool)1, (int)4, (bool)0, (int)1, (bool)1, (int)4")) == "k_block_duo<async,coded,wo4,bx>"
+    assert libbar_name(base.format("(bool)1, (int)4, (bool)0, (int)1, (bool)0, (int)0")) == "k_block_duo<async,coded>"
+    assert libbar_name(base.format("(bool)0, (int)4, (bool)0, (int)1, (bool)1")) == "k_block_duo<sync,coded,bx>"
+    assert libbar_name(base.format("(bool)1, (int)4, (bool)1, (int)2")) == "k_block_duo<async,staged>"
+    assert libbar_name("void bar::<unnamed>::k_block_resident<16, 2>(bar::<unnamed>::KP)").startswith("void bar")
+    # the committed captures name a kernel variant libbar can report
+    for wl in ("c4", "c5"):
+        tj = json.load(open(os.path.join(ROOT, "profiles", f"traffic_{wl}_async.json")))
+        assert tj["kernel"].startswith("k_block_duo<async,coded") and tj["dram_bytes_per_launch"] > 0
