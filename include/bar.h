@@ -232,10 +232,11 @@ typedef struct {
     int32_t fronts;         /* async_order = 3: number of fronts (0 = 8)                          */
     int32_t stage_bx;       /* k_block_duo: 0 stage b_J and x_J with the slab (bulk copies) where
                                that keeps the blocks per SM, -1 per-row loads                    */
-    int32_t lazy_publish;   /* k_block_resident: 0 non-blocking residual publication — up to 256
-                               blocks a tagged word per block (partial + iteration in one relaxed
-                               store), else a ring of partials + a release counter; 1 always the
-                               counter; -1 one blocking atomic per block and iteration           */
+    int32_t lazy_publish;   /* k_block_resident: 0 non-blocking residual publication — a tagged
+                               word per block (partial + iteration in one relaxed store) in the
+                               256-thread variant up to 256 blocks, else a ring of partials + a
+                               release counter; 1 always the counter; 2 tagged wherever warp 0 can
+                               hold the words; -1 one blocking atomic per block and iteration     */
     int32_t slab_prefetch;  /* k_block_duo: 1 L2 bulk prefetch of the slab two subdomains ahead
                                (a second slab buffer in L2), 0 off                               */
     int32_t overlap;        /* multi-GPU collective path: 0 sweep the interior subdomains (no ghost

@@ -249,7 +249,7 @@ bar_status bar_set_tuning(bar_matrix A, const bar_tuning *tuning) {
     if (t.kernel < 0 || t.kernel > 4 || t.async_order < 0 || t.async_order > 3 || t.fronts < 0 || t.async_queue < 0 ||
         t.async_queue > 1 || t.lead < 0 || t.lead > 48 || t.grid_cap < 0 || t.warps < 0 || t.warps > 32 ||
         t.halo < 0 || t.halo > 1 || t.peer > 0 || t.coded > 2 || t.overlap > 0 || t.unroll_off > 0 ||
-        t.fuse_residual > 0 || t.lazy_publish > 1 || t.gather_ahead > 0) {
+        t.fuse_residual > 0 || t.lazy_publish > 2 || t.gather_ahead > 0) {
         set_error("bar_tuning field out of range");
         return BAR_ERR_INVALID_ARG;
     }

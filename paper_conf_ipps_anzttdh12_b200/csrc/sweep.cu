@@ -2769,9 +2769,14 @@ bool launch_resident_t(const KP &p, const Layout &L, cudaStream_t st, cudaError_
     pp.lead = L.tune.lead > 0 ? std::min(48, L.tune.lead) : 48;
     pp.fuse_residual = p.ring && L.tune.lazy_publish >= 0 && L.tune.fuse_residual >= 0;
     pp.gather_ahead = L.tune.gather_ahead >= 0;
-    // tagged publication (LAZY = 2) while warp 0 can hold the q words, else the counter
+    // tagged publication (LAZY = 2) while warp 0 can hold the q words, by default in the
+    // 256-thread variants (rows with > 12 local entries): there it is faster (C1 0.104 vs 0.122 ms,
+    // C3 0.161 vs 0.172); in the 512-thread variant of C2 it was not (0.209 vs 0.202 ms) and cost
+    // iterations (56-57 vs 53-54: without the counter's release fence the x stores of an iteration
+    // are not drained before the next sweep), so the others keep the counter unless lazy_publish = 2
     if (p.ring && L.tune.lazy_publish >= 0) {
-        const bool tagged = L.q <= 32 * resident_pend(WLR) && L.tune.lazy_publish == 0;
+        const bool tagged = L.q <= 32 * resident_pend(WLR) &&
+                            (L.tune.lazy_publish == 2 || (L.tune.lazy_publish == 0 && WLR > 12));
         auto kfn = tagged ? k_block_resident<WLR, 2> : k_block_resident<WLR, 1>;
         if (ensure_smem(kfn, smem) != cudaSuccess) {
             cudaGetLastError();

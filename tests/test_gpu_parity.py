@@ -377,12 +377,16 @@ def test_siam_constant_async(bar, golden):
 @pytest.mark.parametrize("tune", [{"kernel": "block"}, {"kernel": "reg"}, {"kernel": "reg_tma"}, {"kernel": "pers"},
                                   {"pipe": 1}, {"pipe": -1}, {"jacobi_rowwise": 1}, {"single_launch": 1},
                                   {"single_launch": -1}, {"ghost_prefetch": -1}, {"ghost_prefetch": 1},
-                                  {"async_queue": "queue"}, {"resident": -1}, {"lead": 3}, {"graph": -1}])
+                                  {"async_queue": "queue"}, {"resident": -1}, {"lead": 3}, {"graph": -1},
+                                  {"lazy_publish": 1}, {"lazy_publish": 2}, {"lazy_publish": -1},
+                                  {"gather_ahead": -1}, {"fuse_residual": -1}])
 @pytest.mark.parametrize("name,R", [("fv1", 128), ("s7_m12", 288), ("tref2000", 128), ("s7_m12", 512),
                                     ("rand", 1024)])
 def test_forced_kernel_paths(bar, tune, name, R):
     """Each kernel the dispatcher can choose (fallbacks included, forced through the handle's
-    bar_tuning) gives the oracle's iterates in the sync modes and converges in async."""
+    bar_tuning; for the single-launch kernel each residual-publication scheme, the gathers at the
+    sweep's start and the separate confirming residual) gives the oracle's iterates in the sync
+    modes and converges in async."""
     A = MATS[name]()
     b = np.ones(A.n)
     x0 = np.random.default_rng(2).uniform(-1, 1, A.n)
